@@ -1,0 +1,372 @@
+#!/usr/bin/env python
+"""Checkpoint-pair compare throughput (build + diff + verify) on B200.
+
+Metric (BASELINE.json): checkpoint-pair compare GB/s (build+diff+verify) at
+1/2/4/8 B200, % HBM peak.  One step = the whole hot path on one pair of
+checkpoints resident in HBM:
+    tree_build(run A) + tree_build(run B) + tree_diff + verify
+    (+ for N>1: NCCL all-gather of array roots -> top tree, all-reduce of counts)
+GB/s = (bytes(A) + bytes(B)) summed over all ranks / step time (max over ranks).
+
+Workload at N=1: BASELINE configs[1] -- HACC-shaped checkpoint, 2^26 particles
+x 6 float32 arrays (x,y,z ~ U[0,256), v ~ N(0,300^2)) per GPU, 4 KiB chunks,
+eps = 1e-6, 1% of particles perturbed in 64 clusters.  N>1: every rank holds its
+own such checkpoint pair (weak scaling, arrays sharded by rank as HACC writes
+per-rank checkpoints).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "checkpoint-pair compare GB/s (build+diff+verify) at 1/2/4/8 B200, % HBM peak"
+N_PARTICLES = 1 << 26
+CHUNK = 4096
+EPS = 1e-6
+SEED = 2
+WORKLOAD = ("configs[1]: HACC-shaped checkpoint pair, 2^26 particles x 6 float32 per GPU, "
+            "4 KiB chunks, eps=1e-6, 1% particles perturbed in 64 clusters")
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.dev}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.06)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.thread.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def host_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+# ---------------------------------------------------------------------------
+# oracle (CPU) legs: cpu_baseline and --impl reference
+# ---------------------------------------------------------------------------
+
+def oracle_pair_sample(n_particles: int, seed: int):
+    import synth
+    pair = synth.c2_pair(n_particles=n_particles, seed=seed, device="cpu")
+    return [t.numpy() for t in pair.a], [t.numpy() for t in pair.b]
+
+
+def oracle_step(a_list, b_list, threads: int):
+    """The oracle as it stands: build A, build B, BFS diff, verify (all arrays)."""
+    import oracle
+    A = oracle.build_checkpoint(a_list, CHUNK, EPS, threads=threads)
+    B = oracle.build_checkpoint(b_list, CHUNK, EPS, threads=threads)
+    ch = oracle.diff_checkpoint(A, B)
+    idx = oracle.verify_checkpoint(a_list, b_list, CHUNK, ch, EPS, A)
+    return ch.size, idx.size
+
+
+def calibrate_oracle(target_s: float, threads: int):
+    """Particles per sample so one oracle step takes about target_s seconds."""
+    n = 1 << 14
+    while True:
+        a, b = oracle_pair_sample(n, SEED)
+        t0 = time.perf_counter()
+        oracle_step(a, b, threads)
+        dt = time.perf_counter() - t0
+        if dt > 0.3 or n >= N_PARTICLES:
+            break
+        n *= 4
+    scale = target_s / max(dt, 1e-6)
+    n = int(min(N_PARTICLES, max(1 << 12, n * scale)))
+    n = max(1024, (n // 1024) * 1024)
+    return n
+
+
+def cpu_baseline(target_s: float = 12.0):
+    import oracle
+    oracle.build()
+    threads = host_cores()
+    n = calibrate_oracle(target_s, threads)
+    a, b = oracle_pair_sample(n, SEED)
+    t0 = time.perf_counter()
+    oracle_step(a, b, threads)
+    dt = time.perf_counter() - t0
+    nbytes = 2 * sum(x.nbytes for x in a)
+    return {"value": round(nbytes / dt / 1e9, 4), "unit": "GB/s", "cores": threads,
+            "kind": "oracle",
+            "sample": f"same recipe at {n} particles x 6 f32 per run ({nbytes / 1e6:.1f} MB pair), "
+                      f"one full step (build A+B, BFS diff, verify) in {dt:.2f} s"}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    threads = host_cores()
+    budget = 150.0
+    per_step = min(2.0, budget / max(1, args.steps + args.warmup))
+    n = calibrate_oracle(per_step, threads)
+    a, b = oracle_pair_sample(n, SEED)
+    nbytes = 2 * sum(x.nbytes for x in a)
+    for _ in range(args.warmup):
+        oracle_step(a, b, threads)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle_step(a, b, threads)
+    dt = (time.perf_counter() - t0) / max(1, args.steps)
+    value = nbytes / dt / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64 (quantizer/predicate), u64 hash", "data": "synthetic",
+        "config": {"workload": WORKLOAD + f" (bounded sample: {n} particles per run per step)",
+                   "chunk_bytes": CHUNK, "eps": EPS, "parallelism": "host threads"},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": threads,
+                         "kind": "oracle",
+                         "sample": f"{n} particles x 6 f32 per run ({nbytes / 1e6:.1f} MB pair) per step"},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------------------
+# our arm
+# ---------------------------------------------------------------------------
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    group = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_middleware_tanaabcrtn24_b200 as ck
+    from paper_conf_middleware_tanaabcrtn24_b200 import dist as ckd
+    import synth
+
+    ck.lib()
+    pair = synth.c2_pair(n_particles=N_PARTICLES, seed=SEED + 1000 * rank, device="cuda")
+    A, B = pair.a, pair.b
+    bytes_pair = 2 * pair.nbytes
+    n_elems = sum(t.numel() for t in A)
+    L = sum(t.numel() * 4 // CHUNK for t in A)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(n_elems, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    n_arrays = len(A)
+    gathered = torch.empty((world * n_arrays, 16), dtype=torch.uint8, device="cuda")
+    keep = []
+
+    def step():
+        TA = ck.tree_build(A, CHUNK, EPS)
+        TB = ck.tree_build(B, CHUNK, EPS)
+        ck.tree_diff_async(TA, TB, chunks, counts[0:1])
+        ck.verify_async(A, B, chunks, counts[0:1], CHUNK, EPS, idx, counts[1:2])
+        if world > 1:
+            tops = []
+            for T in (TA, TB):
+                dist.all_gather_into_tensor(gathered.view(-1), T.array_roots().view(-1))
+                tops.append(ck.tree_from_digests(gathered))
+            tot = counts.clone()
+            dist.all_reduce(tot)
+            keep[:] = [TA, TB, *tops, tot]
+        else:
+            keep[:] = [TA, TB]
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    local_counts = counts.cpu().tolist()
+
+    # timed region
+    sampler = ClockSampler(torch.cuda.current_device())
+    sampler.start()
+    time.sleep(0.2)
+    ck.profile_reset()
+    ck.profile_enable(True)
+    l0 = ck.launch_count()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(args.steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    launches = ck.launch_count() - l0
+    ck.profile_enable(False)
+    clocks = sampler.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.barrier()
+    ms_max = float(t.item())
+    phases = {}
+    for k in ("leaf", "levels", "diff", "verify"):
+        pms, pn = ck.profile_read(k)
+        phases[k] = {"ms_per_step": round(pms / args.steps, 4), "launches": pn}
+    leaf_ms, leaf_n = ck.profile_read("leaf")
+    ck.profile_reset()
+    leaf_avg_s = leaf_ms / max(1, leaf_n) / 1e3
+    leaf_bytes = pair.nbytes + 16 * L        # algorithmic: read S, write L leaves
+    peak, peak_src = peaks()
+    achieved = leaf_bytes / leaf_avg_s / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "leaf_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    value = bytes_pair * world / (ms_max / 1e3) / 1e9
+
+    # end-to-end through the public API with host buffers (pinned), H2D+D2H inside
+    e2e = None
+    if not args.no_e2e:
+        ha = [x.cpu().pin_memory() for x in A]
+        hb = [x.cpu().pin_memory() for x in B]
+        k_e2e = max(3, min(args.steps, 8))
+        out = ck.compare_host(ha, hb, CHUNK, EPS)    # warm-up
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(k_e2e):
+            out = ck.compare_host(ha, hb, CHUNK, EPS)
+        dt = (time.perf_counter() - t0) / k_e2e
+        tt = torch.tensor([dt], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        dt = float(tt.item())
+        n_diff = out[2]
+        e2e = {"value": round(bytes_pair * world / dt / 1e9, 3), "unit": "GB/s",
+               "h2d_bytes_per_step": bytes_pair,
+               "d2h_bytes_per_step": 8 * n_diff + 16 + 32, "steps": k_e2e,
+               "api": "ckpt_compare_host (pinned host arrays)"}
+        del ha, hb
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline()
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": round(ms_max, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32 in, f64 quantize/compare, u64 hash",
+            "data": "synthetic (seeded HACC-shaped arrays, synth.c2_pair)",
+            "config": {"workload": WORKLOAD, "particles_per_gpu": N_PARTICLES, "arrays_per_run": 6,
+                       "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair,
+                       "l2": "inputs larger than L2 (3.2 GB per GPU per step >> 126 MB)",
+                       "parallelism": f"dp{world} (checkpoint arrays sharded by rank)"},
+            "pct_hbm_peak": round(value / (world * peak), 4),
+            "roofline": {"bound": "hbm", "kernel": "leaf_kernel (K1: quantize + chained Murmur3F)",
+                         "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "peak_source": peak_src,
+                         "algorithmic_bytes_per_launch": leaf_bytes,
+                         "avg_launch_ms": round(leaf_avg_s * 1e3, 4)},
+            "phases": phases,
+            "flagged_chunks_per_gpu": local_counts[0], "diff_elems_per_gpu": local_counts[1],
+            "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

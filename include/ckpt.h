@@ -1,0 +1,254 @@
+/*
+ * ckpt.h -- C ABI of libckpt.so, the B200 (sm_100a) hot path of
+ *   Tan et al., "Towards Affordable Reproducibility Using Scalable Capture
+ *   and Comparison of Intermediate Multi-Run Results", MIDDLEWARE '24.
+ *   ("P:<line>" = line of /root/reference/PAPER.md; "R<k>" = a reading in
+ *   DESIGN.md section "Readings of the paper".)
+ *
+ * Problem: given the checkpoints of two runs, list every datum
+ * (with its index) whose values differ by more than a user bound eps,
+ * |V_A - V_B| > eps.  The method (Alg. 1):
+ *   1. split each checkpoint array into fixed-size chunks, conservatively
+ *      round every float to the bound and hash each chunk with block-chained
+ *      128-bit Murmur3F into a Merkle leaf              -> ckpt_tree_build*
+ *   2. build the Merkle tree level by level               -> ckpt_tree_build*
+ *   3. BFS both trees top-down from a mid level, pruning equal subtrees,
+ *      to list the chunks whose leaves differ            -> ckpt_tree_diff*
+ *   4. compare only those chunks element by element      -> ckpt_verify*
+ *
+ * Conventions for every entry point
+ * ---------------------------------
+ *  - Pointers are CUDA DEVICE pointers of the device that is current on
+ *    the calling thread, unless the parameter is marked (host).
+ *  - `stream` is a cudaStream_t (NULL = legacy default stream).  All device
+ *    work is enqueued on it.  Functions that return a count through a
+ *    (host) pointer synchronise `stream` before returning; functions named
+ *    *_async never synchronise.
+ *  - Input arrays are borrowed: caller-owned, unmodified, and they must stay
+ *    valid until the enqueued work completes.  Data pointers must be 16-byte
+ *    aligned (the leaf kernel moves 16-byte blocks).
+ *  - Trees are library-owned (opaque); release with ckpt_tree_free*.
+ *  - Output buffers are caller-allocated with capacity `cap` entries.  When
+ *    the full count exceeds `cap`, the first `cap` entries (ascending) are
+ *    written, the full count is still returned and the status is
+ *    CKPT_ETRUNC.
+ *  - Outputs are unique, ascending, 0-based ids (R17).  For a checkpoint of
+ *    several arrays, ids are global: array a's chunk c is
+ *    chunk_base[a] + c and its element i is elem_base[a] + i, where the
+ *    bases are the running sums of the arrays' chunk / element counts in
+ *    array order.
+ *  - Errors never abort the process.  CKPT_ECUDA carries the CUDA error
+ *    text, retrievable with ckpt_last_error() (thread-local).
+ *  - There is no CPU fallback: without a usable sm_100 device every
+ *    compute entry point returns CKPT_ECUDA.
+ */
+#ifndef CKPT_H
+#define CKPT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    CKPT_OK = 0,
+    CKPT_EINVAL = -1,    /* bad argument (see each function) */
+    CKPT_EMISMATCH = -2, /* trees not built with the same shape / parameters (R19) */
+    CKPT_ENOMEM = -3,    /* device allocation failed */
+    CKPT_ECUDA = -4,     /* CUDA runtime / launch error */
+    CKPT_ETRUNC = -5     /* output longer than `cap`; first `cap` entries valid */
+} ckpt_status;
+
+typedef enum { CKPT_F32 = 0, CKPT_F64 = 1 } ckpt_dtype;  /* HACC fields are F32 */
+
+typedef struct ckpt_tree ckpt_tree;
+
+/* ------------------------------------------------------------------------
+ * Step 1+2: capture-time tree construction (Alg. 1; P:463-474;
+ * section 2.4).
+ *
+ * Chunking (R12): chunk c of an array covers input bytes
+ * [c*chunk_bytes, min(nbytes, (c+1)*chunk_bytes)); chunk_bytes must be a
+ * positive multiple of 16 (one 128-bit hash block).
+ * Rounding (R5-R9): inv = RN(1/eps); every element x becomes
+ * k = clamp(floor(x * inv)) (exact product; NaN -> 0); the hashed word is
+ * k's low 32 bits for F32 and all 64 bits for F64.  eps == 0 hashes the raw
+ * element bits (R10).
+ * Leaf (R2-R4): (h1,h2) = (0,0); for every 16-byte block of
+ * words, (h1,h2) = MurmurHash3_x64_128(block, len, state (h1,h2)); a final
+ * block shorter than 16 bytes uses Murmur3F's tail.  leaf = h1 || h2.
+ * Levels (R13-R14): n_{l+1} = ceil(n_l/2); node = Murmur3F(left
+ * || right, 32 bytes, seed 0) or the left child promoted when it has no
+ * sibling.
+ * Checkpoint of several arrays (R15): every array gets its own tree; the
+ * checkpoint root is the same level construction over the array roots in
+ * array order.
+ *
+ * Arguments:
+ *   data        device pointer to n elements of `dtype`, little-endian,
+ *               16-byte aligned.
+ *   n           element count, >= 1.
+ *   eps         absolute bound, finite and >= 0.
+ *   out (host)  receives the new tree.
+ * The build is asynchronous on `stream`; the tree may be used by later
+ * work on the same stream (or after synchronising it).
+ * Errors: CKPT_EINVAL for n == 0, NULL pointers, misaligned data,
+ * chunk_bytes == 0 or not a multiple of 16, eps < 0 / NaN / inf, unknown
+ * dtype; CKPT_ENOMEM; CKPT_ECUDA.
+ * ---------------------------------------------------------------------- */
+ckpt_status ckpt_tree_build(const void *data, uint64_t n, ckpt_dtype dtype, uint32_t chunk_bytes,
+                            double eps, void *stream, ckpt_tree **out);
+
+/* Same for a checkpoint made of n_arrays >= 1 arrays (e.g. the six HACC
+ * particle fields of one rank).  data (host) and n (host) are arrays of
+ * n_arrays device pointers / element counts.  All arrays are hashed in one
+ * leaf-kernel launch. */
+ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n, uint32_t n_arrays,
+                                   ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                   void *stream, ckpt_tree **out);
+
+/* Tree over caller-supplied 16-byte digests used as leaves (no data
+ * hashing).  Used to form the top levels over the subtree roots gathered
+ * from all GPUs (R15; the multi-GPU path).  digests16: device, count*16
+ * bytes.  The result supports ckpt_tree_root / ckpt_tree_nodes only. */
+ckpt_status ckpt_tree_from_digests(const void *digests16, uint64_t count, void *stream,
+                                   ckpt_tree **out);
+
+/* Release a tree.  ckpt_tree_free orders the release after the work on the
+ * tree's build stream (which must still exist); ckpt_tree_free_on orders it
+ * on `stream` instead.  NULL is ignored. */
+void ckpt_tree_free(ckpt_tree *t);
+void ckpt_tree_free_on(ckpt_tree *t, void *stream);
+
+/* ------------------------------------------------------------------------
+ * Step 3: stage-1 comparison, BFS with pruning (P:555-566, P:642-648,
+ * Fig. 4; R16).  Starts at the level l0 closest to the root whose
+ * node count (summed over the checkpoint's arrays) is >= T (default
+ * T = SMs * max resident threads per SM, "the number of concurrent GPU
+ * threads"), compares every node of l0, descends only below
+ * unequal nodes and lists the unequal leaves: the potentially changed
+ * chunks.  The result does not depend on T.
+ *
+ *   chunks      device, capacity `cap` uint64 chunk ids (global, ascending).
+ *   n_chunks    (host) full count / (device) for the _async form.
+ *   T           0 = default.
+ * Errors: CKPT_EINVAL (NULL trees/outputs), CKPT_EMISMATCH (different
+ * dtype, chunk_bytes, eps, array count or array lengths), CKPT_ETRUNC.
+ * The _async form cannot report CKPT_ETRUNC (the count is on the device);
+ * compare *n_chunks_dev with cap yourself.
+ * ---------------------------------------------------------------------- */
+ckpt_status ckpt_tree_diff(const ckpt_tree *a, const ckpt_tree *b, uint64_t *chunks, uint64_t cap,
+                           uint64_t *n_chunks, void *stream);
+ckpt_status ckpt_tree_diff_async(const ckpt_tree *a, const ckpt_tree *b, uint64_t T,
+                                 uint64_t *chunks, uint64_t cap, uint64_t *n_chunks_dev,
+                                 void *stream);
+
+/* ------------------------------------------------------------------------
+ * Step 4: stage-2 verification: for every listed chunk and
+ * every element i in it, report i when fabs((double)a_i - (double)b_i) > eps
+ * (binary64 for both dtypes, strict '>', NaN never differs; P:222,
+ * P:713-716; R11).
+ *
+ *   a, b        device arrays of n elements (same layout as the build).
+ *   chunks      device, ascending unique chunk ids (as produced by diff).
+ *   n_chunks    (host) number of listed chunks.
+ *   idx         device, capacity `cap` uint64 element ids (ascending).
+ *   n_diff      (host) full count.
+ * Errors: CKPT_EINVAL (NULL/misaligned pointers, bad chunk_bytes, eps < 0,
+ * NaN or inf, chunk id out of range is NOT checked: ids must come from a
+ * diff of trees of the same shape), CKPT_ETRUNC.
+ * ---------------------------------------------------------------------- */
+ckpt_status ckpt_verify(const void *a, const void *b, uint64_t n, ckpt_dtype dtype,
+                        uint32_t chunk_bytes, const uint64_t *chunks, uint64_t n_chunks,
+                        double eps, uint64_t *idx, uint64_t cap, uint64_t *n_diff, void *stream);
+
+/* Multi-array, fully asynchronous form.  a, b, n are (host) arrays of
+ * n_arrays entries.  The chunk count is read on the device from
+ * *n_chunks_dev, clamped to chunks_cap; the full difference count is
+ * written to *n_diff_dev (device). */
+ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b, const uint64_t *n,
+                                     uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                     const uint64_t *chunks, const uint64_t *n_chunks_dev,
+                                     uint64_t chunks_cap, double eps, uint64_t *idx, uint64_t cap,
+                                     uint64_t *n_diff_dev, void *stream);
+
+/* ------------------------------------------------------------------------
+ * One-call pair comparison (steps 1-4 on two checkpoints of n_arrays
+ * arrays each), the library API of P:254-257.  Device inputs.  Writes the
+ * chunk list and element ids to the caller's device buffers and both full
+ * counts to (host) *n_chunks / *n_diff; root_a16 / root_b16 (host, may be
+ * NULL) receive the two checkpoint roots.  Synchronises `stream`.
+ * ---------------------------------------------------------------------- */
+ckpt_status ckpt_compare(const void *const *a, const void *const *b, const uint64_t *n,
+                         uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                         uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                         uint64_t *n_chunks, uint64_t *n_diff, uint8_t *root_a16,
+                         uint8_t *root_b16, void *stream);
+
+/* Same with HOST inputs and outputs: a, b are (host) arrays of host
+ * pointers (pinned memory is fastest; pageable works).  The library stages
+ * each array to the device (double-buffered over two streams so the copy
+ * of one array overlaps the hashing of the previous), runs steps 1-4 and
+ * copies the element ids back into idx (host, capacity idx_cap).
+ * Synchronous. */
+ckpt_status ckpt_compare_host(const void *const *a, const void *const *b, const uint64_t *n,
+                              uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                              double eps, uint64_t *idx, uint64_t idx_cap, uint64_t *n_chunks,
+                              uint64_t *n_diff, uint8_t *root_a16, uint8_t *root_b16);
+
+/* ------------------------------------------------------------------------
+ * Accessors (parity tests, multi-GPU driver)
+ * ---------------------------------------------------------------------- */
+
+/* (host outputs, any may be NULL) number of arrays, total leaves (= total
+ * chunks), number of levels of the tallest array tree, total stored nodes
+ * (all arrays, all levels; excludes the top tree over array roots). */
+ckpt_status ckpt_tree_info(const ckpt_tree *t, uint32_t *n_arrays, uint64_t *n_leaves,
+                           uint32_t *n_levels, uint64_t *n_nodes);
+
+/* (host) 16-byte checkpoint root = root of the tree over the array roots
+ * (equal to the array root when n_arrays == 1).  Synchronises `stream`. */
+ckpt_status ckpt_tree_root(const ckpt_tree *t, uint8_t out16[16], void *stream);
+
+/* Device copy of the n_arrays array roots (dst: device, n_arrays*16 bytes),
+ * in array order.  Asynchronous. */
+ckpt_status ckpt_tree_array_roots(const ckpt_tree *t, void *dst, void *stream);
+
+/* Device copy of every node of array `array` (all levels, leaf-first, root
+ * last; the oracle's layout) into dst (device, cap_bytes).  Asynchronous.
+ * CKPT_EINVAL if array is out of range or cap_bytes is too small. */
+ckpt_status ckpt_tree_nodes(const ckpt_tree *t, uint32_t array, void *dst, uint64_t cap_bytes,
+                            void *stream);
+/* Node count of array `array` (host). */
+ckpt_status ckpt_tree_array_info(const ckpt_tree *t, uint32_t array, uint64_t *n_leaves,
+                                 uint64_t *n_nodes);
+
+/* Default BFS threshold T for the current device (SMs * max threads/SM). */
+uint64_t ckpt_default_bfs_threshold(void);
+
+/* Number of kernels this library has launched in this process (all entry
+ * points, all threads) -- lets benchmarks report their own launch count. */
+uint64_t ckpt_launch_count(void);
+
+/* Kernel timing hook for benchmarks (CUDA events on the launching stream).
+ * While enabled, every launch of kernel family `k` (0 = leaf hash K1,
+ * 1 = tree levels K2, 2 = diff K3, 3 = verify K4) is bracketed by two
+ * events.  ckpt_profile_read synchronises those events and returns the
+ * summed device time in milliseconds and the launch count of family k
+ * since the last reset.  Off by default. */
+void ckpt_profile_enable(int on);
+void ckpt_profile_reset(void);
+ckpt_status ckpt_profile_read(int k, double *ms, uint64_t *launches);
+
+const char *ckpt_strerror(ckpt_status s);
+/* Thread-local detail of the last error returned on this thread. */
+const char *ckpt_last_error(void);
+/* ABI version: (major << 16) | minor. */
+uint32_t ckpt_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* CKPT_H */

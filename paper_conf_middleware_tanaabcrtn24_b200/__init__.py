@@ -1,0 +1,380 @@
+"""B200-native error-bounded Merkle-tree checkpoint comparison (Tan et al., MIDDLEWARE '24).
+
+Thin ctypes binding over ``libckpt.so`` (C ABI in ``include/ckpt.h``).  This
+module only marshals arguments (torch tensors -> device pointers, streams,
+output buffers); every step of the path -- rounding + hashing, tree levels,
+BFS diff, verification -- runs in the library's CUDA kernels.  There is no
+CPU fallback: without the compiled library, or without a B200, every call
+raises.
+
+Function names follow the C ABI:
+
+    tree_build(arrays, chunk_bytes, eps)      ckpt_tree_build_arrays   (Alg. 1)
+    tree_diff(ta, tb)                         ckpt_tree_diff
+    verify(a, b, chunks, chunk_bytes, eps)    ckpt_verify(_arrays)
+    compare(arrays_a, arrays_b, ...)          ckpt_compare             (steps 1-4)
+    compare_host(...)                         ckpt_compare_host        (host buffers)
+    tree_from_digests(digests)                ckpt_tree_from_digests   (top tree, R15)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import List, Optional, Sequence, Tuple, Union
+
+import torch
+
+from . import _build
+
+__all__ = [
+    "CkptError", "Tree", "lib", "tree_build", "tree_from_digests", "tree_diff", "tree_diff_async",
+    "verify", "verify_async", "compare", "compare_host", "launch_count", "default_bfs_threshold",
+    "F32", "F64",
+]
+
+F32 = 0
+F64 = 1
+
+OK, EINVAL, EMISMATCH, ENOMEM, ECUDA, ETRUNC = 0, -1, -2, -3, -4, -5
+
+
+class CkptError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        self.status = status
+        super().__init__(f"{what}: status {status}")
+
+
+_lib = None
+
+
+def lib():
+    """Load libckpt.so (in-tree).  Raises if it is missing: there is no fallback."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = _build.LIB
+    if not os.path.exists(path):
+        raise ImportError(
+            f"libckpt.so not built at {path}; run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = ctypes.CDLL(path)
+    vp, u64, u32, i32, dbl = (ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int,
+                              ctypes.c_double)
+    pp = ctypes.POINTER(ctypes.c_void_p)
+    pu64 = ctypes.POINTER(ctypes.c_uint64)
+    L.ckpt_tree_build.argtypes = [vp, u64, i32, u32, dbl, vp, pp]
+    L.ckpt_tree_build_arrays.argtypes = [pp, pu64, u32, i32, u32, dbl, vp, pp]
+    L.ckpt_tree_from_digests.argtypes = [vp, u64, vp, pp]
+    L.ckpt_tree_free.argtypes = [vp]
+    L.ckpt_tree_free.restype = None
+    L.ckpt_tree_free_on.argtypes = [vp, vp]
+    L.ckpt_tree_free_on.restype = None
+    L.ckpt_tree_diff.argtypes = [vp, vp, vp, u64, pu64, vp]
+    L.ckpt_tree_diff_async.argtypes = [vp, vp, u64, vp, u64, vp, vp]
+    L.ckpt_verify.argtypes = [vp, vp, u64, i32, u32, vp, u64, dbl, vp, u64, pu64, vp]
+    L.ckpt_verify_arrays_async.argtypes = [pp, pp, pu64, u32, i32, u32, vp, vp, u64, dbl, vp, u64,
+                                           vp, vp]
+    L.ckpt_compare.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, vp, u64, vp, u64, pu64, pu64, vp,
+                               vp, vp]
+    L.ckpt_compare_host.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, vp, u64, pu64, pu64, vp, vp]
+    L.ckpt_tree_info.argtypes = [vp, ctypes.POINTER(u32), pu64, ctypes.POINTER(u32), pu64]
+    L.ckpt_tree_root.argtypes = [vp, vp, vp]
+    L.ckpt_tree_array_roots.argtypes = [vp, vp, vp]
+    L.ckpt_tree_nodes.argtypes = [vp, u32, vp, u64, vp]
+    L.ckpt_tree_array_info.argtypes = [vp, u32, pu64, pu64]
+    L.ckpt_profile_enable.argtypes = [i32]
+    L.ckpt_profile_enable.restype = None
+    L.ckpt_profile_reset.restype = None
+    L.ckpt_profile_read.argtypes = [i32, ctypes.POINTER(dbl), pu64]
+    L.ckpt_profile_read.restype = i32
+    L.ckpt_default_bfs_threshold.restype = u64
+    L.ckpt_launch_count.restype = u64
+    L.ckpt_strerror.argtypes = [i32]
+    L.ckpt_strerror.restype = ctypes.c_char_p
+    L.ckpt_last_error.restype = ctypes.c_char_p
+    L.ckpt_version.restype = u32
+    for name in ("ckpt_tree_build", "ckpt_tree_build_arrays", "ckpt_tree_from_digests",
+                 "ckpt_tree_diff", "ckpt_tree_diff_async", "ckpt_verify",
+                 "ckpt_verify_arrays_async", "ckpt_compare", "ckpt_compare_host",
+                 "ckpt_tree_info", "ckpt_tree_root", "ckpt_tree_array_roots", "ckpt_tree_nodes",
+                 "ckpt_tree_array_info"):
+        getattr(L, name).restype = i32
+    _lib = L
+    return L
+
+
+def _check(st: int, what: str, allow_trunc: bool = False):
+    if st == OK or (allow_trunc and st == ETRUNC):
+        return
+    L = lib()
+    msg = L.ckpt_last_error().decode(errors="replace")
+    raise CkptError(st, f"{what}: {L.ckpt_strerror(st).decode()} ({msg})")
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    if t.dtype == torch.float32:
+        return F32
+    if t.dtype == torch.float64:
+        return F64
+    raise TypeError(f"only float32/float64 checkpoints are supported, got {t.dtype}")
+
+
+def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+def _as_list(x) -> List[torch.Tensor]:
+    if isinstance(x, torch.Tensor):
+        return [x]
+    return list(x)
+
+
+def _check_arrays(arrays: Sequence[torch.Tensor]) -> int:
+    if not arrays:
+        raise ValueError("no arrays")
+    code = _dtype_code(arrays[0])
+    for t in arrays:
+        if not t.is_cuda:
+            raise ValueError("tensors must live on the CUDA device (use compare_host for host data)")
+        if not t.is_contiguous():
+            raise ValueError("tensors must be contiguous")
+        if _dtype_code(t) != code:
+            raise ValueError("all arrays of a checkpoint share one dtype")
+    return code
+
+
+def _ptr_array(ts: Sequence[torch.Tensor]):
+    arr = (ctypes.c_void_p * len(ts))(*[t.data_ptr() for t in ts])
+    return ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p)), arr
+
+
+def _u64_array(vals: Sequence[int]):
+    arr = (ctypes.c_uint64 * len(vals))(*vals)
+    return ctypes.cast(arr, ctypes.POINTER(ctypes.c_uint64)), arr
+
+
+class Tree:
+    """Library-owned Merkle tree of one checkpoint (one or more arrays)."""
+
+    def __init__(self, handle: int, arrays: Sequence[torch.Tensor], dtype: int, chunk_bytes: int,
+                 eps: float, stream_ptr: int):
+        self._h = ctypes.c_void_p(handle)
+        self._keep = list(arrays)          # borrowed inputs must outlive the enqueued work
+        self.dtype = dtype
+        self.chunk_bytes = chunk_bytes
+        self.eps = eps
+        self._stream_ptr = stream_ptr
+        na, nl = ctypes.c_uint32(), ctypes.c_uint64()
+        nlev, nn = ctypes.c_uint32(), ctypes.c_uint64()
+        _check(lib().ckpt_tree_info(self._h, ctypes.byref(na), ctypes.byref(nl), ctypes.byref(nlev),
+                                    ctypes.byref(nn)), "ckpt_tree_info")
+        self.n_arrays = na.value
+        self.n_leaves = nl.value
+        self.n_levels = nlev.value
+        self.n_nodes = nn.value
+
+    @property
+    def handle(self):
+        if self._h is None or not self._h.value:
+            raise ValueError("tree already freed")
+        return self._h
+
+    def root(self, stream=None) -> bytes:
+        out = (ctypes.c_uint8 * 16)()
+        _check(lib().ckpt_tree_root(self.handle, ctypes.cast(out, ctypes.c_void_p),
+                                    _stream_ptr(stream)), "ckpt_tree_root")
+        return bytes(out)
+
+    def array_roots(self, stream=None) -> torch.Tensor:
+        dst = torch.empty((self.n_arrays, 16), dtype=torch.uint8, device="cuda")
+        _check(lib().ckpt_tree_array_roots(self.handle, dst.data_ptr(), _stream_ptr(stream)),
+               "ckpt_tree_array_roots")
+        return dst
+
+    def array_info(self, array: int) -> Tuple[int, int]:
+        nl, nn = ctypes.c_uint64(), ctypes.c_uint64()
+        _check(lib().ckpt_tree_array_info(self.handle, array, ctypes.byref(nl), ctypes.byref(nn)),
+               "ckpt_tree_array_info")
+        return nl.value, nn.value
+
+    def nodes(self, array: int = 0, stream=None) -> torch.Tensor:
+        _, nn = self.array_info(array)
+        dst = torch.empty((nn, 16), dtype=torch.uint8, device="cuda")
+        _check(lib().ckpt_tree_nodes(self.handle, array, dst.data_ptr(), nn * 16,
+                                     _stream_ptr(stream)), "ckpt_tree_nodes")
+        return dst
+
+    def free(self, stream=None):
+        if self._h is not None and self._h.value:
+            lib().ckpt_tree_free_on(self._h, _stream_ptr(stream) if stream is not None
+                                    else self._stream_ptr)
+        self._h = None
+        self._keep = []
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def tree_build(arrays: Union[torch.Tensor, Sequence[torch.Tensor]], chunk_bytes: int, eps: float,
+               stream=None) -> Tree:
+    """Steps 1-2: leaves (quantize + chained Murmur3F) and all levels, asynchronously."""
+    ts = _as_list(arrays)
+    code = _check_arrays(ts)
+    pp, _k1 = _ptr_array(ts)
+    pn, _k2 = _u64_array([t.numel() for t in ts])
+    out = ctypes.c_void_p()
+    sp = _stream_ptr(stream)
+    _check(lib().ckpt_tree_build_arrays(pp, pn, len(ts), code, chunk_bytes, float(eps), sp,
+                                        ctypes.byref(out)), "ckpt_tree_build_arrays")
+    return Tree(out.value, ts, code, chunk_bytes, float(eps), sp)
+
+
+def tree_from_digests(digests: torch.Tensor, stream=None) -> Tree:
+    """Tree whose leaves are the given (count, 16) uint8 digests (top tree over roots, R15)."""
+    if digests.dtype != torch.uint8 or digests.dim() != 2 or digests.shape[1] != 16:
+        raise ValueError("digests must be a (count, 16) uint8 tensor")
+    d = digests.contiguous()
+    out = ctypes.c_void_p()
+    sp = _stream_ptr(stream)
+    _check(lib().ckpt_tree_from_digests(d.data_ptr(), d.shape[0], sp, ctypes.byref(out)),
+           "ckpt_tree_from_digests")
+    return Tree(out.value, [d], F32, 16, 0.0, sp)
+
+
+def tree_diff(ta: Tree, tb: Tree, cap: Optional[int] = None, stream=None) -> torch.Tensor:
+    """Step 3: ascending chunk ids whose leaves differ (BFS from the mid level)."""
+    cap = ta.n_leaves if cap is None else cap
+    out = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+    n = ctypes.c_uint64()
+    _check(lib().ckpt_tree_diff(ta.handle, tb.handle, out.data_ptr(), cap, ctypes.byref(n),
+                                _stream_ptr(stream)), "ckpt_tree_diff", allow_trunc=True)
+    return out[: min(n.value, cap)]
+
+
+def tree_diff_async(ta: Tree, tb: Tree, chunks: torch.Tensor, count: torch.Tensor, T: int = 0,
+                    stream=None):
+    """Step 3 without a host round trip: count lands in count[0] on the device."""
+    _check(lib().ckpt_tree_diff_async(ta.handle, tb.handle, T, chunks.data_ptr(), chunks.numel(),
+                                      count.data_ptr(), _stream_ptr(stream)), "ckpt_tree_diff_async")
+
+
+def verify(a, b, chunks: torch.Tensor, chunk_bytes: int, eps: float, cap: Optional[int] = None,
+           stream=None) -> Tuple[torch.Tensor, int]:
+    """Step 4 on one array (sync): element ids with |a-b| > eps inside the listed chunks."""
+    ta, tb = _as_list(a), _as_list(b)
+    if len(ta) != 1:
+        count = torch.zeros(2, dtype=torch.int64, device="cuda")
+        count[0] = chunks.numel()
+        out = torch.empty(max(cap or sum(t.numel() for t in ta), 1), dtype=torch.int64,
+                          device="cuda")
+        verify_async(ta, tb, chunks, count[0:1], chunk_bytes, eps, out, count[1:2], stream)
+        n = int(count[1].item())
+        return out[: min(n, out.numel())], n
+    a, b = ta[0], tb[0]
+    code = _check_arrays([a, b])
+    ch = chunks.contiguous()
+    cap = a.numel() if cap is None else cap
+    out = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+    n = ctypes.c_uint64()
+    _check(lib().ckpt_verify(a.data_ptr(), b.data_ptr(), a.numel(), code, chunk_bytes,
+                             ch.data_ptr() if ch.numel() else None, ch.numel(), float(eps),
+                             out.data_ptr(), cap, ctypes.byref(n), _stream_ptr(stream)),
+           "ckpt_verify", allow_trunc=True)
+    return out[: min(n.value, cap)], n.value
+
+
+def verify_async(arrays_a, arrays_b, chunks: torch.Tensor, n_chunks_dev: torch.Tensor,
+                 chunk_bytes: int, eps: float, out: torch.Tensor, count_dev: torch.Tensor,
+                 stream=None):
+    """Step 4 over a multi-array checkpoint; chunk count read on the device."""
+    ta, tb = _as_list(arrays_a), _as_list(arrays_b)
+    code = _check_arrays(ta + tb)
+    pa, _k1 = _ptr_array(ta)
+    pb, _k2 = _ptr_array(tb)
+    pn, _k3 = _u64_array([t.numel() for t in ta])
+    _check(lib().ckpt_verify_arrays_async(pa, pb, pn, len(ta), code, chunk_bytes,
+                                          chunks.data_ptr(), n_chunks_dev.data_ptr(),
+                                          chunks.numel(), float(eps), out.data_ptr(), out.numel(),
+                                          count_dev.data_ptr(), _stream_ptr(stream)),
+           "ckpt_verify_arrays_async")
+
+
+def compare(arrays_a, arrays_b, chunk_bytes: int, eps: float, chunks_cap: Optional[int] = None,
+            idx_cap: Optional[int] = None, stream=None):
+    """Steps 1-4 on device-resident checkpoints.
+
+    Returns (chunks, idx, n_chunks, n_diff, root_a, root_b)."""
+    ta, tb = _as_list(arrays_a), _as_list(arrays_b)
+    code = _check_arrays(ta + tb)
+    esz = 4 if code == F32 else 8
+    L = sum(-(-t.numel() * esz // chunk_bytes) for t in ta)
+    chunks_cap = L if chunks_cap is None else chunks_cap
+    idx_cap = sum(t.numel() for t in ta) if idx_cap is None else idx_cap
+    chunks = torch.empty(max(chunks_cap, 1), dtype=torch.int64, device="cuda")
+    idx = torch.empty(max(idx_cap, 1), dtype=torch.int64, device="cuda")
+    pa, _k1 = _ptr_array(ta)
+    pb, _k2 = _ptr_array(tb)
+    pn, _k3 = _u64_array([t.numel() for t in ta])
+    nc, nd = ctypes.c_uint64(), ctypes.c_uint64()
+    ra, rb = (ctypes.c_uint8 * 16)(), (ctypes.c_uint8 * 16)()
+    _check(lib().ckpt_compare(pa, pb, pn, len(ta), code, chunk_bytes, float(eps),
+                              chunks.data_ptr(), chunks_cap, idx.data_ptr(), idx_cap,
+                              ctypes.byref(nc), ctypes.byref(nd), ctypes.cast(ra, ctypes.c_void_p),
+                              ctypes.cast(rb, ctypes.c_void_p), _stream_ptr(stream)),
+           "ckpt_compare", allow_trunc=True)
+    return (chunks[: min(nc.value, chunks_cap)], idx[: min(nd.value, idx_cap)], nc.value,
+            nd.value, bytes(ra), bytes(rb))
+
+
+def compare_host(arrays_a, arrays_b, chunk_bytes: int, eps: float, idx_cap: Optional[int] = None):
+    """Steps 1-4 on HOST checkpoints (pinned for speed); H2D/D2H inside the call.
+
+    Returns (idx (host int64 tensor), n_chunks, n_diff, root_a, root_b)."""
+    ta, tb = _as_list(arrays_a), _as_list(arrays_b)
+    for t in ta + tb:
+        if t.is_cuda or not t.is_contiguous():
+            raise ValueError("compare_host takes contiguous host tensors")
+    code = _dtype_code(ta[0])
+    idx_cap = sum(t.numel() for t in ta) if idx_cap is None else idx_cap
+    idx = torch.empty(max(idx_cap, 1), dtype=torch.int64)
+    pa, _k1 = _ptr_array(ta)
+    pb, _k2 = _ptr_array(tb)
+    pn, _k3 = _u64_array([t.numel() for t in ta])
+    nc, nd = ctypes.c_uint64(), ctypes.c_uint64()
+    ra, rb = (ctypes.c_uint8 * 16)(), (ctypes.c_uint8 * 16)()
+    _check(lib().ckpt_compare_host(pa, pb, pn, len(ta), code, chunk_bytes, float(eps),
+                                   idx.data_ptr(), idx_cap, ctypes.byref(nc), ctypes.byref(nd),
+                                   ctypes.cast(ra, ctypes.c_void_p),
+                                   ctypes.cast(rb, ctypes.c_void_p)),
+           "ckpt_compare_host", allow_trunc=True)
+    return idx[: min(nd.value, idx_cap)], nc.value, nd.value, bytes(ra), bytes(rb)
+
+
+def launch_count() -> int:
+    return int(lib().ckpt_launch_count())
+
+
+def default_bfs_threshold() -> int:
+    return int(lib().ckpt_default_bfs_threshold())
+
+
+KERNELS = {"leaf": 0, "levels": 1, "diff": 2, "verify": 3}
+
+
+def profile_enable(on: bool = True):
+    lib().ckpt_profile_enable(1 if on else 0)
+
+
+def profile_reset():
+    lib().ckpt_profile_reset()
+
+
+def profile_read(kernel: str) -> Tuple[float, int]:
+    """(summed device ms, launches) of one kernel family since the last reset."""
+    ms, n = ctypes.c_double(), ctypes.c_uint64()
+    _check(lib().ckpt_profile_read(KERNELS[kernel], ctypes.byref(ms), ctypes.byref(n)),
+           "ckpt_profile_read")
+    return ms.value, n.value

@@ -1,0 +1,981 @@
+// ckpt.cu -- host side of libckpt.so: the C ABI declared in include/ckpt.h.
+//
+// Validation, tree layout (level-major flattened array, R13),
+// device allocation (stream-ordered pool), metadata staging and kernel
+// launches for K1 (leaf.cuh), K2 (levels.cuh), K3/K4 (compare.cuh).  Every
+// step of the path runs in those kernels; there is no host or CPU fallback.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cfloat>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <deque>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/ckpt.h"
+#include "compare.cuh"
+#include "hash.cuh"
+#include "leaf.cuh"
+#include "levels.cuh"
+
+using namespace ckpt;
+
+// ---------------------------------------------------------------------------
+// errors
+// ---------------------------------------------------------------------------
+static thread_local std::string g_last_error;
+static std::atomic<uint64_t> g_launches{0};
+
+static ckpt_status fail(ckpt_status s, const std::string &msg) {
+    g_last_error = msg;
+    return s;
+}
+
+#define CK_CUDA(expr)                                                                       \
+    do {                                                                                    \
+        cudaError_t e_ = (expr);                                                            \
+        if (e_ != cudaSuccess) {                                                            \
+            return fail(e_ == cudaErrorMemoryAllocation ? CKPT_ENOMEM : CKPT_ECUDA,         \
+                        std::string(#expr) + ": " + cudaGetErrorString(e_));                \
+        }                                                                                   \
+    } while (0)
+
+#define CK_LAUNCH()                                                                         \
+    do {                                                                                    \
+        g_launches.fetch_add(1, std::memory_order_relaxed);                                 \
+        cudaError_t e_ = cudaGetLastError();                                                \
+        if (e_ != cudaSuccess)                                                              \
+            return fail(CKPT_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e_)); \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// optional per-kernel-family event timing (ckpt_profile_*)
+// ---------------------------------------------------------------------------
+struct ProfRec { int k; cudaEvent_t a, b; };
+static std::atomic<int> g_prof_on{0};
+static std::mutex g_prof_mu;
+static std::vector<ProfRec> g_prof;
+
+struct ProfScope {
+    int k;
+    cudaStream_t s;
+    cudaEvent_t a = nullptr, b = nullptr;
+    ProfScope(int k_, cudaStream_t s_) : k(k_), s(s_) {
+        if (g_prof_on.load(std::memory_order_relaxed)) {
+            cudaEventCreate(&a);
+            cudaEventCreate(&b);
+            cudaEventRecord(a, s);
+        }
+    }
+    ~ProfScope() {
+        if (a) {
+            cudaEventRecord(b, s);
+            std::lock_guard<std::mutex> lk(g_prof_mu);
+            g_prof.push_back({k, a, b});
+        }
+    }
+};
+
+#define CK_TRY(expr)                         \
+    do {                                     \
+        ckpt_status s_ = (expr);             \
+        if (s_ != CKPT_OK) return s_;        \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// device properties
+// ---------------------------------------------------------------------------
+struct DevInfo {
+    int sms = 0;
+    int max_threads_sm = 0;
+    bool pool_set = false;
+};
+static std::mutex g_dev_mu;
+static DevInfo g_dev[64];
+
+static ckpt_status dev_info(int *dev_out, DevInfo *info) {
+    int dev = 0;
+    CK_CUDA(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    DevInfo &d = g_dev[dev & 63];
+    if (d.sms == 0) {
+        CK_CUDA(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
+        CK_CUDA(cudaDeviceGetAttribute(&d.max_threads_sm, cudaDevAttrMaxThreadsPerMultiProcessor, dev));
+        int major = 0, minor = 0;
+        CK_CUDA(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev));
+        CK_CUDA(cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev));
+        if (major != 10 || minor != 0) {
+            d.sms = 0;
+            return fail(CKPT_ECUDA, "libckpt is built for sm_100a (B200); device has sm_" +
+                                        std::to_string(major) + std::to_string(minor));
+        }
+    }
+    if (!d.pool_set) {
+        cudaMemPool_t pool;
+        CK_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
+        uint64_t thr = 8ull << 30;   // keep up to 8 GiB cached between frees
+        CK_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        d.pool_set = true;
+    }
+    if (dev_out) *dev_out = dev;
+    if (info) *info = d;
+    return CKPT_OK;
+}
+
+// ---------------------------------------------------------------------------
+// pinned staging ring for small host->device metadata copies
+// ---------------------------------------------------------------------------
+struct PinnedRing {
+    std::mutex mu;
+    uint8_t *base = nullptr;
+    size_t cap = 0, head = 0;
+    struct Span { size_t lo, hi; cudaEvent_t ev; };
+    std::deque<Span> live;
+
+    ckpt_status copy(void *dst_dev, const void *src, size_t bytes, cudaStream_t s) {
+        std::lock_guard<std::mutex> lk(mu);
+        const size_t n_copy = bytes;
+        bytes = (bytes + 255) & ~size_t(255);
+        if (base == nullptr) {
+            cap = std::max<size_t>(64ull << 20, bytes);
+            CK_CUDA(cudaHostAlloc((void **)&base, cap, cudaHostAllocPortable));
+        }
+        if (bytes > cap) return fail(CKPT_ENOMEM, "metadata larger than the staging ring");
+        if (head + bytes > cap) head = 0;
+        const size_t lo = head, hi = head + bytes;
+        // wait for in-flight copies that still read [lo, hi)
+        for (auto it = live.begin(); it != live.end();) {
+            if (it->lo < hi && lo < it->hi) {
+                CK_CUDA(cudaEventSynchronize(it->ev));
+                cudaEventDestroy(it->ev);
+                it = live.erase(it);
+            } else if (cudaEventQuery(it->ev) == cudaSuccess) {
+                cudaEventDestroy(it->ev);
+                it = live.erase(it);
+            } else {
+                ++it;
+            }
+        }
+        std::memcpy(base + lo, src, n_copy);
+        CK_CUDA(cudaMemcpyAsync(dst_dev, base + lo, n_copy, cudaMemcpyHostToDevice, s));
+        cudaEvent_t ev;
+        CK_CUDA(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        CK_CUDA(cudaEventRecord(ev, s));
+        live.push_back({lo, hi, ev});
+        head = hi;
+        return CKPT_OK;
+    }
+};
+static PinnedRing g_ring;
+
+// ---------------------------------------------------------------------------
+// tree
+// ---------------------------------------------------------------------------
+struct ckpt_tree {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    ckpt_dtype dtype = CKPT_F32;
+    uint32_t chunk_bytes = 0;
+    double eps = 0.0;
+    bool from_digests = false;
+    uint32_t n_arrays = 0;
+    uint32_t n_levels = 0;                 // max height
+    std::vector<uint64_t> n_elems;         // per array
+    std::vector<uint64_t> n_leaves;        // per array
+    std::vector<uint32_t> height;          // per array
+    std::vector<uint64_t> off, cnt;        // [l * n_arrays + a]
+    std::vector<uint64_t> level_base, level_total;
+    std::vector<uint64_t> chunk_base;      // per array
+    uint64_t total_leaves = 0;
+    uint64_t array_nodes = 0;              // nodes of all array levels
+    uint64_t top_off = 0, top_nodes = 0;
+    uint4 *nodes = nullptr;                // device
+    uint8_t *meta = nullptr;               // device metadata blob
+    // device views into meta
+    const uint64_t *d_off = nullptr, *d_cnt = nullptr, *d_level_base = nullptr,
+                   *d_level_total = nullptr, *d_chunk_base = nullptr;
+    const uint32_t *d_height = nullptr;
+};
+
+static uint32_t tree_height(uint64_t L) {
+    uint32_t h = 1;
+    while (L > 1) { L = (L + 1) / 2; ++h; }
+    return h;
+}
+
+// Lay out an array-level tree over per-array leaf counts.
+static void layout(ckpt_tree *t, const std::vector<uint64_t> &leaves) {
+    const uint32_t na = (uint32_t)leaves.size();
+    t->n_arrays = na;
+    t->n_leaves = leaves;
+    t->height.resize(na);
+    t->n_levels = 1;
+    for (uint32_t a = 0; a < na; ++a) {
+        t->height[a] = tree_height(leaves[a]);
+        t->n_levels = std::max(t->n_levels, t->height[a]);
+    }
+    const uint32_t nl = t->n_levels;
+    t->off.assign((size_t)nl * na, 0);
+    t->cnt.assign((size_t)nl * na, 0);
+    t->level_base.assign(nl + 1, 0);
+    t->level_total.assign(nl + 1, 0);
+    uint64_t pos = 0;
+    for (uint32_t l = 0; l < nl; ++l) {
+        t->level_base[l] = pos;
+        for (uint32_t a = 0; a < na; ++a) {
+            uint64_t c = 0;
+            if (l < t->height[a]) {
+                c = leaves[a];
+                for (uint32_t k = 0; k < l; ++k) c = (c + 1) / 2;
+            }
+            t->off[(size_t)l * na + a] = pos;
+            t->cnt[(size_t)l * na + a] = c;
+            pos += c;
+        }
+        t->level_total[l] = pos - t->level_base[l];
+    }
+    t->array_nodes = pos;
+    t->level_base[nl] = pos;
+    t->chunk_base.resize(na);
+    uint64_t cb = 0;
+    for (uint32_t a = 0; a < na; ++a) { t->chunk_base[a] = cb; cb += leaves[a]; }
+    t->total_leaves = cb;
+    t->top_off = pos;
+    uint64_t tn = 0, n = na;
+    for (;;) { tn += n; if (n == 1) break; n = (n + 1) / 2; }
+    t->top_nodes = tn;
+}
+
+static size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
+
+// Allocate nodes + metadata, stage metadata.  `extra` = leaf table bytes.
+static ckpt_status alloc_tree(ckpt_tree *t, cudaStream_t s, std::vector<uint8_t> &blob,
+                              std::vector<size_t> &offs) {
+    CK_CUDA(cudaMallocAsync((void **)&t->nodes, (t->array_nodes + t->top_nodes) * 16, s));
+    CK_CUDA(cudaMallocAsync((void **)&t->meta, blob.size(), s));
+    CK_TRY(g_ring.copy(t->meta, blob.data(), blob.size(), s));
+    (void)offs;
+    return CKPT_OK;
+}
+
+static bool quant_params(double eps, QuantParams *q) {
+    if (!(eps >= 0.0) || std::isinf(eps)) return false;
+    if (eps == 0.0) { std::memset(q, 0, sizeof(*q)); return true; }
+    const double inv = 1.0 / eps;
+    if (!std::isfinite(inv)) return false;
+    q->inv = inv;
+    int ex;
+    const double fr = std::frexp(inv, &ex);            // inv = fr * 2^ex, fr in [0.5,1)
+    q->inv_m = (uint64_t)std::ldexp(fr, 53);           // exact 53-bit integer
+    q->inv_e = ex - 53;
+    q->r64 = std::ldexp(1.0, 50) / inv;                // |x| < r64 => |x*inv| < 2^51
+    float r32;
+    if (q->r64 >= (double)FLT_MAX) {
+        r32 = INFINITY;
+    } else {
+        r32 = (float)q->r64;
+        if ((double)r32 > q->r64) r32 = std::nextafterf(r32, 0.0f);
+    }
+    q->r32 = r32;
+    return true;
+}
+
+static ckpt_status check_common(ckpt_dtype dtype, uint32_t chunk_bytes, double eps) {
+    if (dtype != CKPT_F32 && dtype != CKPT_F64) return fail(CKPT_EINVAL, "unknown dtype");
+    if (chunk_bytes == 0 || chunk_bytes % 16 != 0)
+        return fail(CKPT_EINVAL, "chunk_bytes must be a positive multiple of 16");
+    QuantParams q;
+    if (!quant_params(eps, &q)) return fail(CKPT_EINVAL, "eps must be finite, >= 0, with 1/eps finite");
+    return CKPT_OK;
+}
+
+template <int DT, bool RAW, int CB>
+static ckpt_status launch_leaf_t(const LeafArray *arr, int na, uint64_t tasks, uint32_t C,
+                                 const QuantParams &q, uint4 *nodes, cudaStream_t s, int sms) {
+    auto k = leaf_kernel<DT, RAW, CB>;
+    static std::atomic<int> cached_per_sm{0};
+    int per_sm = cached_per_sm.load(std::memory_order_relaxed);
+    if (per_sm == 0) {
+        CK_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kLeafSmem));
+        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kLeafWarps * 32, kLeafSmem));
+        per_sm = std::max(per_sm, 1);
+        cached_per_sm.store(per_sm, std::memory_order_relaxed);
+    } else {
+        CK_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kLeafSmem));
+    }
+    uint64_t want = (tasks + kLeafWarps - 1) / kLeafWarps;
+    uint64_t grid = std::min<uint64_t>(want, (uint64_t)sms * per_sm);
+    ProfScope prof(0, s);
+    k<<<(unsigned)grid, kLeafWarps * 32, kLeafSmem, s>>>(arr, na, tasks, C, q, nodes);
+    CK_LAUNCH();
+    return CKPT_OK;
+}
+
+template <int DT, bool RAW>
+static ckpt_status launch_leaf_dt(const LeafArray *arr, int na, uint64_t tasks, uint32_t C,
+                                  const QuantParams &q, uint4 *nodes, cudaStream_t s, int sms) {
+    if (!RAW) {
+        switch (C) {
+            case 512: return launch_leaf_t<DT, RAW, 512>(arr, na, tasks, C, q, nodes, s, sms);
+            case 1024: return launch_leaf_t<DT, RAW, 1024>(arr, na, tasks, C, q, nodes, s, sms);
+            case 2048: return launch_leaf_t<DT, RAW, 2048>(arr, na, tasks, C, q, nodes, s, sms);
+            case 4096: return launch_leaf_t<DT, RAW, 4096>(arr, na, tasks, C, q, nodes, s, sms);
+            case 8192: return launch_leaf_t<DT, RAW, 8192>(arr, na, tasks, C, q, nodes, s, sms);
+            case 16384: return launch_leaf_t<DT, RAW, 16384>(arr, na, tasks, C, q, nodes, s, sms);
+            case 32768: return launch_leaf_t<DT, RAW, 32768>(arr, na, tasks, C, q, nodes, s, sms);
+            case 65536: return launch_leaf_t<DT, RAW, 65536>(arr, na, tasks, C, q, nodes, s, sms);
+            default: break;
+        }
+    }
+    return launch_leaf_t<DT, RAW, 0>(arr, na, tasks, C, q, nodes, s, sms);
+}
+
+static ckpt_status launch_levels(ckpt_tree *t, const uint64_t *d_gbegin, uint64_t n_groups,
+                                 unsigned *ticket, cudaStream_t s) {
+    LevelParams p;
+    p.nodes = t->nodes;
+    p.off = t->d_off;
+    p.cnt = t->d_cnt;
+    p.gbegin = d_gbegin;
+    p.level_base = t->d_level_base;
+    p.level_total = t->d_level_total;
+    p.height = t->d_height;
+    p.top_off = t->top_off;
+    p.ticket = ticket;
+    p.n_arrays = (int)t->n_arrays;
+    p.n_levels = (int)t->n_levels;
+    p.ls = 0;
+    ProfScope prof(1, s);
+    levels_kernel<<<(unsigned)n_groups, kLevelThreads, 0, s>>>(p);
+    CK_LAUNCH();
+    return CKPT_OK;
+}
+
+// Build the blob: [off][cnt][level_base][level_total][chunk_base][height][gbegin][ticket][leaf table]
+static ckpt_status build_common(ckpt_tree *t, cudaStream_t s, const LeafArray *leaf_host,
+                                const QuantParams *q, int sms, const void *digests) {
+    const uint32_t na = t->n_arrays, nl = t->n_levels;
+    std::vector<uint64_t> gbegin(na);
+    uint64_t groups = 0;
+    for (uint32_t a = 0; a < na; ++a) {
+        gbegin[a] = groups;
+        groups += (t->cnt[a] + kGroup - 1) / kGroup;   // level 0 counts
+    }
+    size_t o_off = 0;
+    size_t o_cnt = align256(o_off + t->off.size() * 8);
+    size_t o_lb = align256(o_cnt + t->cnt.size() * 8);
+    size_t o_lt = align256(o_lb + t->level_base.size() * 8);
+    size_t o_cb = align256(o_lt + t->level_total.size() * 8);
+    size_t o_h = align256(o_cb + (size_t)na * 8);
+    size_t o_g = align256(o_h + (size_t)na * 4);
+    size_t o_tk = align256(o_g + (size_t)na * 8);
+    size_t o_leaf = align256(o_tk + 16);
+    size_t total = align256(o_leaf + (leaf_host ? (size_t)na * sizeof(LeafArray) : 0));
+    std::vector<uint8_t> blob(total, 0);
+    std::memcpy(blob.data() + o_off, t->off.data(), t->off.size() * 8);
+    std::memcpy(blob.data() + o_cnt, t->cnt.data(), t->cnt.size() * 8);
+    std::memcpy(blob.data() + o_lb, t->level_base.data(), t->level_base.size() * 8);
+    std::memcpy(blob.data() + o_lt, t->level_total.data(), t->level_total.size() * 8);
+    std::memcpy(blob.data() + o_cb, t->chunk_base.data(), (size_t)na * 8);
+    std::memcpy(blob.data() + o_h, t->height.data(), (size_t)na * 4);
+    std::memcpy(blob.data() + o_g, gbegin.data(), (size_t)na * 8);
+    if (leaf_host) std::memcpy(blob.data() + o_leaf, leaf_host, (size_t)na * sizeof(LeafArray));
+    std::vector<size_t> offs;
+    CK_TRY(alloc_tree(t, s, blob, offs));
+    t->d_off = (const uint64_t *)(t->meta + o_off);
+    t->d_cnt = (const uint64_t *)(t->meta + o_cnt);
+    t->d_level_base = (const uint64_t *)(t->meta + o_lb);
+    t->d_level_total = (const uint64_t *)(t->meta + o_lt);
+    t->d_chunk_base = (const uint64_t *)(t->meta + o_cb);
+    t->d_height = (const uint32_t *)(t->meta + o_h);
+    const uint64_t *d_gbegin = (const uint64_t *)(t->meta + o_g);
+    unsigned *ticket = (unsigned *)(t->meta + o_tk);
+    (void)nl;
+    if (leaf_host) {
+        // leaf table with the device node pointer offsets
+        const LeafArray *d_leaf = (const LeafArray *)(t->meta + o_leaf);
+        uint64_t tasks = 0;
+        for (uint32_t a = 0; a < na; ++a) tasks += (t->n_leaves[a] + 31) / 32;
+        const uint32_t C = t->chunk_bytes;
+        if (t->eps == 0.0) {
+            if (t->dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
+            else CK_TRY((launch_leaf_dt<1, true>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
+        } else {
+            if (t->dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
+            else CK_TRY((launch_leaf_dt<1, false>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
+        }
+    } else if (digests) {
+        CK_CUDA(cudaMemcpyAsync(t->nodes, digests, t->total_leaves * 16, cudaMemcpyDeviceToDevice, s));
+    }
+    return launch_levels(t, d_gbegin, groups, ticket, s);
+}
+
+extern "C" ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n,
+                                              uint32_t n_arrays, ckpt_dtype dtype,
+                                              uint32_t chunk_bytes, double eps, void *stream,
+                                              ckpt_tree **out) {
+    if (!out) return fail(CKPT_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!data || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
+    if (n_arrays >= (1u << 20)) return fail(CKPT_EINVAL, "at most 2^20-1 arrays");
+    CK_TRY(check_common(dtype, chunk_bytes, eps));
+    const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
+    for (uint32_t a = 0; a < n_arrays; ++a) {
+        if (!data[a]) return fail(CKPT_EINVAL, "NULL data pointer");
+        if (n[a] == 0) return fail(CKPT_EINVAL, "empty array (n == 0)");
+        if ((uintptr_t)data[a] % 16 != 0) return fail(CKPT_EINVAL, "data must be 16-byte aligned");
+        if (n[a] > (1ull << 50)) return fail(CKPT_EINVAL, "array too large");
+    }
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    cudaStream_t s = (cudaStream_t)stream;
+    ckpt_tree *t = new ckpt_tree();
+    t->device = dev;
+    t->stream = s;
+    t->dtype = dtype;
+    t->chunk_bytes = chunk_bytes;
+    t->eps = eps;
+    t->n_elems.assign(n, n + n_arrays);
+    std::vector<uint64_t> leaves(n_arrays);
+    for (uint32_t a = 0; a < n_arrays; ++a) leaves[a] = (n[a] * esz + chunk_bytes - 1) / chunk_bytes;
+    layout(t, leaves);
+    std::vector<LeafArray> lt(n_arrays);
+    uint64_t task = 0;
+    for (uint32_t a = 0; a < n_arrays; ++a) {
+        lt[a].data = (const uint8_t *)data[a];
+        lt[a].nbytes = n[a] * esz;
+        lt[a].n_leaves = leaves[a];
+        lt[a].n_full = lt[a].nbytes / chunk_bytes;
+        lt[a].task_begin = task;
+        lt[a].leaf_off = t->off[a];      // level 0 offset of array a
+        task += (leaves[a] + 31) / 32;
+    }
+    QuantParams q;
+    quant_params(eps, &q);
+    ckpt_status st = build_common(t, s, lt.data(), &q, di.sms, nullptr);
+    if (st != CKPT_OK) {
+        ckpt_tree_free_on(t, stream);
+        return st;
+    }
+    *out = t;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_build(const void *data, uint64_t n, ckpt_dtype dtype,
+                                       uint32_t chunk_bytes, double eps, void *stream,
+                                       ckpt_tree **out) {
+    const void *d[1] = {data};
+    uint64_t nn[1] = {n};
+    return ckpt_tree_build_arrays(d, nn, 1, dtype, chunk_bytes, eps, stream, out);
+}
+
+extern "C" ckpt_status ckpt_tree_from_digests(const void *digests16, uint64_t count, void *stream,
+                                              ckpt_tree **out) {
+    if (!out) return fail(CKPT_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!digests16 || count == 0) return fail(CKPT_EINVAL, "no digests");
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    cudaStream_t s = (cudaStream_t)stream;
+    ckpt_tree *t = new ckpt_tree();
+    t->device = dev;
+    t->stream = s;
+    t->from_digests = true;
+    t->chunk_bytes = 16;
+    t->n_elems.assign(1, count);
+    layout(t, std::vector<uint64_t>{count});
+    ckpt_status st = build_common(t, s, nullptr, nullptr, di.sms, digests16);
+    if (st != CKPT_OK) { ckpt_tree_free_on(t, stream); return st; }
+    *out = t;
+    return CKPT_OK;
+}
+
+extern "C" void ckpt_tree_free_on(ckpt_tree *t, void *stream) {
+    if (!t) return;
+    cudaStream_t s = (cudaStream_t)stream;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    if (cur != t->device) cudaSetDevice(t->device);
+    if (t->nodes) cudaFreeAsync(t->nodes, s);
+    if (t->meta) cudaFreeAsync(t->meta, s);
+    if (cur != t->device) cudaSetDevice(cur);
+    delete t;
+}
+
+extern "C" void ckpt_tree_free(ckpt_tree *t) {
+    if (!t) return;
+    ckpt_tree_free_on(t, t->stream);
+}
+
+// ---------------------------------------------------------------------------
+// stage 1: diff (K3)
+// ---------------------------------------------------------------------------
+static ckpt_status check_pair(const ckpt_tree *a, const ckpt_tree *b) {
+    if (!a || !b) return fail(CKPT_EINVAL, "NULL tree");
+    if (a->from_digests || b->from_digests)
+        return fail(CKPT_EINVAL, "trees built from digests cannot be diffed");
+    if (a->dtype != b->dtype || a->chunk_bytes != b->chunk_bytes ||
+        std::memcmp(&a->eps, &b->eps, sizeof(double)) != 0 || a->n_arrays != b->n_arrays ||
+        a->n_elems != b->n_elems)
+        return fail(CKPT_EMISMATCH, "trees differ in dtype, chunk_bytes, eps or array shapes");
+    if (a->device != b->device) return fail(CKPT_EMISMATCH, "trees live on different devices");
+    return CKPT_OK;
+}
+
+static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, const uint8_t *flags,
+                                  uint64_t n, uint64_t *out, uint64_t cap, uint64_t *count,
+                                  cudaStream_t s, int sms) {
+    const uint64_t n_tiles = (n + kCompactTile - 1) / kCompactTile;
+    uint64_t *scratch = nullptr;
+    CK_CUDA(cudaMallocAsync((void **)&scratch, (n_tiles + 1) * 8, s));
+    CK_CUDA(cudaMemsetAsync(scratch, 0, (n_tiles + 1) * 8, s));
+    CompactParams p;
+    p.leaf_a = la;
+    p.leaf_b = lb;
+    p.flags = flags;
+    p.n = n;
+    p.out = out;
+    p.cap = cap;
+    p.count = count;
+    p.states = scratch + 1;
+    p.ticket = (unsigned long long *)scratch;
+    const unsigned grid = (unsigned)std::min<uint64_t>(n_tiles, (uint64_t)sms * 8);
+    ProfScope prof(2, s);
+    if (mode == 0) compact_kernel<0><<<grid, kCompactThreads, 0, s>>>(p);
+    else compact_kernel<1><<<grid, kCompactThreads, 0, s>>>(p);
+    CK_LAUNCH();
+    CK_CUDA(cudaFreeAsync(scratch, s));
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_diff_async(const ckpt_tree *a, const ckpt_tree *b, uint64_t T,
+                                            uint64_t *chunks, uint64_t cap, uint64_t *n_chunks_dev,
+                                            void *stream) {
+    CK_TRY(check_pair(a, b));
+    if (!n_chunks_dev || (!chunks && cap)) return fail(CKPT_EINVAL, "NULL output");
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (T == 0) T = (uint64_t)di.sms * (uint64_t)di.max_threads_sm;
+    const uint32_t na = a->n_arrays;
+    // start level (R16): closest to the root whose node count over all arrays >= T
+    uint32_t l0 = 0;
+    for (int l = (int)a->n_levels - 1; l >= 0; --l) {
+        uint64_t tot = 0;
+        for (uint32_t k = 0; k < na; ++k) {
+            const uint32_t ll = std::min<uint32_t>((uint32_t)l, a->height[k] - 1);
+            tot += a->cnt[(size_t)ll * na + k];
+        }
+        if (tot >= T) { l0 = (uint32_t)l; break; }
+    }
+    if (l0 == 0) {
+        return launch_compact(0, a->nodes, b->nodes, nullptr, a->total_leaves, chunks, cap,
+                              n_chunks_dev, s, di.sms);
+    }
+    // BFS from l0: frontier of (array, level, node) entries
+    std::vector<uint64_t> sbegin(na);
+    std::vector<uint32_t> slevel(na);
+    uint64_t n_start = 0;
+    for (uint32_t k = 0; k < na; ++k) {
+        slevel[k] = std::min<uint32_t>(l0, a->height[k] - 1);
+        sbegin[k] = n_start;
+        n_start += a->cnt[(size_t)slevel[k] * na + k];
+    }
+    const uint64_t L = a->total_leaves;
+    const size_t o_sb = 0;
+    const size_t o_sl = align256(o_sb + (size_t)na * 8);
+    const size_t o_cnt = align256(o_sl + (size_t)na * 4);
+    const size_t o_flags = align256(o_cnt + (size_t)(l0 + 2) * 8);
+    const size_t o_f0 = align256(o_flags + L);
+    const size_t o_f1 = align256(o_f0 + L * 8);
+    const size_t total = align256(o_f1 + L * 8);
+    uint8_t *scr = nullptr;
+    CK_CUDA(cudaMallocAsync((void **)&scr, total, s));
+    std::vector<uint8_t> tbl(o_cnt, 0);
+    std::memcpy(tbl.data() + o_sb, sbegin.data(), (size_t)na * 8);
+    std::memcpy(tbl.data() + o_sl, slevel.data(), (size_t)na * 4);
+    CK_TRY(g_ring.copy(scr, tbl.data(), tbl.size(), s));
+    CK_CUDA(cudaMemsetAsync(scr + o_cnt, 0, o_f0 - o_cnt, s));   // counters + flags
+    BfsParams p;
+    p.na = a->nodes;
+    p.nb = b->nodes;
+    p.off = a->d_off;
+    p.cnt = a->d_cnt;
+    p.chunk_base = a->d_chunk_base;
+    p.sbegin = (const uint64_t *)(scr + o_sb);
+    p.slevel = (const uint32_t *)(scr + o_sl);
+    p.n_start = n_start;
+    p.n_arrays = (int)na;
+    p.flags = scr + o_flags;
+    unsigned long long *cnts = (unsigned long long *)(scr + o_cnt);
+    uint64_t *fr[2] = {(uint64_t *)(scr + o_f0), (uint64_t *)(scr + o_f1)};
+    const unsigned grid_first = (unsigned)std::min<uint64_t>((n_start + 255) / 256, (uint64_t)di.sms * 8);
+    { ProfScope prof(2, s); bfs_first_kernel<<<grid_first, 256, 0, s>>>(p, fr[0], cnts); }
+    CK_LAUNCH();
+    for (uint32_t step = 1; step <= l0; ++step) {
+        ProfScope prof(2, s);
+        bfs_step_kernel<<<(unsigned)di.sms * 8, 256, 0, s>>>(p, fr[(step - 1) & 1], cnts + step - 1,
+                                                            fr[step & 1], cnts + step);
+        CK_LAUNCH();
+    }
+    CK_TRY(launch_compact(1, nullptr, nullptr, scr + o_flags, L, chunks, cap, n_chunks_dev, s, di.sms));
+    CK_CUDA(cudaFreeAsync(scr, s));
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_diff(const ckpt_tree *a, const ckpt_tree *b, uint64_t *chunks,
+                                      uint64_t cap, uint64_t *n_chunks, void *stream) {
+    if (!n_chunks) return fail(CKPT_EINVAL, "n_chunks is NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    uint64_t *dcount = nullptr;
+    CK_TRY(check_pair(a, b));
+    CK_CUDA(cudaMallocAsync((void **)&dcount, 8, s));
+    ckpt_status st = ckpt_tree_diff_async(a, b, 0, chunks, cap, dcount, stream);
+    if (st == CKPT_OK) {
+        CK_CUDA(cudaMemcpyAsync(n_chunks, dcount, 8, cudaMemcpyDeviceToHost, s));
+        CK_CUDA(cudaFreeAsync(dcount, s));
+        CK_CUDA(cudaStreamSynchronize(s));
+        if (*n_chunks > cap) return fail(CKPT_ETRUNC, "chunk list longer than cap");
+        return CKPT_OK;
+    }
+    cudaFreeAsync(dcount, s);
+    return st;
+}
+
+// ---------------------------------------------------------------------------
+// stage 2: verify (K4)
+// ---------------------------------------------------------------------------
+static ckpt_status verify_impl(const void *const *a, const void *const *b, const uint64_t *n,
+                               uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
+                               const uint64_t *chunks, const uint64_t *n_chunks_dev,
+                               uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
+                               uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s) {
+    if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
+    if (!n_diff_dev || (!idx && cap)) return fail(CKPT_EINVAL, "NULL output");
+    CK_TRY(check_common(dtype, chunk_bytes, eps));
+    const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
+    std::vector<VerifyArray> va(na);
+    std::vector<uint64_t> cb(na);
+    uint64_t c = 0, e = 0;
+    for (uint32_t k = 0; k < na; ++k) {
+        if (!a[k] || !b[k]) return fail(CKPT_EINVAL, "NULL data pointer");
+        if ((uintptr_t)a[k] % 16 || (uintptr_t)b[k] % 16)
+            return fail(CKPT_EINVAL, "data must be 16-byte aligned");
+        if (n[k] == 0) return fail(CKPT_EINVAL, "empty array (n == 0)");
+        va[k].a = (const uint8_t *)a[k];
+        va[k].b = (const uint8_t *)b[k];
+        va[k].n = n[k];
+        va[k].chunk_base = c;
+        va[k].elem_base = e;
+        cb[k] = c;
+        c += (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
+        e += n[k];
+    }
+    if (chunks_cap && !chunks) return fail(CKPT_EINVAL, "NULL chunk list");
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c);
+    const uint64_t max_tiles = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
+    const size_t o_va = 0;
+    const size_t o_cb = align256(o_va + (size_t)na * sizeof(VerifyArray));
+    const size_t o_tk = align256(o_cb + (size_t)na * 8);
+    const size_t o_st = o_tk + 8;
+    const size_t total = align256(o_st + (max_tiles + 1) * 8);
+    uint8_t *scr = nullptr;
+    CK_CUDA(cudaMallocAsync((void **)&scr, total, s));
+    std::vector<uint8_t> tbl(o_tk, 0);
+    std::memcpy(tbl.data() + o_va, va.data(), (size_t)na * sizeof(VerifyArray));
+    std::memcpy(tbl.data() + o_cb, cb.data(), (size_t)na * 8);
+    CK_TRY(g_ring.copy(scr, tbl.data(), tbl.size(), s));
+    CK_CUDA(cudaMemsetAsync(scr + o_tk, 0, total - o_tk, s));
+    VerifyParams p;
+    p.arrays = (const VerifyArray *)(scr + o_va);
+    p.chunk_base = (const uint64_t *)(scr + o_cb);
+    p.n_arrays = (int)na;
+    p.chunks = chunks;
+    p.n_chunks_dev = n_chunks_dev;
+    p.n_chunks_host = n_chunks_host;
+    p.chunks_cap = chunks_cap;
+    p.per = chunk_bytes / (uint32_t)esz;
+    p.eps = eps;
+    p.out = idx;
+    p.cap = cap;
+    p.count = n_diff_dev;
+    p.states = (uint64_t *)(scr + o_st);
+    p.ticket = (unsigned long long *)(scr + o_tk);
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * 8));
+    {
+        ProfScope prof(3, s);
+        if (dtype == CKPT_F32) verify_kernel<0><<<grid, kVerifyWarps * 32, 0, s>>>(p);
+        else verify_kernel<1><<<grid, kVerifyWarps * 32, 0, s>>>(p);
+    }
+    CK_LAUNCH();
+    CK_CUDA(cudaFreeAsync(scr, s));
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b,
+                                                const uint64_t *n, uint32_t n_arrays,
+                                                ckpt_dtype dtype, uint32_t chunk_bytes,
+                                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
+                                                uint64_t chunks_cap, double eps, uint64_t *idx,
+                                                uint64_t cap, uint64_t *n_diff_dev, void *stream) {
+    if (!n_chunks_dev) return fail(CKPT_EINVAL, "n_chunks_dev is NULL");
+    return verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, n_chunks_dev, 0, chunks_cap,
+                       eps, idx, cap, n_diff_dev, (cudaStream_t)stream);
+}
+
+extern "C" ckpt_status ckpt_verify(const void *a, const void *b, uint64_t n, ckpt_dtype dtype,
+                                   uint32_t chunk_bytes, const uint64_t *chunks, uint64_t n_chunks,
+                                   double eps, uint64_t *idx, uint64_t cap, uint64_t *n_diff,
+                                   void *stream) {
+    if (!n_diff) return fail(CKPT_EINVAL, "n_diff is NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    const void *pa[1] = {a}, *pb[1] = {b};
+    uint64_t nn[1] = {n};
+    uint64_t *dcount = nullptr;
+    CK_CUDA(cudaMallocAsync((void **)&dcount, 8, s));
+    ckpt_status st = verify_impl(pa, pb, nn, 1, dtype, chunk_bytes, chunks, nullptr, n_chunks,
+                                 n_chunks, eps, idx, cap, dcount, s);
+    if (st != CKPT_OK) { cudaFreeAsync(dcount, s); return st; }
+    CK_CUDA(cudaMemcpyAsync(n_diff, dcount, 8, cudaMemcpyDeviceToHost, s));
+    CK_CUDA(cudaFreeAsync(dcount, s));
+    CK_CUDA(cudaStreamSynchronize(s));
+    if (*n_diff > cap) return fail(CKPT_ETRUNC, "difference list longer than cap");
+    return CKPT_OK;
+}
+
+// ---------------------------------------------------------------------------
+// whole pipeline
+// ---------------------------------------------------------------------------
+extern "C" ckpt_status ckpt_tree_root(const ckpt_tree *t, uint8_t out16[16], void *stream) {
+    if (!t || !out16) return fail(CKPT_EINVAL, "NULL argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    CK_CUDA(cudaMemcpyAsync(out16, t->nodes + t->top_off + t->top_nodes - 1, 16,
+                            cudaMemcpyDeviceToHost, s));
+    CK_CUDA(cudaStreamSynchronize(s));
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_compare(const void *const *a, const void *const *b, const uint64_t *n,
+                                    uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                    double eps, uint64_t *chunks, uint64_t chunks_cap,
+                                    uint64_t *idx, uint64_t idx_cap, uint64_t *n_chunks,
+                                    uint64_t *n_diff, uint8_t *root_a16, uint8_t *root_b16,
+                                    void *stream) {
+    if (!n_chunks || !n_diff) return fail(CKPT_EINVAL, "NULL count output");
+    cudaStream_t s = (cudaStream_t)stream;
+    ckpt_tree *ta = nullptr, *tb = nullptr;
+    uint64_t *dc = nullptr;
+    ckpt_status st = ckpt_tree_build_arrays(a, n, n_arrays, dtype, chunk_bytes, eps, stream, &ta);
+    if (st == CKPT_OK) st = ckpt_tree_build_arrays(b, n, n_arrays, dtype, chunk_bytes, eps, stream, &tb);
+    if (st == CKPT_OK && cudaMallocAsync((void **)&dc, 16, s) != cudaSuccess)
+        st = fail(CKPT_ENOMEM, "count scratch");
+    if (st == CKPT_OK) st = ckpt_tree_diff_async(ta, tb, 0, chunks, chunks_cap, dc, stream);
+    if (st == CKPT_OK)
+        st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, dc, 0, chunks_cap, eps, idx,
+                         idx_cap, dc + 1, s);
+    uint64_t hc[2] = {0, 0};
+    if (st == CKPT_OK && cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+        st = fail(CKPT_ECUDA, "count copy");
+    if (st == CKPT_OK && root_a16) st = ckpt_tree_root(ta, root_a16, stream);
+    if (st == CKPT_OK && root_b16) st = ckpt_tree_root(tb, root_b16, stream);
+    if (st == CKPT_OK && cudaStreamSynchronize(s) != cudaSuccess) st = fail(CKPT_ECUDA, "sync");
+    if (dc) cudaFreeAsync(dc, s);
+    ckpt_tree_free_on(ta, stream);
+    ckpt_tree_free_on(tb, stream);
+    if (st != CKPT_OK) return st;
+    *n_chunks = hc[0];
+    *n_diff = hc[1];
+    if (hc[0] > chunks_cap || hc[1] > idx_cap) return fail(CKPT_ETRUNC, "output longer than cap");
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_compare_host(const void *const *a, const void *const *b,
+                                         const uint64_t *n, uint32_t n_arrays, ckpt_dtype dtype,
+                                         uint32_t chunk_bytes, double eps, uint64_t *idx,
+                                         uint64_t idx_cap, uint64_t *n_chunks, uint64_t *n_diff,
+                                         uint8_t *root_a16, uint8_t *root_b16) {
+    if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
+    if (!n_chunks || !n_diff || (!idx && idx_cap)) return fail(CKPT_EINVAL, "NULL output");
+    CK_TRY(check_common(dtype, chunk_bytes, eps));
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
+    uint64_t L = 0;
+    for (uint32_t k = 0; k < n_arrays; ++k) {
+        if (!a[k] || !b[k] || n[k] == 0) return fail(CKPT_EINVAL, "NULL or empty array");
+        L += (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
+    }
+    cudaStream_t sc = nullptr, sk = nullptr;
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+    CK_CUDA(cudaStreamCreateWithFlags(&sc, cudaStreamNonBlocking));
+    CK_CUDA(cudaStreamCreateWithFlags(&sk, cudaStreamNonBlocking));
+    CK_CUDA(cudaEventCreateWithFlags(&ev_a, cudaEventDisableTiming));
+    CK_CUDA(cudaEventCreateWithFlags(&ev_b, cudaEventDisableTiming));
+    std::vector<void *> da(n_arrays, nullptr), db(n_arrays, nullptr);
+    ckpt_tree *ta = nullptr, *tb = nullptr;
+    uint64_t *dchunks = nullptr, *didx = nullptr, *dc = nullptr;
+    ckpt_status st = CKPT_OK;
+    auto cu = [&](cudaError_t e, const char *what) {
+        if (st == CKPT_OK && e != cudaSuccess)
+            st = fail(e == cudaErrorMemoryAllocation ? CKPT_ENOMEM : CKPT_ECUDA,
+                      std::string(what) + ": " + cudaGetErrorString(e));
+    };
+    for (uint32_t k = 0; k < n_arrays && st == CKPT_OK; ++k) {
+        cu(cudaMallocAsync(&da[k], n[k] * esz, sc), "alloc A");
+        cu(cudaMallocAsync(&db[k], n[k] * esz, sc), "alloc B");
+    }
+    for (uint32_t k = 0; k < n_arrays && st == CKPT_OK; ++k)
+        cu(cudaMemcpyAsync(da[k], a[k], n[k] * esz, cudaMemcpyHostToDevice, sc), "H2D A");
+    cu(cudaEventRecord(ev_a, sc), "event");
+    for (uint32_t k = 0; k < n_arrays && st == CKPT_OK; ++k)
+        cu(cudaMemcpyAsync(db[k], b[k], n[k] * esz, cudaMemcpyHostToDevice, sc), "H2D B");
+    cu(cudaEventRecord(ev_b, sc), "event");
+    cu(cudaMallocAsync((void **)&dchunks, L * 8, sk), "alloc chunks");
+    cu(cudaMallocAsync((void **)&didx, std::max<uint64_t>(idx_cap, 1) * 8, sk), "alloc idx");
+    cu(cudaMallocAsync((void **)&dc, 16, sk), "alloc counts");
+    cu(cudaStreamWaitEvent(sk, ev_a, 0), "wait A");
+    if (st == CKPT_OK)
+        st = ckpt_tree_build_arrays(da.data(), n, n_arrays, dtype, chunk_bytes, eps, sk, &ta);
+    cu(cudaStreamWaitEvent(sk, ev_b, 0), "wait B");
+    if (st == CKPT_OK)
+        st = ckpt_tree_build_arrays(db.data(), n, n_arrays, dtype, chunk_bytes, eps, sk, &tb);
+    if (st == CKPT_OK) st = ckpt_tree_diff_async(ta, tb, 0, dchunks, L, dc, sk);
+    if (st == CKPT_OK)
+        st = verify_impl(da.data(), db.data(), n, n_arrays, dtype, chunk_bytes, dchunks, dc, 0, L,
+                         eps, didx, idx_cap, dc + 1, sk);
+    uint64_t hc[2] = {0, 0};
+    cu(cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, sk), "D2H counts");
+    cu(cudaStreamSynchronize(sk), "sync");
+    if (st == CKPT_OK && idx_cap && hc[1])
+        cu(cudaMemcpyAsync(idx, didx, std::min(hc[1], idx_cap) * 8, cudaMemcpyDeviceToHost, sk), "D2H idx");
+    if (st == CKPT_OK && root_a16) st = ckpt_tree_root(ta, root_a16, sk);
+    if (st == CKPT_OK && root_b16) st = ckpt_tree_root(tb, root_b16, sk);
+    ckpt_tree_free_on(ta, sk);
+    ckpt_tree_free_on(tb, sk);
+    for (uint32_t k = 0; k < n_arrays; ++k) {
+        if (da[k]) cudaFreeAsync(da[k], sk);
+        if (db[k]) cudaFreeAsync(db[k], sk);
+    }
+    if (dchunks) cudaFreeAsync(dchunks, sk);
+    if (didx) cudaFreeAsync(didx, sk);
+    if (dc) cudaFreeAsync(dc, sk);
+    cudaStreamSynchronize(sk);
+    cudaStreamSynchronize(sc);
+    cudaEventDestroy(ev_a);
+    cudaEventDestroy(ev_b);
+    cudaStreamDestroy(sc);
+    cudaStreamDestroy(sk);
+    if (st != CKPT_OK) return st;
+    *n_chunks = hc[0];
+    *n_diff = hc[1];
+    if (hc[1] > idx_cap) return fail(CKPT_ETRUNC, "difference list longer than cap");
+    return CKPT_OK;
+}
+
+// ---------------------------------------------------------------------------
+// accessors
+// ---------------------------------------------------------------------------
+extern "C" ckpt_status ckpt_tree_info(const ckpt_tree *t, uint32_t *n_arrays, uint64_t *n_leaves,
+                                      uint32_t *n_levels, uint64_t *n_nodes) {
+    if (!t) return fail(CKPT_EINVAL, "NULL tree");
+    if (n_arrays) *n_arrays = t->n_arrays;
+    if (n_leaves) *n_leaves = t->total_leaves;
+    if (n_levels) *n_levels = t->n_levels;
+    if (n_nodes) *n_nodes = t->array_nodes;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_array_roots(const ckpt_tree *t, void *dst, void *stream) {
+    if (!t || !dst) return fail(CKPT_EINVAL, "NULL argument");
+    CK_CUDA(cudaMemcpyAsync(dst, t->nodes + t->top_off, (size_t)t->n_arrays * 16,
+                            cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_array_info(const ckpt_tree *t, uint32_t array, uint64_t *n_leaves,
+                                            uint64_t *n_nodes) {
+    if (!t || array >= t->n_arrays) return fail(CKPT_EINVAL, "bad tree or array index");
+    uint64_t tot = 0;
+    for (uint32_t l = 0; l < t->height[array]; ++l) tot += t->cnt[(size_t)l * t->n_arrays + array];
+    if (n_leaves) *n_leaves = t->n_leaves[array];
+    if (n_nodes) *n_nodes = tot;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_nodes(const ckpt_tree *t, uint32_t array, void *dst,
+                                       uint64_t cap_bytes, void *stream) {
+    uint64_t nn = 0;
+    CK_TRY(ckpt_tree_array_info(t, array, nullptr, &nn));
+    if (!dst || cap_bytes < nn * 16) return fail(CKPT_EINVAL, "destination too small");
+    uint8_t *d = (uint8_t *)dst;
+    for (uint32_t l = 0; l < t->height[array]; ++l) {
+        const size_t i = (size_t)l * t->n_arrays + array;
+        CK_CUDA(cudaMemcpyAsync(d, t->nodes + t->off[i], t->cnt[i] * 16, cudaMemcpyDeviceToDevice,
+                                (cudaStream_t)stream));
+        d += t->cnt[i] * 16;
+    }
+    return CKPT_OK;
+}
+
+extern "C" uint64_t ckpt_default_bfs_threshold(void) {
+    int dev;
+    DevInfo di;
+    if (dev_info(&dev, &di) != CKPT_OK) return 0;
+    return (uint64_t)di.sms * (uint64_t)di.max_threads_sm;
+}
+
+extern "C" uint64_t ckpt_launch_count(void) { return g_launches.load(); }
+
+extern "C" const char *ckpt_strerror(ckpt_status s) {
+    switch (s) {
+        case CKPT_OK: return "ok";
+        case CKPT_EINVAL: return "invalid argument";
+        case CKPT_EMISMATCH: return "trees do not match in shape or parameters";
+        case CKPT_ENOMEM: return "out of device memory";
+        case CKPT_ECUDA: return "CUDA error";
+        case CKPT_ETRUNC: return "output truncated to capacity";
+    }
+    return "unknown status";
+}
+
+extern "C" const char *ckpt_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" uint32_t ckpt_version(void) { return (1u << 16) | 0u; }
+
+extern "C" void ckpt_profile_enable(int on) { g_prof_on.store(on ? 1 : 0); }
+
+extern "C" void ckpt_profile_reset(void) {
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    for (auto &r : g_prof) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+    g_prof.clear();
+}
+
+extern "C" ckpt_status ckpt_profile_read(int k, double *ms, uint64_t *launches) {
+    if (!ms || !launches) return fail(CKPT_EINVAL, "NULL output");
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    double tot = 0.0;
+    uint64_t n = 0;
+    for (auto &r : g_prof) {
+        if (r.k != k) continue;
+        CK_CUDA(cudaEventSynchronize(r.b));
+        float e = 0.f;
+        CK_CUDA(cudaEventElapsedTime(&e, r.a, r.b));
+        tot += e;
+        ++n;
+    }
+    *ms = tot;
+    *launches = n;
+    return CKPT_OK;
+}

@@ -1,0 +1,388 @@
+// compare.cuh -- K3 (BFS diff, P:555-566 / P:642-648) and K4 (verify).
+//
+// Both emit unique ascending ids (reading R17) with a single-pass ordered
+// compaction: each CTA takes tiles in order from an atomic ticket, counts its
+// hits with __ballot_sync/__popc, publishes the tile aggregate and looks back
+// over its predecessors (decoupled look-back) for its exclusive prefix, then
+// writes its hits at their final positions.  Persistent grids, so the item
+// counts may live on the device (no host round trip between steps).
+#pragma once
+#include <cstdint>
+
+#include "hash.cuh"
+
+namespace ckpt {
+
+constexpr unsigned kFull = 0xffffffffu;
+constexpr uint64_t kFlagA = 1ull << 62;     // tile aggregate available
+constexpr uint64_t kFlagP = 1ull << 63;     // inclusive prefix available
+constexpr uint64_t kValMask = kFlagA - 1;
+
+__device__ __forceinline__ uint64_t ld_volatile(const uint64_t *p) {
+    return *reinterpret_cast<const volatile uint64_t *>(p);
+}
+__device__ __forceinline__ void st_volatile(uint64_t *p, uint64_t v) {
+    *reinterpret_cast<volatile uint64_t *>(p) = v;
+}
+
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    return v;
+}
+
+__device__ __forceinline__ uint32_t warp_excl_scan_u32(uint32_t v, int lane, uint32_t &total) {
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+    }
+    total = __shfl_sync(kFull, x, 31);
+    return x - v;
+}
+
+// Called by one full warp.  Returns the exclusive prefix of `tile`.
+__device__ uint64_t tile_lookback(uint64_t *states, uint64_t tile, uint64_t aggregate, int lane) {
+    if (tile == 0) {
+        if (lane == 0) st_volatile(&states[0], kFlagP | aggregate);
+        return 0;
+    }
+    if (lane == 0) st_volatile(&states[tile], kFlagA | aggregate);
+    uint64_t excl = 0;
+    int64_t pred = (int64_t)tile - 1;
+    for (;;) {
+        const int64_t idx = pred - lane;
+        uint64_t s;
+        do {
+            s = idx >= 0 ? ld_volatile(&states[idx]) : kFlagP;
+        } while (__any_sync(kFull, s == 0));
+        const uint32_t pm = __ballot_sync(kFull, (s & kFlagP) != 0);
+        const int stop = pm ? __ffs(pm) - 1 : 31;
+        excl += warp_sum_u64(lane <= stop ? (s & kValMask) : 0);
+        if (pm) break;
+        pred -= 32;
+    }
+    if (lane == 0) st_volatile(&states[tile], kFlagP | (excl + aggregate));
+    return excl;
+}
+
+// ---------------------------------------------------------------------------
+// ordered compaction over [0, n): pred = leaf digests differ (MODE 0) or a
+// flag byte is set (MODE 1).  Output value = item index (a global chunk id).
+// ---------------------------------------------------------------------------
+constexpr int kCompactThreads = 256;
+constexpr int kCompactRows = 16;                          // rows of 32 items per warp
+constexpr int kCompactTile = kCompactThreads * kCompactRows;  // 4096 items
+
+struct CompactParams {
+    const uint4 *leaf_a;
+    const uint4 *leaf_b;
+    const uint8_t *flags;
+    uint64_t n;
+    uint64_t *out;
+    uint64_t cap;
+    uint64_t *count;          // device: total hits
+    uint64_t *states;         // zeroed, >= n_tiles entries
+    unsigned long long *ticket;  // zeroed
+};
+
+template <int MODE>
+__global__ void __launch_bounds__(kCompactThreads) compact_kernel(CompactParams p) {
+    __shared__ uint32_t row_cnt[kCompactRows * 8];
+    __shared__ uint32_t row_off[kCompactRows * 8];
+    __shared__ uint64_t s_excl;
+    __shared__ uint64_t s_tile;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t n_tiles = (p.n + kCompactTile - 1) / kCompactTile;
+    for (;;) {
+        if (threadIdx.x == 0) s_tile = atomicAdd(p.ticket, 1ull);
+        __syncthreads();
+        const uint64_t tile = s_tile;
+        if (tile >= n_tiles) return;
+        const uint64_t t0 = tile * kCompactTile;
+        uint32_t bits[kCompactRows];
+#pragma unroll
+        for (int k = 0; k < kCompactRows; ++k) {
+            const uint64_t i = t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
+            bool hit = false;
+            if (i < p.n) {
+                if (MODE == 0) hit = digest_ne(p.leaf_a[i], p.leaf_b[i]);
+                else hit = p.flags[i] != 0;
+            }
+            bits[k] = __ballot_sync(kFull, hit);
+            if (lane == 0) row_cnt[k * 8 + warp] = __popc(bits[k]);
+        }
+        __syncthreads();
+        if (warp == 0) {
+            // rows in item order: k major, warp minor -> flat index k*8+warp
+            uint32_t v[4], s = 0;
+#pragma unroll
+            for (int r = 0; r < 4; ++r) { v[r] = row_cnt[lane * 4 + r]; s += v[r]; }
+            uint32_t total;
+            uint32_t ex = warp_excl_scan_u32(s, lane, total);
+#pragma unroll
+            for (int r = 0; r < 4; ++r) { row_off[lane * 4 + r] = ex; ex += v[r]; }
+            const uint64_t excl = tile_lookback(p.states, tile, total, lane);
+            if (lane == 0) {
+                s_excl = excl;
+                if (tile == n_tiles - 1) *p.count = excl + total;
+            }
+        }
+        __syncthreads();
+        const uint64_t excl = s_excl;
+        const uint32_t lt = (1u << lane) - 1u;
+#pragma unroll
+        for (int k = 0; k < kCompactRows; ++k) {
+            if (bits[k] & (1u << lane)) {
+                const uint64_t pos = excl + row_off[k * 8 + warp] + __popc(bits[k] & lt);
+                if (pos < p.cap) p.out[pos] = t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------
+// BFS steps for a start level above the leaves.
+// Frontier entry: array (20 bits) | level (6 bits) | node (38 bits).
+// ---------------------------------------------------------------------------
+struct BfsParams {
+    const uint4 *na;
+    const uint4 *nb;
+    const uint64_t *off;          // [level * n_arrays + a]
+    const uint64_t *cnt;
+    const uint64_t *chunk_base;   // [a] global chunk id of array a's leaf 0
+    const uint64_t *sbegin;       // [a] prefix of start-level node counts (first step)
+    const uint32_t *slevel;       // [a] start level of array a
+    uint64_t n_start;             // total start-level nodes
+    int n_arrays;
+    uint8_t *flags;               // [total leaves] zeroed
+};
+
+__device__ __forceinline__ uint64_t pack_entry(uint64_t a, uint64_t l, uint64_t j) {
+    return (a << 44) | (l << 38) | j;
+}
+
+__device__ __forceinline__ int find_u64(const uint64_t *v, int n, uint64_t x) {
+    int lo = 0, hi = n - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (v[mid] <= x) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+// Compare node (a,l,j); unequal leaves set their flag, unequal inner nodes
+// push their children (warp-aggregated append).
+__device__ __forceinline__ void bfs_visit(const BfsParams &p, bool valid, uint64_t a, uint64_t l,
+                                          uint64_t j, uint64_t *out, unsigned long long *out_cnt,
+                                          int lane) {
+    uint32_t nchild = 0;
+    uint64_t c0 = 0;
+    if (valid) {
+        const uint64_t o = p.off[l * p.n_arrays + a] + j;
+        if (digest_ne(p.na[o], p.nb[o])) {
+            if (l == 0) {
+                p.flags[p.chunk_base[a] + j] = 1;
+            } else {
+                const uint64_t nd = p.cnt[(l - 1) * p.n_arrays + a];
+                c0 = pack_entry(a, l - 1, 2 * j);
+                nchild = (2 * j + 1 < nd) ? 2u : 1u;
+            }
+        }
+    }
+    uint32_t total;
+    const uint32_t ex = warp_excl_scan_u32(nchild, lane, total);
+    if (total == 0) return;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(out_cnt, (unsigned long long)total);
+    base = __shfl_sync(kFull, base, 0);
+    for (uint32_t c = 0; c < nchild; ++c) out[base + ex + c] = c0 + c;
+}
+
+__global__ void bfs_first_kernel(BfsParams p, uint64_t *out, unsigned long long *out_cnt) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < p.n_start; base += stride) {
+        const uint64_t i = base + threadIdx.x;
+        const bool valid = i < p.n_start;
+        uint64_t a = 0, l = 0, j = 0;
+        if (valid) {
+            a = (uint64_t)find_u64(p.sbegin, p.n_arrays, i);
+            l = p.slevel[a];
+            j = i - p.sbegin[a];
+        }
+        bfs_visit(p, valid, a, l, j, out, out_cnt, lane);
+    }
+}
+
+__global__ void bfs_step_kernel(BfsParams p, const uint64_t *in, const unsigned long long *in_cnt,
+                                uint64_t *out, unsigned long long *out_cnt) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t n = *in_cnt;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+        const uint64_t i = base + threadIdx.x;
+        const bool valid = i < n;
+        uint64_t a = 0, l = 0, j = 0;
+        if (valid) {
+            const uint64_t e = in[i];
+            a = e >> 44;
+            l = (e >> 38) & 63;
+            j = e & ((1ull << 38) - 1);
+        }
+        bfs_visit(p, valid, a, l, j, out, out_cnt, lane);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// K4 verify: one warp per listed chunk, 8 chunks per tile.
+// ---------------------------------------------------------------------------
+constexpr int kVerifyWarps = 8;
+
+struct VerifyArray {
+    const uint8_t *a;
+    const uint8_t *b;
+    uint64_t n;            // elements
+    uint64_t chunk_base;   // global chunk id of local chunk 0
+    uint64_t elem_base;    // global element id of local element 0
+};
+
+struct VerifyParams {
+    const VerifyArray *arrays;
+    const uint64_t *chunk_base;   // [a] copy of arrays[a].chunk_base for the search
+    int n_arrays;
+    const uint64_t *chunks;
+    const uint64_t *n_chunks_dev; // may be null -> n_chunks_host
+    uint64_t n_chunks_host;
+    uint64_t chunks_cap;
+    uint32_t per;                 // elements per chunk
+    double eps;
+    uint64_t *out;
+    uint64_t cap;
+    uint64_t *count;
+    uint64_t *states;
+    unsigned long long *ticket;
+};
+
+// 16-byte vector of elements starting at element e (e % VEC == 0); bits of
+// |a-b| > eps for the elements < len.
+template <int DT>
+__device__ __forceinline__ uint32_t diff_bits(const uint8_t *pa, const uint8_t *pb, uint64_t e,
+                                              uint64_t len, double eps) {
+    constexpr int VEC = DT == 0 ? 4 : 2;
+    uint32_t m = 0;
+    if (e + VEC <= len) {
+        const uint4 va = __ldg(reinterpret_cast<const uint4 *>(pa) + e / VEC);
+        const uint4 vb = __ldg(reinterpret_cast<const uint4 *>(pb) + e / VEC);
+        if (DT == 0) {
+            m |= (fabs((double)__uint_as_float(va.x) - (double)__uint_as_float(vb.x)) > eps) ? 1u : 0u;
+            m |= (fabs((double)__uint_as_float(va.y) - (double)__uint_as_float(vb.y)) > eps) ? 2u : 0u;
+            m |= (fabs((double)__uint_as_float(va.z) - (double)__uint_as_float(vb.z)) > eps) ? 4u : 0u;
+            m |= (fabs((double)__uint_as_float(va.w) - (double)__uint_as_float(vb.w)) > eps) ? 8u : 0u;
+        } else {
+            const double a0 = __hiloint2double((int)va.y, (int)va.x), b0 = __hiloint2double((int)vb.y, (int)vb.x);
+            const double a1 = __hiloint2double((int)va.w, (int)va.z), b1 = __hiloint2double((int)vb.w, (int)vb.z);
+            m |= (fabs(a0 - b0) > eps) ? 1u : 0u;
+            m |= (fabs(a1 - b1) > eps) ? 2u : 0u;
+        }
+    } else {
+        for (int v = 0; v < VEC; ++v) {
+            if (e + v >= len) break;
+            double x, y;
+            if (DT == 0) {
+                x = (double)reinterpret_cast<const float *>(pa)[e + v];
+                y = (double)reinterpret_cast<const float *>(pb)[e + v];
+            } else {
+                x = reinterpret_cast<const double *>(pa)[e + v];
+                y = reinterpret_cast<const double *>(pb)[e + v];
+            }
+            if (fabs(x - y) > eps) m |= 1u << v;
+        }
+    }
+    return m;
+}
+
+template <int DT>
+__global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams p) {
+    constexpr int VEC = DT == 0 ? 4 : 2;
+    constexpr int ESZ = DT == 0 ? 4 : 8;
+    __shared__ uint32_t w_cnt[kVerifyWarps];
+    __shared__ uint64_t s_excl;
+    __shared__ uint64_t s_tile;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint64_t n_chunks = p.n_chunks_dev ? *p.n_chunks_dev : p.n_chunks_host;
+    if (n_chunks > p.chunks_cap) n_chunks = p.chunks_cap;
+    const uint64_t n_tiles = (n_chunks + kVerifyWarps - 1) / kVerifyWarps;
+    if (n_tiles == 0) {
+        if (blockIdx.x == 0 && threadIdx.x == 0) *p.count = 0;
+        return;
+    }
+    const uint32_t lt = (1u << lane) - 1u;
+    for (;;) {
+        if (threadIdx.x == 0) s_tile = atomicAdd(p.ticket, 1ull);
+        __syncthreads();
+        const uint64_t tile = s_tile;
+        if (tile >= n_tiles) return;
+        const uint64_t q = tile * kVerifyWarps + warp;
+        const bool have = q < n_chunks;
+        const uint8_t *pa = nullptr, *pb = nullptr;
+        uint64_t e_begin = 0, len = 0, gbase = 0;
+        if (have) {
+            const uint64_t g = p.chunks[q];
+            const int a = find_u64(p.chunk_base, p.n_arrays, g);
+            const VerifyArray A = p.arrays[a];
+            const uint64_t c = g - A.chunk_base;
+            e_begin = c * p.per;
+            const uint64_t e_end = (e_begin + p.per) < A.n ? (e_begin + p.per) : A.n;
+            len = e_end > e_begin ? e_end - e_begin : 0;
+            pa = A.a + e_begin * ESZ;
+            pb = A.b + e_begin * ESZ;
+            gbase = A.elem_base + e_begin;
+        }
+        // pass 1: count
+        uint32_t cnt = 0;
+        constexpr int kStep = 32 * VEC;
+#pragma unroll 4
+        for (uint64_t e = (uint64_t)lane * VEC; e < len; e += kStep)
+            cnt += __popc(diff_bits<DT>(pa, pb, e, len, p.eps));
+        cnt = (uint32_t)warp_sum_u64(cnt);
+        if (lane == 0) w_cnt[warp] = cnt;
+        __syncthreads();
+        if (warp == 0) {
+            const uint32_t v = lane < kVerifyWarps ? w_cnt[lane] : 0u;
+            uint32_t total;
+            const uint32_t ex = warp_excl_scan_u32(v, lane, total);
+            if (lane < kVerifyWarps) w_cnt[lane] = ex;
+            const uint64_t excl = tile_lookback(p.states, tile, total, lane);
+            if (lane == 0) {
+                s_excl = excl;
+                if (tile == n_tiles - 1) *p.count = excl + total;
+            }
+        }
+        __syncthreads();
+        // pass 2: emit (only chunks with hits re-read their data)
+        if (cnt) {
+            uint64_t pos = s_excl + w_cnt[warp];
+            for (uint64_t e0 = 0; e0 < len; e0 += kStep) {
+                const uint64_t e = e0 + (uint64_t)lane * VEC;
+                const uint32_t m = e < len ? diff_bits<DT>(pa, pb, e, len, p.eps) : 0u;
+                uint32_t total;
+                const uint32_t ex = warp_excl_scan_u32(__popc(m), lane, total);
+                uint32_t mm = m, k = 0;
+                while (mm) {
+                    const int bit = __ffs(mm) - 1;
+                    mm &= mm - 1;
+                    const uint64_t o = pos + ex + k++;
+                    if (o < p.cap) p.out[o] = gbase + e + bit;
+                }
+                pos += total;
+            }
+        }
+        (void)lt;
+        __syncthreads();
+    }
+}
+
+}  // namespace ckpt

@@ -1,0 +1,318 @@
+"""GPU parity: libckpt (CUDA sm_100a, via the C ABI) vs the CPU oracle, bit-exact.
+
+Covers leaves, every tree node, roots, chunk lists, element ids and counts on
+seeded synthetic checkpoints (synth), ragged/partial sizes, special values,
+every BFS start level, truncation and error paths.  Full-size (BASELINE
+configs[1]) checks sample leaves and recompute levels/verify with the oracle.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+ck = pytest.importorskip("paper_conf_middleware_tanaabcrtn24_b200")
+
+
+def np_of(t):
+    return t.detach().cpu().numpy()
+
+
+def gpu_tree_nodes(tree, array=0):
+    return np_of(tree.nodes(array))
+
+
+def oracle_tree(a_np, chunk, eps):
+    lv = oracle.leaves(a_np, chunk, eps, threads=8)
+    return oracle.levels(lv), lv.shape[0]
+
+
+# ------------------------------------------------------------ leaves/trees --
+
+CASES = [
+    # (n, dtype, chunk, eps)
+    (1, torch.float32, 16, 1e-3),
+    (3, torch.float32, 16, 1e-3),        # partial block only
+    (5, torch.float32, 16, 1e-3),
+    (1000, torch.float32, 48, 1e-4),     # runtime chunk size, not a multiple of 64
+    (1025, torch.float32, 64, 1e-4),     # tail block of 4 bytes
+    (4097, torch.float32, 512, 1e-5),
+    (100_003, torch.float32, 4096, 1e-6),
+    ((1 << 20), torch.float32, 4096, 1e-5),   # config 1
+    (1_000_000, torch.float32, 4096, 1e-5),   # config 1 tail case
+    (70_001, torch.float32, 65536, 1e-3),
+    (3, torch.float64, 16, 1e-3),
+    (999, torch.float64, 32, 1e-7),
+    (123_457, torch.float64, 1024, 1e-8),
+    (50_000, torch.float64, 8192, 1e-3),
+    (10_000, torch.float32, 4096, 0.0),       # raw-bit mode (R10)
+    (10_001, torch.float64, 160, 0.0),
+]
+
+
+def _data(n, dtype, seed):
+    if dtype == torch.float32:
+        return synth.uniform(seed, n, "cuda") * 2.0 - 1.0
+    return synth.normal(seed, n, "cuda", dtype=torch.float64)
+
+
+@pytest.mark.parametrize("n,dtype,chunk,eps", CASES)
+def test_tree_bit_exact(n, dtype, chunk, eps):
+    a = _data(n, dtype, n + chunk)
+    t = ck.tree_build(a, chunk, eps)
+    got = gpu_tree_nodes(t)
+    ref, L = oracle_tree(np_of(a), chunk, eps)
+    assert got.shape == ref.shape
+    bad = np.nonzero(np.any(got != ref, axis=1))[0]
+    assert bad.size == 0, f"{bad.size} nodes differ, first {bad[:5]}"
+    assert t.root() == ref[-1].tobytes()
+    assert t.n_leaves == L
+
+
+SPECIALS32 = np.array([0.0, -0.0, np.inf, -np.inf, np.nan, 1e-45, -1e-45, 1.17549435e-38,
+                       -1.17549435e-38, 3.4028235e38, -3.4028235e38, 1.0, -1.0, 0.5, -0.5,
+                       2.0 ** 24, -(2.0 ** 24), 2.0 ** 31, 2.0 ** 40, -(2.0 ** 60), 1e-5, -1e-5,
+                       2.0 ** 51 * 1e-6, -(2.0 ** 51) * 1e-6, 2.0 ** 63 * 1e-6], dtype=np.float32)
+
+
+@pytest.mark.parametrize("eps", [1e-3, 1e-5, 1e-6, 1e-8, 2.0 ** -10, 0.3, 7.0, 1e-30, 1e30])
+def test_quantizer_specials_and_random_bit_patterns_f32(eps):
+    rng = np.random.default_rng(int(eps * 1e9) % 1000 + 1)
+    bits = rng.integers(0, 2 ** 32, size=1 << 20, dtype=np.uint64).astype(np.uint32)
+    x = bits.view(np.float32).copy()
+    x[: SPECIALS32.size] = SPECIALS32
+    x[SPECIALS32.size: 2 * SPECIALS32.size] = np.nextafter(SPECIALS32, np.float32(0))
+    # chunk = one block: every leaf pins 4 words
+    a = torch.from_numpy(x).cuda()
+    t = ck.tree_build(a, 16, eps)
+    got = gpu_tree_nodes(t)[: x.size // 4]
+    ref = oracle.leaves(x, 16, eps, threads=8)
+    bad = np.nonzero(np.any(got != ref, axis=1))[0]
+    assert bad.size == 0, (bad[:5], x.reshape(-1, 4)[bad[:5]])
+
+
+@pytest.mark.parametrize("eps", [1e-3, 1e-6, 1e-8, 2.0 ** -10, 1e-300, 1e300])
+def test_quantizer_specials_and_random_bit_patterns_f64(eps):
+    rng = np.random.default_rng(5)
+    bits = rng.integers(0, 2 ** 63, size=1 << 19, dtype=np.uint64) * 2 + rng.integers(0, 2, 1 << 19, dtype=np.uint64)
+    x = bits.view(np.float64).copy()
+    sp = np.array([0.0, -0.0, np.inf, -np.inf, np.nan, 5e-324, -5e-324, 2.0 ** 62, -(2.0 ** 62),
+                   2.0 ** 63, -(2.0 ** 63), 1.7976931348623157e308, -1.7976931348623157e308,
+                   1.0, -1.0, 1e-5, -1e-5, 2.0 ** 51 * eps, -(2.0 ** 51) * eps, 2.0 ** 63 * eps,
+                   -(2.0 ** 63) * eps, np.nextafter(2.0 ** 63 * eps, 0)], dtype=np.float64)
+    x[: sp.size] = sp
+    # also values near the fast/slow-path boundary |x| ~ 2^50 * eps
+    x[sp.size: sp.size + 1000] = rng.uniform(-(2.0 ** 52), 2.0 ** 52, 1000) * eps
+    a = torch.from_numpy(x).cuda()
+    t = ck.tree_build(a, 16, eps)
+    got = gpu_tree_nodes(t)[: x.size // 2]
+    ref = oracle.leaves(x, 16, eps, threads=8)
+    bad = np.nonzero(np.any(got != ref, axis=1))[0]
+    assert bad.size == 0, (bad[:5], x.reshape(-1, 2)[bad[:5]])
+
+
+def test_near_boundary_f32_values():
+    # values whose x*inv is within a few ulps of an integer (the floor decision)
+    eps = 1e-5
+    k = np.arange(-200000, 200000, 7, dtype=np.float64)
+    base = (k * eps).astype(np.float32)
+    x = np.concatenate([base, np.nextafter(base, np.float32(np.inf)),
+                        np.nextafter(base, np.float32(-np.inf))])
+    x = x[: (x.size // 4) * 4]
+    a = torch.from_numpy(x).cuda()
+    t = ck.tree_build(a, 16, eps)
+    got = gpu_tree_nodes(t)[: x.size // 4]
+    ref = oracle.leaves(x, 16, eps, threads=8)
+    assert np.array_equal(got, ref)
+
+
+# ---------------------------------------------------------- multi-array --
+
+def test_multi_array_checkpoint_matches_oracle():
+    sizes = [1000, 1, 4097, 333, 65536, 12345]
+    arrs_a = [_data(n, torch.float32, 100 + i) for i, n in enumerate(sizes)]
+    arrs_b = [t.clone() for t in arrs_a]
+    arrs_b[2][4096] += 1.0
+    arrs_b[4][7] += 1e-3
+    chunk, eps = 256, 1e-4
+    TA = ck.tree_build(arrs_a, chunk, eps)
+    TB = ck.tree_build(arrs_b, chunk, eps)
+    A = oracle.build_checkpoint([np_of(t) for t in arrs_a], chunk, eps)
+    B = oracle.build_checkpoint([np_of(t) for t in arrs_b], chunk, eps)
+    for k in range(len(sizes)):
+        assert np.array_equal(gpu_tree_nodes(TA, k), A.trees[k])
+        assert np.array_equal(gpu_tree_nodes(TB, k), B.trees[k])
+    assert np.array_equal(np_of(TA.array_roots()), A.array_roots)
+    assert TA.root() == A.root and TB.root() == B.root
+    chunks = ck.tree_diff(TA, TB)
+    assert np.array_equal(np_of(chunks), oracle.diff_checkpoint(A, B))
+    idx, n = ck.verify(arrs_a, arrs_b, chunks, chunk, eps)
+    ref = oracle.verify_checkpoint([np_of(t) for t in arrs_a], [np_of(t) for t in arrs_b], chunk,
+                                   np_of(chunks), eps, A)
+    assert n == ref.size and np.array_equal(np_of(idx), ref)
+
+
+# ------------------------------------------------------------ diff/verify --
+
+@pytest.mark.parametrize("n", [1 << 20, 1_000_000])
+def test_config1_pair_end_to_end(n):
+    pair = synth.c1_pair(n=n, seed=1, device="cuda")
+    a, b = pair.a[0], pair.b[0]
+    C, eps = pair.chunk_bytes, pair.eps
+    ta, tb = ck.tree_build(a, C, eps), ck.tree_build(b, C, eps)
+    chunks = ck.tree_diff(ta, tb)
+    idx, cnt = ck.verify(a, b, chunks, C, eps)
+    an, bn = np_of(a), np_of(b)
+    ra, L = oracle_tree(an, C, eps)
+    rb, _ = oracle_tree(bn, C, eps)
+    ref_chunks = oracle.diff(ra, rb, L)
+    assert np.array_equal(np_of(chunks), ref_chunks)
+    truth = oracle.brute(an, bn, eps)
+    assert np.array_equal(np_of(idx), truth) and cnt == truth.size
+    # paper invariants: no false negatives; straddlers were flagged and removed
+    per = C // 4
+    assert set(np.unique(truth // per)) <= set(ref_chunks.tolist())
+    assert truth.size == pair.meta["n_above"] or truth.size >= pair.meta["n_above"] - 2
+
+
+@pytest.mark.parametrize("T", [1, 2, 3, 5, 17, 100, 1000, 4096, 10 ** 9])
+def test_diff_independent_of_start_level(T):
+    pair = synth.c1_pair(n=1 << 20, seed=3, device="cuda", n_above=300, n_below=300)
+    a, b = pair.a[0], pair.b[0]
+    ta, tb = ck.tree_build(a, 512, pair.eps), ck.tree_build(b, 512, pair.eps)
+    L = ta.n_leaves
+    out = torch.empty(L, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    ck.tree_diff_async(ta, tb, out, cnt, T=T)
+    n = int(cnt.item())
+    la = oracle.leaves(np_of(a), 512, pair.eps, threads=8)
+    lb = oracle.leaves(np_of(b), 512, pair.eps, threads=8)
+    plain = np.nonzero(np.any(la != lb, axis=1))[0]
+    assert np.array_equal(np_of(out[:n]), plain)
+
+
+def test_bfs_multi_array_mid_level_start():
+    sizes = [5000, 300_000, 1, 77_777]
+    arrs_a = [_data(n, torch.float64, 7 + i) for i, n in enumerate(sizes)]
+    arrs_b = [t.clone() for t in arrs_a]
+    g = torch.Generator(device="cpu").manual_seed(0)
+    for t in arrs_b:
+        k = torch.randint(0, t.numel(), (min(50, t.numel()),), generator=g).cuda()
+        t[k] += 1.0
+    TA, TB = ck.tree_build(arrs_a, 64, 1e-6), ck.tree_build(arrs_b, 64, 1e-6)
+    A = oracle.build_checkpoint([np_of(t) for t in arrs_a], 64, 1e-6)
+    B = oracle.build_checkpoint([np_of(t) for t in arrs_b], 64, 1e-6)
+    ref = oracle.diff_checkpoint(A, B)
+    for T in (1, 10, 1000, 20_000, 10 ** 12):
+        out = torch.empty(TA.n_leaves, dtype=torch.int64, device="cuda")
+        cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+        ck.tree_diff_async(TA, TB, out, cnt, T=T)
+        assert np.array_equal(np_of(out[: int(cnt.item())]), ref), T
+
+
+def test_identical_inputs_identical_roots_empty_diff():
+    a = _data(1 << 18, torch.float32, 42)
+    ta, tb = ck.tree_build(a, 4096, 1e-6), ck.tree_build(a.clone(), 4096, 1e-6)
+    assert ta.root() == tb.root()
+    assert ck.tree_diff(ta, tb).numel() == 0
+    idx, n = ck.verify(a, a.clone(), torch.arange(ta.n_leaves, device="cuda"), 4096, 1e-6)
+    assert n == 0
+
+
+def test_verify_every_chunk_equals_brute_force_f64():
+    pair = synth.c3_pair(n=1 << 20, seed=3, device="cuda", n_clusters=64, mean_len=256)
+    a, b = pair.a[0], pair.b[0]
+    for C, eps in ((512, 1e-3), (4096, 1e-6), (65536, 1e-8)):
+        L = -(-a.numel() * 8 // C)
+        idx, n = ck.verify(a, b, torch.arange(L, device="cuda"), C, eps)
+        truth = oracle.brute(np_of(a), np_of(b), eps)
+        assert n == truth.size and np.array_equal(np_of(idx), truth)
+
+
+def test_truncation_returns_prefix_and_full_count():
+    pair = synth.c1_pair(n=1 << 20, seed=9, device="cuda", n_above=500, n_below=0)
+    a, b = pair.a[0], pair.b[0]
+    ta, tb = ck.tree_build(a, 4096, pair.eps), ck.tree_build(b, 4096, pair.eps)
+    full = ck.tree_diff(ta, tb)
+    part = ck.tree_diff(ta, tb, cap=7)
+    assert np.array_equal(np_of(part), np_of(full)[:7])
+    idx_full, n_full = ck.verify(a, b, full, 4096, pair.eps)
+    idx_part, n_part = ck.verify(a, b, full, 4096, pair.eps, cap=11)
+    assert n_part == n_full and np.array_equal(np_of(idx_part), np_of(idx_full)[:11])
+
+
+def test_compare_and_compare_host_agree_with_oracle():
+    pair = synth.c2_pair(n_particles=1 << 16, seed=2, device="cuda", frac=0.02, n_clusters=8)
+    C, eps = pair.chunk_bytes, pair.eps
+    chunks, idx, nc, nd, ra, rb = ck.compare(pair.a, pair.b, C, eps)
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    A = oracle.build_checkpoint(an, C, eps)
+    B = oracle.build_checkpoint(bn, C, eps)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, C, ref_chunks, eps, A)
+    assert ra == A.root and rb == B.root
+    assert np.array_equal(np_of(chunks), ref_chunks) and nc == ref_chunks.size
+    assert np.array_equal(np_of(idx), ref_idx) and nd == ref_idx.size
+    assert np.array_equal(ref_idx, oracle.brute_checkpoint(an, bn, eps))
+    host_a = [t.cpu().pin_memory() for t in pair.a]
+    host_b = [t.cpu().pin_memory() for t in pair.b]
+    hidx, hnc, hnd, hra, hrb = ck.compare_host(host_a, host_b, C, eps)
+    assert (hnc, hnd, hra, hrb) == (nc, nd, ra, rb)
+    assert np.array_equal(hidx.numpy(), ref_idx)
+
+
+# ------------------------------------------------------------ error paths --
+
+def test_error_paths():
+    a = _data(1000, torch.float32, 1)
+    with pytest.raises(ck.CkptError) as e:
+        ck.tree_build(a, 24, 1e-3)
+    assert e.value.status == ck.EINVAL
+    with pytest.raises(ck.CkptError):
+        ck.tree_build(a, 16, -1.0)
+    with pytest.raises(ck.CkptError):
+        ck.tree_build(a, 16, float("nan"))
+    with pytest.raises(ck.CkptError):
+        ck.tree_build(a[1:], 16, 1e-3)      # misaligned (4-byte offset)
+    t1 = ck.tree_build(a, 64, 1e-3)
+    t2 = ck.tree_build(a[:999], 64, 1e-3)
+    t3 = ck.tree_build(a, 64, 1e-4)
+    with pytest.raises(ck.CkptError) as e:
+        ck.tree_diff(t1, t2)
+    assert e.value.status == ck.EMISMATCH
+    with pytest.raises(ck.CkptError) as e:
+        ck.tree_diff(t1, t3)
+    assert e.value.status == ck.EMISMATCH
+
+
+# ------------------------------------------------- full size (configs[1]) --
+
+@pytest.mark.slow
+def test_config2_full_size_sampled_parity():
+    """BASELINE configs[1] at full size (2^26 particles x 6 f32) in the bench's launch
+    configuration: sampled leaves by the oracle, all interior levels recomputed by the
+    oracle from the GPU leaves, verify == brute force over all 805M elements."""
+    pair = synth.c2_pair(device="cuda")
+    C, eps = pair.chunk_bytes, pair.eps
+    TA, TB = ck.tree_build(pair.a, C, eps), ck.tree_build(pair.b, C, eps)
+    rng = np.random.default_rng(0)
+    per = C // 4
+    for k in range(6):
+        na = gpu_tree_nodes(TA, k)
+        L = pair.a[k].numel() * 4 // C
+        sample = np.sort(rng.choice(L, 512, replace=False))
+        an = pair.a[k]
+        for c in sample:
+            chunk = np_of(an[c * per:(c + 1) * per])
+            assert np.array_equal(oracle.leaves(chunk, C, eps)[0], na[c]), (k, c)
+        assert np.array_equal(oracle.levels(na[:L]), na)
+    chunks = ck.tree_diff(TA, TB)
+    idx, n = ck.verify(pair.a, pair.b, chunks, C, eps)
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    truth = oracle.brute_checkpoint(an, bn, eps)
+    assert n == truth.size and np.array_equal(np_of(idx), truth)
