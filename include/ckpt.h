@@ -108,6 +108,17 @@ ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n, u
                                    ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
                                    void *stream, ckpt_tree **out);
 
+/* Several checkpoints' trees with ONE leaf-kernel launch (e.g. run A and run B
+ * of a pair, so the leaf kernel's last wave of chunk chains is fuller).
+ * data (host) / n (host) list the arrays of all trees back to back;
+ * arrays_per_tree (host, n_trees entries) splits them; out (host, n_trees
+ * entries) receives the trees.  Same rules and errors as
+ * ckpt_tree_build_arrays; on error no tree is returned. */
+ckpt_status ckpt_tree_build_batch(const void *const *data, const uint64_t *n,
+                                  const uint32_t *arrays_per_tree, uint32_t n_trees,
+                                  ckpt_dtype dtype, uint32_t chunk_bytes, double eps, void *stream,
+                                  ckpt_tree **out);
+
 /* Tree over caller-supplied 16-byte digests used as leaves (no data
  * hashing).  Used to form the top levels over the subtree roots gathered
  * from all GPUs (R15; the multi-GPU path).  digests16: device, count*16

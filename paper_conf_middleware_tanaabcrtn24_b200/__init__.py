@@ -52,7 +52,7 @@ def lib():
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.LIB
+    path = os.environ.get("CKPT_LIB", _build.LIB)   # CKPT_LIB: a tuning variant of libckpt.so
     if not os.path.exists(path):
         raise ImportError(
             f"libckpt.so not built at {path}; run `python -c 'import __graft_entry__ as g; g.build()'`")
@@ -63,6 +63,7 @@ def lib():
     pu64 = ctypes.POINTER(ctypes.c_uint64)
     L.ckpt_tree_build.argtypes = [vp, u64, i32, u32, dbl, vp, pp]
     L.ckpt_tree_build_arrays.argtypes = [pp, pu64, u32, i32, u32, dbl, vp, pp]
+    L.ckpt_tree_build_batch.argtypes = [pp, pu64, ctypes.POINTER(u32), u32, i32, u32, dbl, vp, pp]
     L.ckpt_tree_from_digests.argtypes = [vp, u64, vp, pp]
     L.ckpt_tree_free.argtypes = [vp]
     L.ckpt_tree_free.restype = None
@@ -92,7 +93,8 @@ def lib():
     L.ckpt_strerror.restype = ctypes.c_char_p
     L.ckpt_last_error.restype = ctypes.c_char_p
     L.ckpt_version.restype = u32
-    for name in ("ckpt_tree_build", "ckpt_tree_build_arrays", "ckpt_tree_from_digests",
+    for name in ("ckpt_tree_build", "ckpt_tree_build_arrays", "ckpt_tree_build_batch",
+                 "ckpt_tree_from_digests",
                  "ckpt_tree_diff", "ckpt_tree_diff_async", "ckpt_verify",
                  "ckpt_verify_arrays_async", "ckpt_compare", "ckpt_compare_host",
                  "ckpt_tree_info", "ckpt_tree_root", "ckpt_tree_array_roots", "ckpt_tree_nodes",
@@ -230,6 +232,23 @@ def tree_build(arrays: Union[torch.Tensor, Sequence[torch.Tensor]], chunk_bytes:
     _check(lib().ckpt_tree_build_arrays(pp, pn, len(ts), code, chunk_bytes, float(eps), sp,
                                         ctypes.byref(out)), "ckpt_tree_build_arrays")
     return Tree(out.value, ts, code, chunk_bytes, float(eps), sp)
+
+
+def tree_build_batch(checkpoints: Sequence[Sequence[torch.Tensor]], chunk_bytes: int, eps: float,
+                     stream=None) -> List[Tree]:
+    """Several checkpoints' trees with one leaf-kernel launch (ckpt_tree_build_batch)."""
+    cks = [_as_list(c) for c in checkpoints]
+    flat = [t for c in cks for t in c]
+    code = _check_arrays(flat)
+    pp, _k1 = _ptr_array(flat)
+    pn, _k2 = _u64_array([t.numel() for t in flat])
+    per = (ctypes.c_uint32 * len(cks))(*[len(c) for c in cks])
+    outs = (ctypes.c_void_p * len(cks))()
+    sp = _stream_ptr(stream)
+    _check(lib().ckpt_tree_build_batch(pp, pn, per, len(cks), code, chunk_bytes, float(eps), sp,
+                                       ctypes.cast(outs, ctypes.POINTER(ctypes.c_void_p))),
+           "ckpt_tree_build_batch")
+    return [Tree(outs[k], cks[k], code, chunk_bytes, float(eps), sp) for k in range(len(cks))]
 
 
 def tree_from_digests(digests: torch.Tensor, stream=None) -> Tree:

@@ -200,6 +200,9 @@ struct ckpt_tree {
     const uint64_t *d_off = nullptr, *d_cnt = nullptr, *d_level_base = nullptr,
                    *d_level_total = nullptr, *d_chunk_base = nullptr;
     const uint32_t *d_height = nullptr;
+    const uint64_t *d_gbegin = nullptr;
+    unsigned *d_ticket = nullptr;
+    uint64_t n_groups = 0;
 };
 
 static uint32_t tree_height(uint64_t L) {
@@ -253,19 +256,12 @@ static void layout(ckpt_tree *t, const std::vector<uint64_t> &leaves) {
 
 static size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
-// Allocate nodes + metadata, stage metadata.  `extra` = leaf table bytes.
-static ckpt_status alloc_tree(ckpt_tree *t, cudaStream_t s, std::vector<uint8_t> &blob,
-                              std::vector<size_t> &offs) {
-    CK_CUDA(cudaMallocAsync((void **)&t->nodes, (t->array_nodes + t->top_nodes) * 16, s));
-    CK_CUDA(cudaMallocAsync((void **)&t->meta, blob.size(), s));
-    CK_TRY(g_ring.copy(t->meta, blob.data(), blob.size(), s));
-    (void)offs;
-    return CKPT_OK;
-}
-
 static bool quant_params(double eps, QuantParams *q) {
     if (!(eps >= 0.0) || std::isinf(eps)) return false;
-    if (eps == 0.0) { std::memset(q, 0, sizeof(*q)); return true; }
+    std::memset(q, 0, sizeof(*q));
+    q->m1 = 0x52dce729ull;
+    q->m2 = 0x38495ab5ull;
+    if (eps == 0.0) return true;
     const double inv = 1.0 / eps;
     if (!std::isfinite(inv)) return false;
     q->inv = inv;
@@ -296,7 +292,7 @@ static ckpt_status check_common(ckpt_dtype dtype, uint32_t chunk_bytes, double e
 
 template <int DT, bool RAW, int CB>
 static ckpt_status launch_leaf_t(const LeafArray *arr, int na, uint64_t tasks, uint32_t C,
-                                 const QuantParams &q, uint4 *nodes, cudaStream_t s, int sms) {
+                                 const QuantParams &q, cudaStream_t s, int sms) {
     auto k = leaf_kernel<DT, RAW, CB>;
     static std::atomic<int> cached_per_sm{0};
     int per_sm = cached_per_sm.load(std::memory_order_relaxed);
@@ -311,71 +307,89 @@ static ckpt_status launch_leaf_t(const LeafArray *arr, int na, uint64_t tasks, u
     uint64_t want = (tasks + kLeafWarps - 1) / kLeafWarps;
     uint64_t grid = std::min<uint64_t>(want, (uint64_t)sms * per_sm);
     ProfScope prof(0, s);
-    k<<<(unsigned)grid, kLeafWarps * 32, kLeafSmem, s>>>(arr, na, tasks, C, q, nodes);
+    k<<<(unsigned)grid, kLeafWarps * 32, kLeafSmem, s>>>(arr, na, tasks, C, q);
     CK_LAUNCH();
     return CKPT_OK;
 }
 
 template <int DT, bool RAW>
 static ckpt_status launch_leaf_dt(const LeafArray *arr, int na, uint64_t tasks, uint32_t C,
-                                  const QuantParams &q, uint4 *nodes, cudaStream_t s, int sms) {
+                                  const QuantParams &q, cudaStream_t s, int sms) {
     if (!RAW) {
         switch (C) {
-            case 512: return launch_leaf_t<DT, RAW, 512>(arr, na, tasks, C, q, nodes, s, sms);
-            case 1024: return launch_leaf_t<DT, RAW, 1024>(arr, na, tasks, C, q, nodes, s, sms);
-            case 2048: return launch_leaf_t<DT, RAW, 2048>(arr, na, tasks, C, q, nodes, s, sms);
-            case 4096: return launch_leaf_t<DT, RAW, 4096>(arr, na, tasks, C, q, nodes, s, sms);
-            case 8192: return launch_leaf_t<DT, RAW, 8192>(arr, na, tasks, C, q, nodes, s, sms);
-            case 16384: return launch_leaf_t<DT, RAW, 16384>(arr, na, tasks, C, q, nodes, s, sms);
-            case 32768: return launch_leaf_t<DT, RAW, 32768>(arr, na, tasks, C, q, nodes, s, sms);
-            case 65536: return launch_leaf_t<DT, RAW, 65536>(arr, na, tasks, C, q, nodes, s, sms);
+            case 512: return launch_leaf_t<DT, RAW, 512>(arr, na, tasks, C, q, s, sms);
+            case 1024: return launch_leaf_t<DT, RAW, 1024>(arr, na, tasks, C, q, s, sms);
+            case 2048: return launch_leaf_t<DT, RAW, 2048>(arr, na, tasks, C, q, s, sms);
+            case 4096: return launch_leaf_t<DT, RAW, 4096>(arr, na, tasks, C, q, s, sms);
+            case 8192: return launch_leaf_t<DT, RAW, 8192>(arr, na, tasks, C, q, s, sms);
+            case 16384: return launch_leaf_t<DT, RAW, 16384>(arr, na, tasks, C, q, s, sms);
+            case 32768: return launch_leaf_t<DT, RAW, 32768>(arr, na, tasks, C, q, s, sms);
+            case 65536: return launch_leaf_t<DT, RAW, 65536>(arr, na, tasks, C, q, s, sms);
             default: break;
         }
     }
-    return launch_leaf_t<DT, RAW, 0>(arr, na, tasks, C, q, nodes, s, sms);
+    return launch_leaf_t<DT, RAW, 0>(arr, na, tasks, C, q, s, sms);
 }
 
-static ckpt_status launch_levels(ckpt_tree *t, const uint64_t *d_gbegin, uint64_t n_groups,
-                                 unsigned *ticket, cudaStream_t s) {
-    LevelParams p;
-    p.nodes = t->nodes;
-    p.off = t->d_off;
-    p.cnt = t->d_cnt;
-    p.gbegin = d_gbegin;
-    p.level_base = t->d_level_base;
-    p.level_total = t->d_level_total;
-    p.height = t->d_height;
-    p.top_off = t->top_off;
-    p.ticket = ticket;
-    p.n_arrays = (int)t->n_arrays;
-    p.n_levels = (int)t->n_levels;
-    p.ls = 0;
-    ProfScope prof(1, s);
-    levels_kernel<<<(unsigned)n_groups, kLevelThreads, 0, s>>>(p);
-    CK_LAUNCH();
+// K2 for up to kMaxLevelTrees trees in one launch.
+static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s) {
+    static std::atomic<int> attr_done{0};
+    if (!attr_done.load()) {
+        CK_CUDA(cudaFuncSetAttribute(levels_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kLevelSmem));
+        attr_done.store(1);
+    }
+    for (int k0 = 0; k0 < n; k0 += kMaxLevelTrees) {
+        LevelBatch b;
+        std::memset(&b, 0, sizeof(b));
+        b.n = std::min(kMaxLevelTrees, n - k0);
+        unsigned ctas = 0;
+        for (int i = 0; i < b.n; ++i) {
+            const ckpt_tree *t = trees[k0 + i];
+            LevelParams &p = b.t[i];
+            p.nodes = t->nodes;
+            p.off = t->d_off;
+            p.cnt = t->d_cnt;
+            p.gbegin = t->d_gbegin;
+            p.level_base = t->d_level_base;
+            p.level_total = t->d_level_total;
+            p.height = t->d_height;
+            p.top_off = t->top_off;
+            p.ticket = t->d_ticket;
+            p.n_arrays = (int)t->n_arrays;
+            p.n_levels = (int)t->n_levels;
+            p.ls = 0;
+            p.n_groups = (unsigned)t->n_groups;
+            b.cta_begin[i] = ctas;
+            ctas += (unsigned)t->n_groups;
+        }
+        b.cta_begin[b.n] = ctas;
+        ProfScope prof(1, s);
+        levels_kernel<<<ctas, kLevelThreads, kLevelSmem, s>>>(b);
+        CK_LAUNCH();
+    }
     return CKPT_OK;
 }
 
-// Build the blob: [off][cnt][level_base][level_total][chunk_base][height][gbegin][ticket][leaf table]
-static ckpt_status build_common(ckpt_tree *t, cudaStream_t s, const LeafArray *leaf_host,
-                                const QuantParams *q, int sms, const void *digests) {
-    const uint32_t na = t->n_arrays, nl = t->n_levels;
+// Allocate a laid-out tree's node storage and device metadata blob:
+// [off][cnt][level_base][level_total][chunk_base][height][gbegin][ticket]
+static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
+    const uint32_t na = t->n_arrays;
     std::vector<uint64_t> gbegin(na);
     uint64_t groups = 0;
     for (uint32_t a = 0; a < na; ++a) {
         gbegin[a] = groups;
         groups += (t->cnt[a] + kGroup - 1) / kGroup;   // level 0 counts
     }
-    size_t o_off = 0;
-    size_t o_cnt = align256(o_off + t->off.size() * 8);
-    size_t o_lb = align256(o_cnt + t->cnt.size() * 8);
-    size_t o_lt = align256(o_lb + t->level_base.size() * 8);
-    size_t o_cb = align256(o_lt + t->level_total.size() * 8);
-    size_t o_h = align256(o_cb + (size_t)na * 8);
-    size_t o_g = align256(o_h + (size_t)na * 4);
-    size_t o_tk = align256(o_g + (size_t)na * 8);
-    size_t o_leaf = align256(o_tk + 16);
-    size_t total = align256(o_leaf + (leaf_host ? (size_t)na * sizeof(LeafArray) : 0));
+    t->n_groups = groups;
+    const size_t o_off = 0;
+    const size_t o_cnt = align256(o_off + t->off.size() * 8);
+    const size_t o_lb = align256(o_cnt + t->cnt.size() * 8);
+    const size_t o_lt = align256(o_lb + t->level_base.size() * 8);
+    const size_t o_cb = align256(o_lt + t->level_total.size() * 8);
+    const size_t o_h = align256(o_cb + (size_t)na * 8);
+    const size_t o_g = align256(o_h + (size_t)na * 4);
+    const size_t o_tk = align256(o_g + (size_t)na * 8);
+    const size_t total = align256(o_tk + 16);
     std::vector<uint8_t> blob(total, 0);
     std::memcpy(blob.data() + o_off, t->off.data(), t->off.size() * 8);
     std::memcpy(blob.data() + o_cnt, t->cnt.data(), t->cnt.size() * 8);
@@ -384,48 +398,57 @@ static ckpt_status build_common(ckpt_tree *t, cudaStream_t s, const LeafArray *l
     std::memcpy(blob.data() + o_cb, t->chunk_base.data(), (size_t)na * 8);
     std::memcpy(blob.data() + o_h, t->height.data(), (size_t)na * 4);
     std::memcpy(blob.data() + o_g, gbegin.data(), (size_t)na * 8);
-    if (leaf_host) std::memcpy(blob.data() + o_leaf, leaf_host, (size_t)na * sizeof(LeafArray));
-    std::vector<size_t> offs;
-    CK_TRY(alloc_tree(t, s, blob, offs));
+    CK_CUDA(cudaMallocAsync((void **)&t->nodes, (t->array_nodes + t->top_nodes) * 16, s));
+    CK_CUDA(cudaMallocAsync((void **)&t->meta, blob.size(), s));
+    CK_TRY(g_ring.copy(t->meta, blob.data(), blob.size(), s));
     t->d_off = (const uint64_t *)(t->meta + o_off);
     t->d_cnt = (const uint64_t *)(t->meta + o_cnt);
     t->d_level_base = (const uint64_t *)(t->meta + o_lb);
     t->d_level_total = (const uint64_t *)(t->meta + o_lt);
     t->d_chunk_base = (const uint64_t *)(t->meta + o_cb);
     t->d_height = (const uint32_t *)(t->meta + o_h);
-    const uint64_t *d_gbegin = (const uint64_t *)(t->meta + o_g);
-    unsigned *ticket = (unsigned *)(t->meta + o_tk);
-    (void)nl;
-    if (leaf_host) {
-        // leaf table with the device node pointer offsets
-        const LeafArray *d_leaf = (const LeafArray *)(t->meta + o_leaf);
-        uint64_t tasks = 0;
-        for (uint32_t a = 0; a < na; ++a) tasks += (t->n_leaves[a] + 31) / 32;
-        const uint32_t C = t->chunk_bytes;
-        if (t->eps == 0.0) {
-            if (t->dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
-            else CK_TRY((launch_leaf_dt<1, true>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
-        } else {
-            if (t->dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
-            else CK_TRY((launch_leaf_dt<1, false>(d_leaf, (int)na, tasks, C, *q, t->nodes, s, sms)));
-        }
-    } else if (digests) {
-        CK_CUDA(cudaMemcpyAsync(t->nodes, digests, t->total_leaves * 16, cudaMemcpyDeviceToDevice, s));
-    }
-    return launch_levels(t, d_gbegin, groups, ticket, s);
+    t->d_gbegin = (const uint64_t *)(t->meta + o_g);
+    t->d_ticket = (unsigned *)(t->meta + o_tk);
+    return CKPT_OK;
 }
 
-extern "C" ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n,
-                                              uint32_t n_arrays, ckpt_dtype dtype,
-                                              uint32_t chunk_bytes, double eps, void *stream,
-                                              ckpt_tree **out) {
-    if (!out) return fail(CKPT_EINVAL, "out is NULL");
-    *out = nullptr;
-    if (!data || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
-    if (n_arrays >= (1u << 20)) return fail(CKPT_EINVAL, "at most 2^20-1 arrays");
+// One leaf-kernel launch over every array of every tree in `table`.
+static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t tasks,
+                                 ckpt_dtype dtype, double eps, uint32_t C, cudaStream_t s, int sms) {
+    QuantParams q;
+    quant_params(eps, &q);
+    LeafArray *d_tab = nullptr;
+    const size_t bytes = table.size() * sizeof(LeafArray);
+    CK_CUDA(cudaMallocAsync((void **)&d_tab, bytes, s));
+    CK_TRY(g_ring.copy(d_tab, table.data(), bytes, s));
+    const int na = (int)table.size();
+    if (eps == 0.0) {
+        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(d_tab, na, tasks, C, q, s, sms)));
+        else CK_TRY((launch_leaf_dt<1, true>(d_tab, na, tasks, C, q, s, sms)));
+    } else {
+        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(d_tab, na, tasks, C, q, s, sms)));
+        else CK_TRY((launch_leaf_dt<1, false>(d_tab, na, tasks, C, q, s, sms)));
+    }
+    CK_CUDA(cudaFreeAsync(d_tab, s));
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint64_t *n,
+                                             const uint32_t *arrays_per_tree, uint32_t n_trees,
+                                             ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                             void *stream, ckpt_tree **out) {
+    if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
+    for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
+    if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
-    for (uint32_t a = 0; a < n_arrays; ++a) {
+    uint64_t total_arrays = 0;
+    for (uint32_t k = 0; k < n_trees; ++k) {
+        if (arrays_per_tree[k] == 0 || arrays_per_tree[k] >= (1u << 20))
+            return fail(CKPT_EINVAL, "every tree needs 1 .. 2^20-1 arrays");
+        total_arrays += arrays_per_tree[k];
+    }
+    for (uint64_t a = 0; a < total_arrays; ++a) {
         if (!data[a]) return fail(CKPT_EINVAL, "NULL data pointer");
         if (n[a] == 0) return fail(CKPT_EINVAL, "empty array (n == 0)");
         if ((uintptr_t)data[a] % 16 != 0) return fail(CKPT_EINVAL, "data must be 16-byte aligned");
@@ -435,36 +458,54 @@ extern "C" ckpt_status ckpt_tree_build_arrays(const void *const *data, const uin
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
     cudaStream_t s = (cudaStream_t)stream;
-    ckpt_tree *t = new ckpt_tree();
-    t->device = dev;
-    t->stream = s;
-    t->dtype = dtype;
-    t->chunk_bytes = chunk_bytes;
-    t->eps = eps;
-    t->n_elems.assign(n, n + n_arrays);
-    std::vector<uint64_t> leaves(n_arrays);
-    for (uint32_t a = 0; a < n_arrays; ++a) leaves[a] = (n[a] * esz + chunk_bytes - 1) / chunk_bytes;
-    layout(t, leaves);
-    std::vector<LeafArray> lt(n_arrays);
-    uint64_t task = 0;
-    for (uint32_t a = 0; a < n_arrays; ++a) {
-        lt[a].data = (const uint8_t *)data[a];
-        lt[a].nbytes = n[a] * esz;
-        lt[a].n_leaves = leaves[a];
-        lt[a].n_full = lt[a].nbytes / chunk_bytes;
-        lt[a].task_begin = task;
-        lt[a].leaf_off = t->off[a];      // level 0 offset of array a
-        task += (leaves[a] + 31) / 32;
+    std::vector<LeafArray> table;
+    table.reserve(total_arrays);
+    uint64_t task = 0, a0 = 0;
+    ckpt_status st = CKPT_OK;
+    for (uint32_t k = 0; k < n_trees && st == CKPT_OK; ++k) {
+        const uint32_t na = arrays_per_tree[k];
+        ckpt_tree *t = new ckpt_tree();
+        out[k] = t;
+        t->device = dev;
+        t->stream = s;
+        t->dtype = dtype;
+        t->chunk_bytes = chunk_bytes;
+        t->eps = eps;
+        t->n_elems.assign(n + a0, n + a0 + na);
+        std::vector<uint64_t> leaves(na);
+        for (uint32_t a = 0; a < na; ++a) leaves[a] = (n[a0 + a] * esz + chunk_bytes - 1) / chunk_bytes;
+        layout(t, leaves);
+        st = prepare_tree(t, s);
+        for (uint32_t a = 0; a < na && st == CKPT_OK; ++a) {
+            LeafArray e;
+            e.data = (const uint8_t *)data[a0 + a];
+            e.nbytes = n[a0 + a] * esz;
+            e.n_leaves = leaves[a];
+            e.n_full = e.nbytes / chunk_bytes;
+            e.task_begin = task;
+            e.out = t->nodes + t->off[a];      // level 0 of array a
+            table.push_back(e);
+            task += (leaves[a] + kRows - 1) / kRows;
+        }
+        a0 += na;
     }
-    QuantParams q;
-    quant_params(eps, &q);
-    ckpt_status st = build_common(t, s, lt.data(), &q, di.sms, nullptr);
+    if (st == CKPT_OK) st = launch_leaves(table, task, dtype, eps, chunk_bytes, s, di.sms);
+    if (st == CKPT_OK) st = launch_levels(out, (int)n_trees, s);
     if (st != CKPT_OK) {
-        ckpt_tree_free_on(t, stream);
+        for (uint32_t k = 0; k < n_trees; ++k) { ckpt_tree_free_on(out[k], stream); out[k] = nullptr; }
         return st;
     }
-    *out = t;
     return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n,
+                                              uint32_t n_arrays, ckpt_dtype dtype,
+                                              uint32_t chunk_bytes, double eps, void *stream,
+                                              ckpt_tree **out) {
+    if (!out) return fail(CKPT_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
+    return ckpt_tree_build_batch(data, n, &n_arrays, 1, dtype, chunk_bytes, eps, stream, out);
 }
 
 extern "C" ckpt_status ckpt_tree_build(const void *data, uint64_t n, ckpt_dtype dtype,
@@ -491,7 +532,10 @@ extern "C" ckpt_status ckpt_tree_from_digests(const void *digests16, uint64_t co
     t->chunk_bytes = 16;
     t->n_elems.assign(1, count);
     layout(t, std::vector<uint64_t>{count});
-    ckpt_status st = build_common(t, s, nullptr, nullptr, di.sms, digests16);
+    ckpt_status st = prepare_tree(t, s);
+    if (st == CKPT_OK && cudaMemcpyAsync(t->nodes, digests16, count * 16, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        st = fail(CKPT_ECUDA, "digest copy");
+    if (st == CKPT_OK) st = launch_levels(&t, 1, s);
     if (st != CKPT_OK) { ckpt_tree_free_on(t, stream); return st; }
     *out = t;
     return CKPT_OK;
@@ -776,8 +820,16 @@ extern "C" ckpt_status ckpt_compare(const void *const *a, const void *const *b, 
     cudaStream_t s = (cudaStream_t)stream;
     ckpt_tree *ta = nullptr, *tb = nullptr;
     uint64_t *dc = nullptr;
-    ckpt_status st = ckpt_tree_build_arrays(a, n, n_arrays, dtype, chunk_bytes, eps, stream, &ta);
-    if (st == CKPT_OK) st = ckpt_tree_build_arrays(b, n, n_arrays, dtype, chunk_bytes, eps, stream, &tb);
+    // both runs' leaves in one leaf-kernel launch (fuller last wave)
+    std::vector<const void *> ab(a, a + n_arrays);
+    ab.insert(ab.end(), b, b + n_arrays);
+    std::vector<uint64_t> nn(n, n + n_arrays);
+    nn.insert(nn.end(), n, n + n_arrays);
+    const uint32_t per[2] = {n_arrays, n_arrays};
+    ckpt_tree *tt[2] = {nullptr, nullptr};
+    ckpt_status st = ckpt_tree_build_batch(ab.data(), nn.data(), per, 2, dtype, chunk_bytes, eps, stream, tt);
+    ta = tt[0];
+    tb = tt[1];
     if (st == CKPT_OK && cudaMallocAsync((void **)&dc, 16, s) != cudaSuccess)
         st = fail(CKPT_ENOMEM, "count scratch");
     if (st == CKPT_OK) st = ckpt_tree_diff_async(ta, tb, 0, chunks, chunks_cap, dc, stream);

@@ -67,13 +67,61 @@ __device__ uint64_t tile_lookback(uint64_t *states, uint64_t tile, uint64_t aggr
     return excl;
 }
 
+// CTA-wide decoupled look-back: every thread inspects one predecessor per
+// round, so a round covers blockDim.x predecessors with one L2 round trip
+// (a warp-wide look-back walks 32 at a time, which is a serial chain when all
+// tiles start together).  Called by all threads; `aggregate` must be the
+// same in every thread.  Returns the tile's exclusive prefix.
+template <int NT>
+__device__ uint64_t cta_lookback(uint64_t *states, uint64_t tile, uint64_t aggregate) {
+    constexpr int NW = NT / 32;
+    __shared__ uint64_t s_sum[NW];
+    __shared__ int s_min[NW];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tile == 0) {
+        if (tid == 0) st_volatile(&states[0], kFlagP | aggregate);
+        return 0;
+    }
+    if (tid == 0) st_volatile(&states[tile], kFlagA | aggregate);
+    uint64_t excl = 0;
+    int64_t hi = (int64_t)tile - 1;
+    for (;;) {
+        const int64_t idx = hi - tid;
+        uint64_t s = kFlagP;                       // before tile 0: inclusive prefix 0
+        if (idx >= 0) {
+            do { s = ld_volatile(&states[idx]); } while (s == 0);
+        }
+        int mp = (s & kFlagP) ? tid : 0x7fffffff;  // nearest predecessor with a prefix
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) mp = min(mp, __shfl_xor_sync(kFull, mp, o));
+        if (lane == 0) s_min[warp] = mp;
+        __syncthreads();
+        int nearest = s_min[0];
+#pragma unroll
+        for (int w = 1; w < NW; ++w) nearest = min(nearest, s_min[w]);
+        const uint64_t wsum = warp_sum_u64(tid <= nearest ? (s & kValMask) : 0);
+        if (lane == 0) s_sum[warp] = wsum;
+        __syncthreads();
+        uint64_t tot = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) tot += s_sum[w];
+        excl += tot;
+        __syncthreads();
+        if (nearest != 0x7fffffff) break;
+        hi -= NT;
+    }
+    if (tid == 0) st_volatile(&states[tile], kFlagP | (excl + aggregate));
+    return excl;
+}
+
 // ---------------------------------------------------------------------------
 // ordered compaction over [0, n): pred = leaf digests differ (MODE 0) or a
 // flag byte is set (MODE 1).  Output value = item index (a global chunk id).
 // ---------------------------------------------------------------------------
 constexpr int kCompactThreads = 256;
-constexpr int kCompactRows = 16;                          // rows of 32 items per warp
-constexpr int kCompactTile = kCompactThreads * kCompactRows;  // 4096 items
+constexpr int kCompactRows = 4;                           // rows of 32 items per warp
+constexpr int kCompactTile = kCompactThreads * kCompactRows;  // 1024 items
+constexpr int kRowsPerLane = kCompactRows * 8 / 32;       // scan: row counts per lane
 
 struct CompactParams {
     const uint4 *leaf_a;
@@ -102,35 +150,46 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(CompactParams 
         if (tile >= n_tiles) return;
         const uint64_t t0 = tile * kCompactTile;
         uint32_t bits[kCompactRows];
+        bool hit[kCompactRows];
+        // all loads first (one round trip per tile), then the ballots
+        if (MODE == 0) {
+            uint4 va[kCompactRows], vb[kCompactRows];
+#pragma unroll
+            for (int k = 0; k < kCompactRows; ++k) {
+                const uint64_t i = t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
+                va[k] = vb[k] = make_uint4(0u, 0u, 0u, 0u);
+                if (i < p.n) { va[k] = __ldcs(p.leaf_a + i); vb[k] = __ldcs(p.leaf_b + i); }
+            }
+#pragma unroll
+            for (int k = 0; k < kCompactRows; ++k) hit[k] = digest_ne(va[k], vb[k]);
+        } else {
+#pragma unroll
+            for (int k = 0; k < kCompactRows; ++k) {
+                const uint64_t i = t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
+                hit[k] = i < p.n && p.flags[i] != 0;
+            }
+        }
 #pragma unroll
         for (int k = 0; k < kCompactRows; ++k) {
-            const uint64_t i = t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
-            bool hit = false;
-            if (i < p.n) {
-                if (MODE == 0) hit = digest_ne(p.leaf_a[i], p.leaf_b[i]);
-                else hit = p.flags[i] != 0;
-            }
-            bits[k] = __ballot_sync(kFull, hit);
+            bits[k] = __ballot_sync(kFull, hit[k]);
             if (lane == 0) row_cnt[k * 8 + warp] = __popc(bits[k]);
         }
         __syncthreads();
         if (warp == 0) {
             // rows in item order: k major, warp minor -> flat index k*8+warp
-            uint32_t v[4], s = 0;
+            uint32_t v[kRowsPerLane], s = 0;
 #pragma unroll
-            for (int r = 0; r < 4; ++r) { v[r] = row_cnt[lane * 4 + r]; s += v[r]; }
+            for (int r = 0; r < kRowsPerLane; ++r) { v[r] = row_cnt[lane * kRowsPerLane + r]; s += v[r]; }
             uint32_t total;
             uint32_t ex = warp_excl_scan_u32(s, lane, total);
 #pragma unroll
-            for (int r = 0; r < 4; ++r) { row_off[lane * 4 + r] = ex; ex += v[r]; }
-            const uint64_t excl = tile_lookback(p.states, tile, total, lane);
-            if (lane == 0) {
-                s_excl = excl;
-                if (tile == n_tiles - 1) *p.count = excl + total;
-            }
+            for (int r = 0; r < kRowsPerLane; ++r) { row_off[lane * kRowsPerLane + r] = ex; ex += v[r]; }
+            if (lane == 0) s_excl = total;
         }
         __syncthreads();
-        const uint64_t excl = s_excl;
+        const uint64_t total = s_excl;
+        const uint64_t excl = cta_lookback<kCompactThreads>(p.states, tile, total);
+        if (threadIdx.x == 0 && tile == n_tiles - 1) *p.count = excl + total;
         const uint32_t lt = (1u << lane) - 1u;
 #pragma unroll
         for (int k = 0; k < kCompactRows; ++k) {
@@ -354,17 +413,17 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams 
             const uint32_t v = lane < kVerifyWarps ? w_cnt[lane] : 0u;
             uint32_t total;
             const uint32_t ex = warp_excl_scan_u32(v, lane, total);
+            __syncwarp();
             if (lane < kVerifyWarps) w_cnt[lane] = ex;
-            const uint64_t excl = tile_lookback(p.states, tile, total, lane);
-            if (lane == 0) {
-                s_excl = excl;
-                if (tile == n_tiles - 1) *p.count = excl + total;
-            }
+            if (lane == 0) s_excl = total;
         }
         __syncthreads();
+        const uint64_t tile_total = s_excl;
+        const uint64_t excl = cta_lookback<kVerifyWarps * 32>(p.states, tile, tile_total);
+        if (threadIdx.x == 0 && tile == n_tiles - 1) *p.count = excl + tile_total;
         // pass 2: emit (only chunks with hits re-read their data)
         if (cnt) {
-            uint64_t pos = s_excl + w_cnt[warp];
+            uint64_t pos = excl + w_cnt[warp];
             for (uint64_t e0 = 0; e0 < len; e0 += kStep) {
                 const uint64_t e = e0 + (uint64_t)lane * VEC;
                 const uint32_t m = e < len ? diff_bits<DT>(pa, pb, e, len, p.eps) : 0u;

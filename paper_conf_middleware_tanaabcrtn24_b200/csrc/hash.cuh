@@ -118,6 +118,7 @@ struct QuantParams {
     uint64_t inv_m;    // inv = inv_m * 2^inv_e exactly
     int32_t inv_e;
     float r32;         // fast path iff |x| < r32 (f32 input)
+    uint64_t m1, m2;   // Murmur3F body constants 0x52dce729 / 0x38495ab5 (see mm32.cuh)
 };
 
 constexpr double kMagic = 6755399441055744.0;            // 1.5 * 2^52

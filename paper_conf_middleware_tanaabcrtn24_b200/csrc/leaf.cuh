@@ -17,6 +17,7 @@
 #include <cstdint>
 
 #include "hash.cuh"
+#include "mm32.cuh"
 
 namespace ckpt {
 
@@ -26,16 +27,30 @@ struct LeafArray {            // one array of the checkpoint (device table)
     uint64_t n_leaves;        // ceil(nbytes / C)
     uint64_t n_full;          // nbytes / C  (chunks of exactly C bytes)
     uint64_t task_begin;      // first global task id of this array
-    uint64_t leaf_off;        // node index of this array's leaf 0
+    uint4 *out;               // this array's leaf 0 in its tree's node storage
 };
 
-constexpr int kLeafWarps = 8;        // warps per CTA
-constexpr int kSeg = 64;             // bytes per chunk per stage
-constexpr int kStages = 4;           // ring depth
+#ifndef CKPT_LEAF_SEG
+#define CKPT_LEAF_SEG 128
+#endif
+#ifndef CKPT_LEAF_STAGES
+#define CKPT_LEAF_STAGES 2
+#endif
+#ifndef CKPT_LEAF_MINB
+#define CKPT_LEAF_MINB 3
+#endif
+#ifndef CKPT_LEAF_CH
+#define CKPT_LEAF_CH 1
+#endif
+constexpr int kLeafWarps = 8;                  // warps per CTA
+constexpr int kCh = CKPT_LEAF_CH;              // chains (chunks) per lane
+constexpr int kRows = 32 * kCh;                // chunks per warp task
+constexpr int kSeg = CKPT_LEAF_SEG;            // bytes per chunk per stage
+constexpr int kStages = CKPT_LEAF_STAGES;      // ring depth
 constexpr int kPitch = kSeg + 16;    // padded row
-constexpr int kSlotBytes = 32 * kPitch;
+constexpr int kSlotBytes = kRows * kPitch;
 constexpr int kWarpSmem = kStages * kSlotBytes;
-constexpr int kLeafSmem = kLeafWarps * kWarpSmem;
+constexpr int kLeafSmem = kLeafWarps * kWarpSmem + 16;   // + the two h*5+c addends
 
 __device__ __forceinline__ void cp_async16(uint32_t smem, const void *gptr, uint32_t src_bytes) {
     asm volatile("cp.async.cg.shared.global.L2::128B [%0], [%1], 16, %2;\n" ::"r"(smem), "l"(gptr),
@@ -59,45 +74,56 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
     return v;
 }
 
-// Hash one 16-byte block of input (as 4 u32 lanes of raw bits) into (h1,h2).
+// Hash one 16-byte block (raw bits in v), exact words for every input:
+// per-element fast/slow selection (generic path: ragged tasks and retries).
 template <int DT, bool RAW>
-__device__ __forceinline__ void chain_block(uint64_t &h1, uint64_t &h2, uint4 v, const QuantParams &q) {
-    uint64_t k1, k2;
+__device__ __forceinline__ void chain_block_exact(U64p &h1, U64p &h2, uint4 v, const QuantParams &q) {
+    uint4 w;
     if (RAW) {
-        k1 = (uint64_t)v.x | ((uint64_t)v.y << 32);
-        k2 = (uint64_t)v.z | ((uint64_t)v.w << 32);
+        w = v;
+    } else if (DT == 0) {
+        w = make_uint4(word_f32(__uint_as_float(v.x), q), word_f32(__uint_as_float(v.y), q),
+                       word_f32(__uint_as_float(v.z), q), word_f32(__uint_as_float(v.w), q));
+    } else {
+        const uint64_t k0 = word_f64(__hiloint2double((int)v.y, (int)v.x), q);
+        const uint64_t k1 = word_f64(__hiloint2double((int)v.w, (int)v.z), q);
+        w = make_uint4((uint32_t)k0, (uint32_t)(k0 >> 32), (uint32_t)k1, (uint32_t)(k1 >> 32));
+    }
+    mm3p_block16(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
+}
+
+// Hash one 16-byte block with the branch-free fast rounding.  `ok` accumulates
+// "every element so far was inside the fast range" (FSETP ... AND chains, no
+// branch); a task whose warp saw any out-of-range element is redone exactly.
+template <int DT, bool RAW>
+__device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, const QuantParams &q,
+                                                 bool &ok) {
+    uint4 w;
+    if (RAW) {
+        w = v;
     } else if (DT == 0) {
         const float x0 = __uint_as_float(v.x), x1 = __uint_as_float(v.y);
         const float x2 = __uint_as_float(v.z), x3 = __uint_as_float(v.w);
-        const bool fast = (fabsf(x0) < q.r32) & (fabsf(x1) < q.r32) & (fabsf(x2) < q.r32) &
-                          (fabsf(x3) < q.r32);
-        uint32_t w0, w1, w2, w3;
-        if (fast) {
-            w0 = (uint32_t)__double2loint(__fma_rd((double)x0, q.inv, kMagic));
-            w1 = (uint32_t)__double2loint(__fma_rd((double)x1, q.inv, kMagic));
-            w2 = (uint32_t)__double2loint(__fma_rd((double)x2, q.inv, kMagic));
-            w3 = (uint32_t)__double2loint(__fma_rd((double)x3, q.inv, kMagic));
-        } else {
-            w0 = word_f32(x0, q);
-            w1 = word_f32(x1, q);
-            w2 = word_f32(x2, q);
-            w3 = word_f32(x3, q);
-        }
-        k1 = (uint64_t)w0 | ((uint64_t)w1 << 32);
-        k2 = (uint64_t)w2 | ((uint64_t)w3 << 32);
+        ok = ok & (fabsf(x0) < q.r32) & (fabsf(x1) < q.r32) & (fabsf(x2) < q.r32) &
+             (fabsf(x3) < q.r32);
+        // k mod 2^32 = low word of RD(x*inv + 1.5*2^52)   (hash.cuh)
+        w.x = (uint32_t)__double2loint(__fma_rd((double)x0, q.inv, kMagic));
+        w.y = (uint32_t)__double2loint(__fma_rd((double)x1, q.inv, kMagic));
+        w.z = (uint32_t)__double2loint(__fma_rd((double)x2, q.inv, kMagic));
+        w.w = (uint32_t)__double2loint(__fma_rd((double)x3, q.inv, kMagic));
     } else {
         const double x0 = __hiloint2double((int)v.y, (int)v.x);
         const double x1 = __hiloint2double((int)v.w, (int)v.z);
-        const bool fast = (fabs(x0) < q.r64) & (fabs(x1) < q.r64);
-        if (fast) {
-            k1 = (uint64_t)__double_as_longlong(__fma_rd(x0, q.inv, kMagic)) - kMagicBits;
-            k2 = (uint64_t)__double_as_longlong(__fma_rd(x1, q.inv, kMagic)) - kMagicBits;
-        } else {
-            k1 = word_f64(x0, q);
-            k2 = word_f64(x1, q);
-        }
+        ok = ok & (fabs(x0) < q.r64) & (fabs(x1) < q.r64);
+        // k = bits(RD(x*inv + 1.5*2^52)) - bits(1.5*2^52); the low word of the magic is 0
+        const double t0 = __fma_rd(x0, q.inv, kMagic);
+        const double t1 = __fma_rd(x1, q.inv, kMagic);
+        w.x = (uint32_t)__double2loint(t0);
+        w.y = (uint32_t)__double2hiint(t0) - 0x43380000u;
+        w.z = (uint32_t)__double2loint(t1);
+        w.w = (uint32_t)__double2hiint(t1) - 0x43380000u;
     }
-    mm3_block16(h1, h2, k1, k2);
+    mm3p_block16(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
 }
 
 // Short final block of `len` bytes (len in {4,8,12} for F32, 8 for F64),
@@ -131,110 +157,156 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
 }
 
 // CB = chunk bytes if known at compile time (multiple of kSeg), else 0.
+// A task is kRows = 32*kCh consecutive chunks of one array; lane l owns the
+// chains of rows l, l+32, ... (kCh independent chains per lane give the
+// scheduler two interleavable instruction streams).
 template <int DT, bool RAW, int CB>
-__global__ void __launch_bounds__(kLeafWarps * 32)
+__global__ void __launch_bounds__(kLeafWarps * 32, CKPT_LEAF_MINB)
 leaf_kernel(const LeafArray *__restrict__ arrays, int n_arrays, uint64_t n_tasks, uint32_t chunk_rt,
-            QuantParams q, uint4 *__restrict__ nodes) {
+            QuantParams q) {
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const uint32_t C = CB ? (uint32_t)CB : chunk_rt;
     const uint32_t n_stages = (C + kSeg - 1) / kSeg;
     const uint32_t ring = (uint32_t)__cvta_generic_to_shared(smem + warp * kWarpSmem);
-    constexpr int kPiecesPerChunk = kSeg / 16;           // 16-B pieces per chunk per stage
-    constexpr int kChunksPerInstr = 32 / kPiecesPerChunk; // chunks covered by one warp instr
-    const int my_q = lane / kPiecesPerChunk;               // chunk (within 8-group) I load
+    constexpr int kPiecesPerChunk = kSeg / 16;            // 16-B pieces per chunk per stage
+    constexpr int kChunksPerInstr = 32 / kPiecesPerChunk;  // rows covered by one warp instr
+    constexpr int kLoads = kRows / kChunksPerInstr;        // cp.async per lane per stage
+    const int my_q = lane / kPiecesPerChunk;                // first row I load
     const int my_sub = lane % kPiecesPerChunk;
-    const uint32_t my_row = ring + (uint32_t)lane * kPitch;  // the row I hash
+    const uint32_t my_row = ring + (uint32_t)lane * kPitch;  // the first row I hash
+    // keep the h*5+c addends in vector registers (a uniform-register pair cannot be the
+    // 64-bit addend of IMAD.WIDE; ptxas would split the add into IADD3 + IADD3.X)
+    {
+        uint64_t *cst = reinterpret_cast<uint64_t *>(smem + kLeafWarps * kWarpSmem);
+        if (threadIdx.x == 0) { cst[0] = q.m1; cst[1] = q.m2; }
+        __syncthreads();
+        q.m1 = *reinterpret_cast<volatile uint64_t *>(cst);
+        q.m2 = *reinterpret_cast<volatile uint64_t *>(cst + 1);
+    }
 
     for (uint64_t task = (uint64_t)blockIdx.x * kLeafWarps + warp; task < n_tasks;
          task += (uint64_t)gridDim.x * kLeafWarps) {
         const int a = find_array(arrays, n_arrays, task);
         const LeafArray A = arrays[a];
-        const uint64_t c0 = (task - A.task_begin) * 32;      // first local chunk of the task
-        const uint8_t *base = A.data + c0 * C;
-        const uint64_t my_chunk = c0 + lane;
-        const bool full_task = (C % kSeg == 0) && (c0 + 32) <= A.n_full;
-        // bytes of my (hashed) chunk
-        uint64_t my_len = 0;
-        if (my_chunk < A.n_leaves) {
-            const uint64_t off = my_chunk * C;
-            my_len = (A.nbytes - off) < C ? (A.nbytes - off) : C;
-        }
-        uint64_t h1 = 0, h2 = 0;
+        const uint64_t c0 = (task - A.task_begin) * kRows;   // first local chunk of the task
+        const bool full_task = (C % kSeg == 0) && (c0 + kRows) <= A.n_full;
+        U64p h1[kCh], h2[kCh];
+#pragma unroll
+        for (int j = 0; j < kCh; ++j) { h1[j] = U64p{0u, 0u}; h2[j] = U64p{0u, 0u}; }
+        bool done = false;
 
         if (full_task) {
-            // ---------------- fast path: 32 full chunks ----------------
-            auto issue = [&](uint32_t s) {
-                const uint32_t slot = ring + (s % kStages) * kSlotBytes;
-                const uint8_t *src = base + (uint64_t)my_q * C + s * kSeg + my_sub * 16;
-                const uint32_t dst = slot + my_q * kPitch + my_sub * 16;
+            // ---------------- fast path: kRows full chunks ----------------
+            const uint8_t *src = A.data + (c0 + my_q) * C + my_sub * 16;
+            const uint32_t dst0 = ring + my_q * kPitch + my_sub * 16;
+            auto issue = [&](const uint8_t *sp, uint32_t slot_off) {
 #pragma unroll
-                for (int i = 0; i < 32 / kChunksPerInstr; ++i)
-                    cp_async16_full(dst + i * kChunksPerInstr * kPitch,
-                                    src + (uint64_t)i * kChunksPerInstr * C);
+                for (int i = 0; i < kLoads; ++i)
+                    cp_async16_full(dst0 + slot_off + i * kChunksPerInstr * kPitch,
+                                    sp + (uint64_t)i * kChunksPerInstr * C);
             };
+            bool ok = true;
 #pragma unroll
             for (int s = 0; s < kStages - 1; ++s) {
-                if ((uint32_t)s < n_stages) issue(s);
+                if ((uint32_t)s < n_stages) issue(src + s * kSeg, s * kSlotBytes);
                 cp_async_commit();
             }
+            src += (kStages - 1) * kSeg;
+            uint32_t slot = 0u;                                   // slot of stage s
+            uint32_t nslot = (kStages - 1) * kSlotBytes;          // slot of stage s+kStages-1
             for (uint32_t s = 0; s < n_stages; ++s) {
-                if (s + kStages - 1 < n_stages) issue(s + kStages - 1);
+                if (s + kStages - 1 < n_stages) issue(src, nslot);
+                src += kSeg;
+                nslot = (nslot == (kStages - 1) * kSlotBytes) ? 0u : nslot + kSlotBytes;
                 cp_async_commit();
                 cp_async_wait<kStages - 1>();
                 __syncwarp();
-                const uint32_t row = my_row + (s % kStages) * kSlotBytes;
-#pragma unroll
-                for (int b = 0; b < kPiecesPerChunk; ++b)
-                    chain_block<DT, RAW>(h1, h2, lds128(row + b * 16), q);
-                __syncwarp();
-            }
-        } else {
-            // ------------- ragged path: the array's last task -------------
-            auto issue = [&](uint32_t s) {
-                const uint32_t slot = ring + (s % kStages) * kSlotBytes;
-#pragma unroll
-                for (int i = 0; i < 32 / kChunksPerInstr; ++i) {
-                    const int qq = my_q + i * kChunksPerInstr;
-                    const uint64_t chunk = c0 + qq;
-                    const uint64_t off = chunk * C + s * kSeg + my_sub * 16;
-                    uint32_t nb = 0;
-                    const uint64_t chunk_end_rel = (uint64_t)(s * kSeg + my_sub * 16);
-                    if (chunk < A.n_leaves && off < A.nbytes && chunk_end_rel < C) {
-                        uint64_t rem = A.nbytes - off;
-                        uint64_t crem = C - chunk_end_rel;
-                        if (crem < rem) rem = crem;
-                        nb = rem >= 16 ? 16u : (uint32_t)rem;
-                    }
-                    const uint8_t *src = nb ? (A.data + off) : A.data;
-                    cp_async16(slot + qq * kPitch + my_sub * 16, src, nb);
-                }
-            };
-#pragma unroll
-            for (int s = 0; s < kStages - 1; ++s) {
-                if ((uint32_t)s < n_stages) issue(s);
-                cp_async_commit();
-            }
-            const uint64_t full_blocks = my_len / 16;
-            for (uint32_t s = 0; s < n_stages; ++s) {
-                if (s + kStages - 1 < n_stages) issue(s + kStages - 1);
-                cp_async_commit();
-                cp_async_wait<kStages - 1>();
-                __syncwarp();
-                const uint32_t row = my_row + (s % kStages) * kSlotBytes;
+                const uint32_t row = my_row + slot;
 #pragma unroll
                 for (int b = 0; b < kPiecesPerChunk; ++b) {
-                    const uint64_t blk = (uint64_t)s * kPiecesPerChunk + b;
-                    if (blk < full_blocks) chain_block<DT, RAW>(h1, h2, lds128(row + b * 16), q);
+#pragma unroll
+                    for (int j = 0; j < kCh; ++j)
+                        chain_block_fast<DT, RAW>(h1[j], h2[j], lds128(row + j * 32 * kPitch + b * 16),
+                                                  q, ok);
                 }
                 __syncwarp();
+                slot = (slot == (kStages - 1) * kSlotBytes) ? 0u : slot + kSlotBytes;
             }
-            const uint32_t tail = (uint32_t)(my_len & 15);
-            if (tail) chain_tail<DT, RAW>(h1, h2, A.data + my_chunk * C + (my_len - tail), tail, q);
+            cp_async_wait<0>();
+            done = __all_sync(0xffffffffu, ok);
         }
-        cp_async_wait<0>();
-        if (my_chunk < A.n_leaves) nodes[A.leaf_off + my_chunk] = digest(h1, h2);
+        if (!done) {
+            // ------ exact path: ragged last task of an array, or a retry ------
+#pragma unroll 1
+            for (int j = 0; j < kCh; ++j) {
+                const uint64_t cj = c0 + 32 * j;                  // 32 chunks at a time
+                const uint64_t my_chunk = cj + lane;
+                uint64_t my_len = 0;
+                if (my_chunk < A.n_leaves) {
+                    const uint64_t off = my_chunk * C;
+                    my_len = (A.nbytes - off) < C ? (A.nbytes - off) : C;
+                }
+                U64p e1{0u, 0u}, e2{0u, 0u};
+                auto issue = [&](uint32_t s) {
+                    const uint32_t slot = ring + (s % kStages) * kSlotBytes;
+#pragma unroll
+                    for (int i = 0; i < 32 / kChunksPerInstr; ++i) {
+                        const int qq = my_q + i * kChunksPerInstr;
+                        const uint64_t chunk = cj + qq;
+                        const uint64_t rel = (uint64_t)(s * kSeg + my_sub * 16);
+                        const uint64_t off = chunk * C + rel;
+                        uint32_t nb = 0;
+                        if (chunk < A.n_leaves && off < A.nbytes && rel < C) {
+                            uint64_t rem = A.nbytes - off;
+                            const uint64_t crem = C - rel;
+                            if (crem < rem) rem = crem;
+                            nb = rem >= 16 ? 16u : (uint32_t)rem;
+                        }
+                        const uint8_t *sp = nb ? (A.data + off) : A.data;
+                        cp_async16(slot + qq * kPitch + my_sub * 16, sp, nb);
+                    }
+                };
+#pragma unroll
+                for (int s = 0; s < kStages - 1; ++s) {
+                    if ((uint32_t)s < n_stages) issue(s);
+                    cp_async_commit();
+                }
+                const uint64_t full_blocks = my_len / 16;
+                for (uint32_t s = 0; s < n_stages; ++s) {
+                    if (s + kStages - 1 < n_stages) issue(s + kStages - 1);
+                    cp_async_commit();
+                    cp_async_wait<kStages - 1>();
+                    __syncwarp();
+                    const uint32_t row = my_row + (s % kStages) * kSlotBytes;
+#pragma unroll
+                    for (int b = 0; b < kPiecesPerChunk; ++b) {
+                        const uint64_t blk = (uint64_t)s * kPiecesPerChunk + b;
+                        if (blk < full_blocks)
+                            chain_block_exact<DT, RAW>(e1, e2, lds128(row + b * 16), q);
+                    }
+                    __syncwarp();
+                }
+                cp_async_wait<0>();
+                __syncwarp();
+                const uint32_t tail = (uint32_t)(my_len & 15);
+                if (tail) {
+                    uint64_t t1 = ((uint64_t)e1.hi << 32) | e1.lo, t2 = ((uint64_t)e2.hi << 32) | e2.lo;
+                    chain_tail<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail, q);
+                    e1 = U64p{(uint32_t)t1, (uint32_t)(t1 >> 32)};
+                    e2 = U64p{(uint32_t)t2, (uint32_t)(t2 >> 32)};
+                }
+#pragma unroll
+                for (int jj = 0; jj < kCh; ++jj)
+                    if (jj == j) { h1[jj] = e1; h2[jj] = e2; }
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < kCh; ++j) {
+            const uint64_t c = c0 + 32 * j + lane;
+            if (c < A.n_leaves) A.out[c] = make_uint4(h1[j].lo, h1[j].hi, h2[j].lo, h2[j].hi);
+        }
         __syncwarp();
     }
 }

@@ -1,121 +1,188 @@
-// levels.cuh -- K2: interior Merkle levels, several levels per launch.
+// levels.cuh -- K2: interior Merkle levels, several trees, one launch.
 //
 // Paper: Alg. 1 lines 13-20 -- "for all node in level do in
 // parallel: Tree(node) <- hash({left, right})", levels bottom-up; flattened
 // array storage.  Reading R13: n_{l+1} = ceil(n_l/2), an odd last
-// node is promoted unchanged, so any aligned group of 2^G nodes of level l is
-// an exact subtree and a CTA can finish G levels of it in shared memory.
+// node is promoted unchanged, so any aligned group of 2^G nodes of a level is
+// an exact subtree.
 //
-// One launch: CTA = one aligned group of kGroup nodes of level `ls` of one
-// array -> levels ls+1 .. ls+kLog (written to global as they are formed).
-// The last CTA to finish (atomic ticket) builds every remaining level of every
-// array from L2 and then the top tree over the array roots (R15), so a whole
-// tree takes one leaf launch + one level launch.
+// Phase 1 (every CTA, no block barrier per level): a CTA of 8 warps takes an
+//   aligned group of 512 nodes of level ls of one array.  Each warp hashes its
+//   64 nodes up 6 levels with register shuffles (lane l holds node l after the
+//   first level; the right child of a level-k node comes from lane
+//   + 2^(k-2)), then warp 0 builds 3 more levels from the 8 warp roots.
+// Phase 2 (last CTA of each tree, atomic ticket): loads the remaining level
+//   of every array into shared memory, builds all upper levels there, then
+//   the top tree over the array roots (R15).  Levels that do not fit in
+//   shared memory are walked through L2.
 #pragma once
 #include <cstdint>
 
 #include "hash.cuh"
+#include "mm32.cuh"
 
 namespace ckpt {
 
-constexpr int kLevelThreads = 512;
-constexpr int kLog = 10;
-constexpr int kGroup = 1 << kLog;       // nodes of level ls per CTA
+constexpr int kLevelThreads = 256;
+constexpr int kLog = 9;
+constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA
+constexpr int kLevelSmemNodes = 6144;        // phase-2 shared memory in nodes (96 KiB)
+constexpr int kLevelSmem = kLevelSmemNodes * 16;
+constexpr int kMaxLevelTrees = 4;
 
 struct LevelParams {
     uint4 *nodes;                 // whole tree storage
     const uint64_t *off;          // [level * n_arrays + a]: node index of array a's level
     const uint64_t *cnt;          // [level * n_arrays + a]: node count (0 above the array's root)
-    const uint64_t *gbegin;       // [a]: first CTA of array a (prefix of ceil(cnt[ls][a]/kGroup))
+    const uint64_t *gbegin;       // [a]: first group of array a (prefix of ceil(cnt[ls][a]/kGroup))
     const uint64_t *level_base;   // [level]: node index of level (all arrays, concatenated)
     const uint64_t *level_total;  // [level]: nodes in level (all arrays)
     const uint32_t *height;       // [a]: number of levels of array a
     uint64_t top_off;             // node index of the top tree's level 0
-    unsigned int *ticket;         // zero-initialised counter
+    unsigned int *ticket;         // zero-initialised counter (reset by the last CTA)
     int n_arrays;
     int n_levels;                 // max height over arrays
     int ls;                       // start level of this launch
+    unsigned int n_groups;        // CTAs of this tree
 };
 
-__device__ __forceinline__ int find_group_array(const uint64_t *gbegin, int n_arrays, uint64_t g) {
-    int lo = 0, hi = n_arrays - 1;
+struct LevelBatch {
+    LevelParams t[kMaxLevelTrees];
+    unsigned int cta_begin[kMaxLevelTrees + 1];
+    int n;
+};
+
+__device__ __forceinline__ int find_le(const uint64_t *v, int n, uint64_t x) {
+    int lo = 0, hi = n - 1;
     while (lo < hi) {
         const int mid = (lo + hi + 1) >> 1;
-        if (gbegin[mid] <= g) lo = mid; else hi = mid - 1;
+        if (v[mid] <= x) lo = mid; else hi = mid - 1;
     }
     return lo;
 }
 
-__device__ __forceinline__ int find_level_array(const uint64_t *off_l, int n_arrays, uint64_t idx) {
-    int lo = 0, hi = n_arrays - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (off_l[mid] <= idx) lo = mid; else hi = mid - 1;
-    }
-    return lo;
+__device__ __forceinline__ uint4 shfl_down4(uint4 v, int d) {
+    return make_uint4(__shfl_down_sync(0xffffffffu, v.x, d), __shfl_down_sync(0xffffffffu, v.y, d),
+                      __shfl_down_sync(0xffffffffu, v.z, d), __shfl_down_sync(0xffffffffu, v.w, d));
 }
 
-__global__ void __launch_bounds__(kLevelThreads) levels_kernel(LevelParams p) {
-    __shared__ uint4 buf[kGroup];
-    __shared__ unsigned int s_ticket;
-    const int tid = threadIdx.x;
+// Levels k0..k1 (relative to the warp's level-(k0-1) nodes held one per lane
+// in `v`, `m` of them valid) with shuffles.  Node j of relative level k lives
+// in lane j << (k - k0 + 1) ... written to global through `write(k, j, v)`.
+template <class W>
+__device__ __forceinline__ uint4 warp_levels(uint4 v, int m, int k0, int k1, int lane, W write) {
+    for (int k = k0, step = 1; k <= k1; ++k, step <<= 1) {
+        const uint4 r = shfl_down4(v, step);
+        const int mk = (m + 1) >> 1;
+        const int j = lane / (2 * step);
+        if ((lane & (2 * step - 1)) == 0 && j < mk) {
+            if (2 * j + 1 < m) v = hash_children32(v, r);
+            write(k, j, v);
+        }
+        m = mk;
+    }
+    return v;
+}
+
+// One level over all arrays, children read from `src` (indexable by node
+// index - src_base) and parents written to global and, if dst != null, to dst.
+__device__ __forceinline__ void build_level(const LevelParams &p, int l, const uint4 *src,
+                                            uint64_t src_base, uint4 *dst, bool from_global) {
     const int na = p.n_arrays;
+    const uint64_t total = p.level_total[l];
+    const uint64_t base = p.level_base[l];
+    const uint64_t *off_l = p.off + (uint64_t)l * na;
+    const uint64_t *off_d = p.off + (uint64_t)(l - 1) * na;
+    const uint64_t *cnt_d = p.cnt + (uint64_t)(l - 1) * na;
+    for (uint64_t i = threadIdx.x; i < total; i += blockDim.x) {
+        const int a = find_le(off_l, na, base + i);
+        const uint64_t j = base + i - off_l[a];
+        const uint64_t c = off_d[a] + 2 * j - src_base;
+        uint4 v = from_global ? __ldcg(src + c) : src[c];
+        if (2 * j + 1 < cnt_d[a]) v = hash_children32(v, from_global ? __ldcg(src + c + 1) : src[c + 1]);
+        p.nodes[base + i] = v;
+        if (dst) dst[i] = v;
+    }
+}
+
+__global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_constant__ LevelBatch pb) {
+    extern __shared__ __align__(16) uint4 sm[];
+    __shared__ uint4 s_root[kLevelThreads / 32];
+    __shared__ unsigned int s_ticket;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    int ti = 0;
+    while (ti + 1 < pb.n && blockIdx.x >= pb.cta_begin[ti + 1]) ++ti;
+    const LevelParams &p = pb.t[ti];
+    const int na = p.n_arrays;
+    // ------------------------------ phase 1 ------------------------------
     {
-        const int a = find_group_array(p.gbegin, na, blockIdx.x);
-        const uint64_t g = blockIdx.x - p.gbegin[a];
+        const uint64_t gid = blockIdx.x - pb.cta_begin[ti];
+        const int a = find_le(p.gbegin, na, gid);
+        const uint64_t g = gid - p.gbegin[a];
         const uint64_t n0 = p.cnt[(uint64_t)p.ls * na + a];
         const uint64_t start = g * kGroup;
-        int m = (int)((n0 - start) < (uint64_t)kGroup ? (n0 - start) : (uint64_t)kGroup);
-        const uint4 *src = p.nodes + p.off[(uint64_t)p.ls * na + a] + start;
-        for (int i = tid; i < m; i += kLevelThreads) buf[i] = src[i];
+        const int m0 = (int)((n0 - start) < (uint64_t)kGroup ? (n0 - start) : (uint64_t)kGroup);
         const int h = (int)p.height[a];
-        for (int k = 1; k <= kLog && p.ls + k < h; ++k) {
-            const int mk = (m + 1) >> 1;
-            __syncthreads();
-            uint4 v[kGroup / 2 / kLevelThreads > 0 ? kGroup / 2 / kLevelThreads : 1];
-#pragma unroll
-            for (int r = 0; r < (kGroup / 2 + kLevelThreads - 1) / kLevelThreads; ++r) {
-                const int j = tid + r * kLevelThreads;
-                if (j < mk) v[r] = (2 * j + 1 < m) ? hash_children(buf[2 * j], buf[2 * j + 1]) : buf[2 * j];
-            }
-            __syncthreads();
-            uint4 *dst = p.nodes + p.off[(uint64_t)(p.ls + k) * na + a] + (start >> k);
-#pragma unroll
-            for (int r = 0; r < (kGroup / 2 + kLevelThreads - 1) / kLevelThreads; ++r) {
-                const int j = tid + r * kLevelThreads;
-                if (j < mk) {
-                    buf[j] = v[r];
-                    dst[j] = v[r];
-                }
-            }
-            m = mk;
+        const uint4 *src = p.nodes + p.off[(uint64_t)p.ls * na + a] + start;
+        auto write = [&](int k, uint64_t jglob, uint4 v) {
+            if (p.ls + k < h) p.nodes[p.off[(uint64_t)(p.ls + k) * na + a] + (start >> k) + jglob] = v;
+        };
+        // warp w: nodes [64w, 64w+64) of the group
+        int mw = m0 - 64 * warp;
+        mw = mw < 0 ? 0 : (mw > 64 ? 64 : mw);
+        uint4 v = make_uint4(0u, 0u, 0u, 0u);
+        if (2 * lane < mw) {
+            v = src[64 * warp + 2 * lane];
+            if (2 * lane + 1 < mw) v = hash_children32(v, src[64 * warp + 2 * lane + 1]);
+            write(1, 32 * warp + lane, v);
         }
-    }
-    // ---- last CTA: remaining levels of every array, then the top tree ----
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) s_ticket = atomicAdd(p.ticket, 1u);
-    __syncthreads();
-    if (s_ticket != gridDim.x - 1) return;
-    __threadfence();
-    for (int l = p.ls + kLog + 1; l < p.n_levels; ++l) {
-        const uint64_t total = p.level_total[l];
-        const uint64_t base = p.level_base[l];
-        const uint64_t *off_l = p.off + (uint64_t)l * na;
-        const uint64_t *off_d = p.off + (uint64_t)(l - 1) * na;
-        const uint64_t *cnt_d = p.cnt + (uint64_t)(l - 1) * na;
-        for (uint64_t i = tid; i < total; i += kLevelThreads) {
-            const int a = find_level_array(off_l, na, base + i);
-            const uint64_t j = base + i - off_l[a];
-            const uint64_t nd = cnt_d[a];
-            const uint4 *c = p.nodes + off_d[a];
-            uint4 v = __ldcg(c + 2 * j);
-            if (2 * j + 1 < nd) v = hash_children(v, __ldcg(c + 2 * j + 1));
-            p.nodes[base + i] = v;
-        }
+        int m1 = (mw + 1) >> 1;
+        v = warp_levels(v, m1, 2, 6, lane, [&](int k, int j, uint4 x) {
+            write(k, (uint64_t)(64 >> k) * warp + j, x);
+        });
+        if (lane == 0) s_root[warp] = v;
         __syncthreads();
+        if (warp == 0) {
+            const int m6 = (m0 + 63) >> 6;       // valid warp roots
+            uint4 x = lane < m6 ? s_root[lane] : make_uint4(0u, 0u, 0u, 0u);
+            warp_levels(x, m6, 7, kLog, lane, [&](int k, int j, uint4 y) { write(k, j, y); });
+        }
     }
-    // top tree: level 0 = array roots in array order
+    // ------------------------------ phase 2 ------------------------------
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        s_ticket = atomicAdd(p.ticket, 1u);
+    }
+    __syncthreads();
+    if (s_ticket != p.n_groups - 1) return;
+    __threadfence();
+    int F = p.ls + kLog;                       // highest level phase 1 completed
+    if (F > p.n_levels - 1) F = p.n_levels - 1;
+    if (F + 1 <= p.n_levels - 1) {
+        const uint64_t nF = p.level_total[F];
+        const uint64_t nF1 = p.level_total[F + 1];
+        if (nF + nF1 <= (uint64_t)kLevelSmemNodes) {
+            // whole remainder in shared memory: ping-pong between two regions
+            uint4 *cur = sm, *nxt = sm + nF;
+            for (uint64_t i = tid; i < nF; i += kLevelThreads) cur[i] = __ldcg(p.nodes + p.level_base[F] + i);
+            __syncthreads();
+            for (int l = F + 1; l < p.n_levels; ++l) {
+                build_level(p, l, cur, p.level_base[l - 1], nxt, false);
+                __syncthreads();
+                uint4 *t = cur;
+                cur = nxt;
+                nxt = t;
+            }
+        } else {
+            for (int l = F + 1; l < p.n_levels; ++l) {
+                build_level(p, l, p.nodes + p.level_base[l - 1], p.level_base[l - 1], nullptr, true);
+                __syncthreads();
+            }
+        }
+    }
+    __syncthreads();
+    // top tree: level 0 = array roots in array order (R15), built in L2 (tiny)
     for (int a = tid; a < na; a += kLevelThreads) {
         const int h = (int)p.height[a];
         p.nodes[p.top_off + a] = __ldcg(p.nodes + p.off[(uint64_t)(h - 1) * na + a]);
@@ -125,9 +192,9 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(LevelParams p) {
     while (n > 1) {
         const uint64_t up = (n + 1) >> 1;
         for (uint64_t j = tid; j < up; j += kLevelThreads) {
-            uint4 v = __ldcg(p.nodes + cur + 2 * j);
-            if (2 * j + 1 < n) v = hash_children(v, __ldcg(p.nodes + cur + 2 * j + 1));
-            p.nodes[cur + n + j] = v;
+            uint4 x = __ldcg(p.nodes + cur + 2 * j);
+            if (2 * j + 1 < n) x = hash_children32(x, __ldcg(p.nodes + cur + 2 * j + 1));
+            p.nodes[cur + n + j] = x;
         }
         __syncthreads();
         cur += n;

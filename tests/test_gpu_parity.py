@@ -155,6 +155,21 @@ def test_multi_array_checkpoint_matches_oracle():
     assert n == ref.size and np.array_equal(np_of(idx), ref)
 
 
+def test_batch_build_equals_separate_builds():
+    sizes_a = [1000, 65536 + 17, 5]
+    arrs_a = [_data(n, torch.float32, 300 + i) for i, n in enumerate(sizes_a)]
+    arrs_b = [t.clone() for t in arrs_a]
+    arrs_b[1][12345] += 1.0
+    arrs_c = [_data(n, torch.float32, 400 + i) for i, n in enumerate([7, 4096 * 33])]
+    TA, TB, TC = ck.tree_build_batch([arrs_a, arrs_b, arrs_c], 512, 1e-5)
+    for T, arrs in ((TA, arrs_a), (TB, arrs_b), (TC, arrs_c)):
+        R = oracle.build_checkpoint([np_of(t) for t in arrs], 512, 1e-5)
+        assert T.root() == R.root
+        for k in range(len(arrs)):
+            assert np.array_equal(gpu_tree_nodes(T, k), R.trees[k])
+    assert np.array_equal(np_of(ck.tree_diff(TA, TB)), [1000 * 4 // 512 + 1 + 12345 * 4 // 512])
+
+
 # ------------------------------------------------------------ diff/verify --
 
 @pytest.mark.parametrize("n", [1 << 20, 1_000_000])
