@@ -245,6 +245,8 @@ def run_ours(args):
             keep[:] = [TA, TB, *tops, tot]
         else:
             keep[:] = [TA, TB]
+        TA.wait()          # the step ends when both trees are complete (K2 runs on a side stream)
+        TB.wait()
 
     for _ in range(max(3, args.warmup)):
         step()

@@ -212,6 +212,13 @@ ckpt_status ckpt_compare_host(const void *const *a, const void *const *b, const 
  * Accessors (parity tests, multi-GPU driver)
  * ---------------------------------------------------------------------- */
 
+/* Make `stream` wait until every level of the tree is built.  The library's
+ * own entry points do this when they need interior nodes (K2 runs on an
+ * internal side stream so that it overlaps a leaf-level diff and the
+ * verify); call it before reading tree memory by other means, or to end a
+ * timed region.  Asynchronous. */
+ckpt_status ckpt_tree_wait(const ckpt_tree *t, void *stream);
+
 /* (host outputs, any may be NULL) number of arrays, total leaves (= total
  * chunks), number of levels of the tallest array tree, total stored nodes
  * (all arrays, all levels; excludes the top tree over array roots). */

@@ -77,6 +77,7 @@ def lib():
     L.ckpt_compare.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, vp, u64, vp, u64, pu64, pu64, vp,
                                vp, vp]
     L.ckpt_compare_host.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, vp, u64, pu64, pu64, vp, vp]
+    L.ckpt_tree_wait.argtypes = [vp, vp]
     L.ckpt_tree_info.argtypes = [vp, ctypes.POINTER(u32), pu64, ctypes.POINTER(u32), pu64]
     L.ckpt_tree_root.argtypes = [vp, vp, vp]
     L.ckpt_tree_array_roots.argtypes = [vp, vp, vp]
@@ -98,7 +99,7 @@ def lib():
                  "ckpt_tree_diff", "ckpt_tree_diff_async", "ckpt_verify",
                  "ckpt_verify_arrays_async", "ckpt_compare", "ckpt_compare_host",
                  "ckpt_tree_info", "ckpt_tree_root", "ckpt_tree_array_roots", "ckpt_tree_nodes",
-                 "ckpt_tree_array_info"):
+                 "ckpt_tree_array_info", "ckpt_tree_wait"):
         getattr(L, name).restype = i32
     _lib = L
     return L
@@ -180,6 +181,10 @@ class Tree:
         if self._h is None or not self._h.value:
             raise ValueError("tree already freed")
         return self._h
+
+    def wait(self, stream=None):
+        """Make `stream` wait until all levels are built (they build on a side stream)."""
+        _check(lib().ckpt_tree_wait(self.handle, _stream_ptr(stream)), "ckpt_tree_wait")
 
     def root(self, stream=None) -> bytes:
         out = (ctypes.c_uint8 * 16)()

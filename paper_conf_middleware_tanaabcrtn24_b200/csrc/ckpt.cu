@@ -98,6 +98,16 @@ struct DevInfo {
 static std::mutex g_dev_mu;
 static DevInfo g_dev[64];
 
+static cudaStream_t g_side[64];
+
+// Per-device non-blocking side stream for K2.
+static ckpt_status side_stream(int dev, cudaStream_t *out) {
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    if (!g_side[dev & 63]) CK_CUDA(cudaStreamCreateWithFlags(&g_side[dev & 63], cudaStreamNonBlocking));
+    *out = g_side[dev & 63];
+    return CKPT_OK;
+}
+
 static ckpt_status dev_info(int *dev_out, DevInfo *info) {
     int dev = 0;
     CK_CUDA(cudaGetDevice(&dev));
@@ -203,7 +213,15 @@ struct ckpt_tree {
     const uint64_t *d_gbegin = nullptr;
     unsigned *d_ticket = nullptr;
     uint64_t n_groups = 0;
+    cudaEvent_t levels_done = nullptr;     // recorded after K2 (on the side stream)
 };
+
+// Work that reads a tree's interior levels or roots waits for K2 first (K2
+// runs on a side stream so it overlaps the leaf-only diff and the verify).
+static ckpt_status wait_levels(const ckpt_tree *t, cudaStream_t s) {
+    if (t && t->levels_done) CK_CUDA(cudaStreamWaitEvent(s, t->levels_done, 0));
+    return CKPT_OK;
+}
 
 static uint32_t tree_height(uint64_t L) {
     uint32_t h = 1;
@@ -490,7 +508,23 @@ extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint
         a0 += na;
     }
     if (st == CKPT_OK) st = launch_leaves(table, task, dtype, eps, chunk_bytes, s, di.sms);
-    if (st == CKPT_OK) st = launch_levels(out, (int)n_trees, s);
+    if (st == CKPT_OK) {
+        // K2 on the side stream, after the leaves; each tree records its own event
+        cudaStream_t ss = nullptr;
+        cudaEvent_t leaves_done = nullptr;
+        st = side_stream(dev, &ss);
+        if (st == CKPT_OK && (cudaEventCreateWithFlags(&leaves_done, cudaEventDisableTiming) != cudaSuccess ||
+                              cudaEventRecord(leaves_done, s) != cudaSuccess ||
+                              cudaStreamWaitEvent(ss, leaves_done, 0) != cudaSuccess))
+            st = fail(CKPT_ECUDA, "side-stream fork");
+        if (leaves_done) cudaEventDestroy(leaves_done);
+        if (st == CKPT_OK) st = launch_levels(out, (int)n_trees, ss);
+        for (uint32_t k = 0; k < n_trees && st == CKPT_OK; ++k) {
+            if (cudaEventCreateWithFlags(&out[k]->levels_done, cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventRecord(out[k]->levels_done, ss) != cudaSuccess)
+                st = fail(CKPT_ECUDA, "side-stream join event");
+        }
+    }
     if (st != CKPT_OK) {
         for (uint32_t k = 0; k < n_trees; ++k) { ckpt_tree_free_on(out[k], stream); out[k] = nullptr; }
         return st;
@@ -547,6 +581,10 @@ extern "C" void ckpt_tree_free_on(ckpt_tree *t, void *stream) {
     int cur = 0;
     cudaGetDevice(&cur);
     if (cur != t->device) cudaSetDevice(t->device);
+    if (t->levels_done) {
+        cudaStreamWaitEvent(s, t->levels_done, 0);
+        cudaEventDestroy(t->levels_done);
+    }
     if (t->nodes) cudaFreeAsync(t->nodes, s);
     if (t->meta) cudaFreeAsync(t->meta, s);
     if (cur != t->device) cudaSetDevice(cur);
@@ -619,6 +657,10 @@ extern "C" ckpt_status ckpt_tree_diff_async(const ckpt_tree *a, const ckpt_tree 
             tot += a->cnt[(size_t)ll * na + k];
         }
         if (tot >= T) { l0 = (uint32_t)l; break; }
+    }
+    if (l0 > 0) {
+        CK_TRY(wait_levels(a, s));
+        CK_TRY(wait_levels(b, s));
     }
     if (l0 == 0) {
         return launch_compact(0, a->nodes, b->nodes, nullptr, a->total_leaves, chunks, cap,
@@ -804,6 +846,7 @@ extern "C" ckpt_status ckpt_verify(const void *a, const void *b, uint64_t n, ckp
 extern "C" ckpt_status ckpt_tree_root(const ckpt_tree *t, uint8_t out16[16], void *stream) {
     if (!t || !out16) return fail(CKPT_EINVAL, "NULL argument");
     cudaStream_t s = (cudaStream_t)stream;
+    CK_TRY(wait_levels(t, s));
     CK_CUDA(cudaMemcpyAsync(out16, t->nodes + t->top_off + t->top_nodes - 1, 16,
                             cudaMemcpyDeviceToHost, s));
     CK_CUDA(cudaStreamSynchronize(s));
@@ -939,6 +982,11 @@ extern "C" ckpt_status ckpt_compare_host(const void *const *a, const void *const
 // ---------------------------------------------------------------------------
 // accessors
 // ---------------------------------------------------------------------------
+extern "C" ckpt_status ckpt_tree_wait(const ckpt_tree *t, void *stream) {
+    if (!t) return fail(CKPT_EINVAL, "NULL tree");
+    return wait_levels(t, (cudaStream_t)stream);
+}
+
 extern "C" ckpt_status ckpt_tree_info(const ckpt_tree *t, uint32_t *n_arrays, uint64_t *n_leaves,
                                       uint32_t *n_levels, uint64_t *n_nodes) {
     if (!t) return fail(CKPT_EINVAL, "NULL tree");
@@ -951,6 +999,7 @@ extern "C" ckpt_status ckpt_tree_info(const ckpt_tree *t, uint32_t *n_arrays, ui
 
 extern "C" ckpt_status ckpt_tree_array_roots(const ckpt_tree *t, void *dst, void *stream) {
     if (!t || !dst) return fail(CKPT_EINVAL, "NULL argument");
+    CK_TRY(wait_levels(t, (cudaStream_t)stream));
     CK_CUDA(cudaMemcpyAsync(dst, t->nodes + t->top_off, (size_t)t->n_arrays * 16,
                             cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
     return CKPT_OK;
@@ -971,6 +1020,7 @@ extern "C" ckpt_status ckpt_tree_nodes(const ckpt_tree *t, uint32_t array, void 
     uint64_t nn = 0;
     CK_TRY(ckpt_tree_array_info(t, array, nullptr, &nn));
     if (!dst || cap_bytes < nn * 16) return fail(CKPT_EINVAL, "destination too small");
+    CK_TRY(wait_levels(t, (cudaStream_t)stream));
     uint8_t *d = (uint8_t *)dst;
     for (uint32_t l = 0; l < t->height[array]; ++l) {
         const size_t i = (size_t)l * t->n_arrays + array;

@@ -104,13 +104,19 @@ __device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, co
     } else if (DT == 0) {
         const float x0 = __uint_as_float(v.x), x1 = __uint_as_float(v.y);
         const float x2 = __uint_as_float(v.z), x3 = __uint_as_float(v.w);
+        const double d0 = (double)x0, d1 = (double)x1, d2 = (double)x2, d3 = (double)x3;
+#ifdef CKPT_RANGE_F64
+        // range test on the FP64 pipe (DSETP) instead of the ALU pipe
+        ok = ok & (fabs(d0) < q.r64) & (fabs(d1) < q.r64) & (fabs(d2) < q.r64) & (fabs(d3) < q.r64);
+#else
         ok = ok & (fabsf(x0) < q.r32) & (fabsf(x1) < q.r32) & (fabsf(x2) < q.r32) &
              (fabsf(x3) < q.r32);
+#endif
         // k mod 2^32 = low word of RD(x*inv + 1.5*2^52)   (hash.cuh)
-        w.x = (uint32_t)__double2loint(__fma_rd((double)x0, q.inv, kMagic));
-        w.y = (uint32_t)__double2loint(__fma_rd((double)x1, q.inv, kMagic));
-        w.z = (uint32_t)__double2loint(__fma_rd((double)x2, q.inv, kMagic));
-        w.w = (uint32_t)__double2loint(__fma_rd((double)x3, q.inv, kMagic));
+        w.x = (uint32_t)__double2loint(__fma_rd(d0, q.inv, kMagic));
+        w.y = (uint32_t)__double2loint(__fma_rd(d1, q.inv, kMagic));
+        w.z = (uint32_t)__double2loint(__fma_rd(d2, q.inv, kMagic));
+        w.w = (uint32_t)__double2loint(__fma_rd(d3, q.inv, kMagic));
     } else {
         const double x0 = __hiloint2double((int)v.y, (int)v.x);
         const double x1 = __hiloint2double((int)v.w, (int)v.z);
