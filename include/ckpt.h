@@ -258,6 +258,11 @@ uint64_t ckpt_launch_count(void);
 void ckpt_profile_enable(int on);
 void ckpt_profile_reset(void);
 ckpt_status ckpt_profile_read(int k, double *ms, uint64_t *launches);
+/* Timeline of the recorded launches since the last reset: for record i,
+ * out[3i] = kernel family, out[3i+1] / out[3i+2] = start / end in ms relative
+ * to the first record's start (host, cap records).  *n_records (host) = the
+ * number recorded.  Synchronises the recorded events. */
+ckpt_status ckpt_profile_timeline(double *out, uint64_t cap, uint64_t *n_records);
 
 const char *ckpt_strerror(ckpt_status s);
 /* Thread-local detail of the last error returned on this thread. */

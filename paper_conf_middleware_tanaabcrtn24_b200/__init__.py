@@ -88,6 +88,8 @@ def lib():
     L.ckpt_profile_reset.restype = None
     L.ckpt_profile_read.argtypes = [i32, ctypes.POINTER(dbl), pu64]
     L.ckpt_profile_read.restype = i32
+    L.ckpt_profile_timeline.argtypes = [ctypes.POINTER(dbl), u64, pu64]
+    L.ckpt_profile_timeline.restype = i32
     L.ckpt_default_bfs_threshold.restype = u64
     L.ckpt_launch_count.restype = u64
     L.ckpt_strerror.argtypes = [i32]
@@ -402,3 +404,13 @@ def profile_read(kernel: str) -> Tuple[float, int]:
     _check(lib().ckpt_profile_read(KERNELS[kernel], ctypes.byref(ms), ctypes.byref(n)),
            "ckpt_profile_read")
     return ms.value, n.value
+
+
+def profile_timeline():
+    """[(kernel, start_ms, end_ms)] of the recorded launches (relative to the first start)."""
+    n = ctypes.c_uint64()
+    _check(lib().ckpt_profile_timeline(None, 0, ctypes.byref(n)), "ckpt_profile_timeline")
+    buf = (ctypes.c_double * (3 * max(n.value, 1)))()
+    _check(lib().ckpt_profile_timeline(buf, n.value, ctypes.byref(n)), "ckpt_profile_timeline")
+    names = {v: k for k, v in KERNELS.items()}
+    return [(names.get(int(buf[3 * i]), "?"), buf[3 * i + 1], buf[3 * i + 2]) for i in range(n.value)]

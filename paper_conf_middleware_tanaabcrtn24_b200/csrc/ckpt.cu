@@ -11,8 +11,10 @@
 #include <cfloat>
 #include <cmath>
 #include <cstdio>
+#include <cstddef>
 #include <cstring>
 #include <deque>
+#include <map>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -103,7 +105,12 @@ static cudaStream_t g_side[64];
 // Per-device non-blocking side stream for K2.
 static ckpt_status side_stream(int dev, cudaStream_t *out) {
     std::lock_guard<std::mutex> lk(g_dev_mu);
-    if (!g_side[dev & 63]) CK_CUDA(cudaStreamCreateWithFlags(&g_side[dev & 63], cudaStreamNonBlocking));
+    if (!g_side[dev & 63]) {
+        // lowest priority: K2's CTAs only take SM slots the diff/verify kernels leave free
+        int lo = 0, hi = 0;
+        CK_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        CK_CUDA(cudaStreamCreateWithPriority(&g_side[dev & 63], cudaStreamNonBlocking, lo));
+    }
     *out = g_side[dev & 63];
     return CKPT_OK;
 }
@@ -211,9 +218,10 @@ struct ckpt_tree {
                    *d_level_total = nullptr, *d_chunk_base = nullptr;
     const uint32_t *d_height = nullptr;
     const uint64_t *d_gbegin = nullptr;
-    unsigned *d_ticket = nullptr;
     uint64_t n_groups = 0;
     cudaEvent_t levels_done = nullptr;     // recorded after K2 (on the side stream)
+    std::vector<uint64_t> meta_host;       // the device blob's contents (8-byte words)
+    uint32_t o_off = 0, o_cnt = 0, o_lb = 0, o_lt = 0, o_cb = 0, o_h = 0, o_g = 0;
 };
 
 // Work that reads a tree's interior levels or roots waits for K2 first (K2
@@ -309,8 +317,8 @@ static ckpt_status check_common(ckpt_dtype dtype, uint32_t chunk_bytes, double e
 }
 
 template <int DT, bool RAW, int CB>
-static ckpt_status launch_leaf_t(const LeafArray *arr, int na, uint64_t tasks, uint32_t C,
-                                 const QuantParams &q, cudaStream_t s, int sms) {
+static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
+    const uint64_t tasks = P.n_tasks;
     auto k = leaf_kernel<DT, RAW, CB>;
     static std::atomic<int> cached_per_sm{0};
     int per_sm = cached_per_sm.load(std::memory_order_relaxed);
@@ -325,54 +333,76 @@ static ckpt_status launch_leaf_t(const LeafArray *arr, int na, uint64_t tasks, u
     uint64_t want = (tasks + kLeafWarps - 1) / kLeafWarps;
     uint64_t grid = std::min<uint64_t>(want, (uint64_t)sms * per_sm);
     ProfScope prof(0, s);
-    k<<<(unsigned)grid, kLeafWarps * 32, kLeafSmem, s>>>(arr, na, tasks, C, q);
+    k<<<(unsigned)grid, kLeafWarps * 32, kLeafSmem, s>>>(P);
     CK_LAUNCH();
     return CKPT_OK;
 }
 
 template <int DT, bool RAW>
-static ckpt_status launch_leaf_dt(const LeafArray *arr, int na, uint64_t tasks, uint32_t C,
-                                  const QuantParams &q, cudaStream_t s, int sms) {
+static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms) {
+    const uint32_t C = P.chunk;
     if (!RAW) {
         switch (C) {
-            case 512: return launch_leaf_t<DT, RAW, 512>(arr, na, tasks, C, q, s, sms);
-            case 1024: return launch_leaf_t<DT, RAW, 1024>(arr, na, tasks, C, q, s, sms);
-            case 2048: return launch_leaf_t<DT, RAW, 2048>(arr, na, tasks, C, q, s, sms);
-            case 4096: return launch_leaf_t<DT, RAW, 4096>(arr, na, tasks, C, q, s, sms);
-            case 8192: return launch_leaf_t<DT, RAW, 8192>(arr, na, tasks, C, q, s, sms);
-            case 16384: return launch_leaf_t<DT, RAW, 16384>(arr, na, tasks, C, q, s, sms);
-            case 32768: return launch_leaf_t<DT, RAW, 32768>(arr, na, tasks, C, q, s, sms);
-            case 65536: return launch_leaf_t<DT, RAW, 65536>(arr, na, tasks, C, q, s, sms);
+            case 512: return launch_leaf_t<DT, RAW, 512>(P, s, sms);
+            case 1024: return launch_leaf_t<DT, RAW, 1024>(P, s, sms);
+            case 2048: return launch_leaf_t<DT, RAW, 2048>(P, s, sms);
+            case 4096: return launch_leaf_t<DT, RAW, 4096>(P, s, sms);
+            case 8192: return launch_leaf_t<DT, RAW, 8192>(P, s, sms);
+            case 16384: return launch_leaf_t<DT, RAW, 16384>(P, s, sms);
+            case 32768: return launch_leaf_t<DT, RAW, 32768>(P, s, sms);
+            case 65536: return launch_leaf_t<DT, RAW, 65536>(P, s, sms);
             default: break;
         }
     }
-    return launch_leaf_t<DT, RAW, 0>(arr, na, tasks, C, q, s, sms);
+    return launch_leaf_t<DT, RAW, 0>(P, s, sms);
 }
 
 // K2 for up to kMaxLevelTrees trees in one launch.
+static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_t **states,
+                               unsigned long long **ticket, uint32_t *epoch);
+
 static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s) {
     static std::atomic<int> attr_done{0};
     if (!attr_done.load()) {
         CK_CUDA(cudaFuncSetAttribute(levels_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kLevelSmem));
         attr_done.store(1);
     }
+    int dev = 0;
+    CK_CUDA(cudaGetDevice(&dev));
+    uint64_t *unused_states;
+    unsigned long long *tickets;
+    uint32_t unused_epoch;
+    CK_TRY(get_scratch(dev, s, 0, &unused_states, &tickets, &unused_epoch));
+    static LevelBatch b;                      // large (kernel parameters); filled per launch
+    static std::mutex b_mu;
+    std::lock_guard<std::mutex> lk(b_mu);
     for (int k0 = 0; k0 < n; k0 += kMaxLevelTrees) {
-        LevelBatch b;
-        std::memset(&b, 0, sizeof(b));
+        std::memset(&b, 0, offsetof(LevelBatch, blob));
         b.n = std::min(kMaxLevelTrees, n - k0);
         unsigned ctas = 0;
+        uint32_t words = 0;
         for (int i = 0; i < b.n; ++i) {
-            const ckpt_tree *t = trees[k0 + i];
+            ckpt_tree *t = trees[k0 + i];
             LevelParams &p = b.t[i];
             p.nodes = t->nodes;
-            p.off = t->d_off;
-            p.cnt = t->d_cnt;
-            p.gbegin = t->d_gbegin;
-            p.level_base = t->d_level_base;
-            p.level_total = t->d_level_total;
-            p.height = t->d_height;
+            p.meta = t->meta;
+            p.meta_words = (uint32_t)t->meta_host.size();
+            if (words + p.meta_words <= (uint32_t)kLevelInlineWords) {
+                std::memcpy(b.blob + words, t->meta_host.data(), (size_t)p.meta_words * 8);
+                p.inl = (int)words;
+                words += p.meta_words;
+            } else {
+                p.inl = -1;
+                CK_TRY(g_ring.copy(t->meta, t->meta_host.data(), t->meta_host.size() * 8, s));
+            }
+            p.o_off = t->o_off;
+            p.o_cnt = t->o_cnt;
+            p.o_lb = t->o_lb;
+            p.o_lt = t->o_lt;
+            p.o_h = t->o_h;
+            p.o_g = t->o_g;
             p.top_off = t->top_off;
-            p.ticket = t->d_ticket;
+            p.ticket = reinterpret_cast<unsigned int *>(tickets + 1 + i);   // slot 0: compactions
             p.n_arrays = (int)t->n_arrays;
             p.n_levels = (int)t->n_levels;
             p.ls = 0;
@@ -399,55 +429,64 @@ static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
         groups += (t->cnt[a] + kGroup - 1) / kGroup;   // level 0 counts
     }
     t->n_groups = groups;
-    const size_t o_off = 0;
-    const size_t o_cnt = align256(o_off + t->off.size() * 8);
-    const size_t o_lb = align256(o_cnt + t->cnt.size() * 8);
-    const size_t o_lt = align256(o_lb + t->level_base.size() * 8);
-    const size_t o_cb = align256(o_lt + t->level_total.size() * 8);
-    const size_t o_h = align256(o_cb + (size_t)na * 8);
-    const size_t o_g = align256(o_h + (size_t)na * 4);
-    const size_t o_tk = align256(o_g + (size_t)na * 8);
-    const size_t total = align256(o_tk + 16);
-    std::vector<uint8_t> blob(total, 0);
-    std::memcpy(blob.data() + o_off, t->off.data(), t->off.size() * 8);
-    std::memcpy(blob.data() + o_cnt, t->cnt.data(), t->cnt.size() * 8);
-    std::memcpy(blob.data() + o_lb, t->level_base.data(), t->level_base.size() * 8);
-    std::memcpy(blob.data() + o_lt, t->level_total.data(), t->level_total.size() * 8);
-    std::memcpy(blob.data() + o_cb, t->chunk_base.data(), (size_t)na * 8);
-    std::memcpy(blob.data() + o_h, t->height.data(), (size_t)na * 4);
-    std::memcpy(blob.data() + o_g, gbegin.data(), (size_t)na * 8);
+    auto al8 = [](size_t x) { return (x + 7) & ~size_t(7); };
+    size_t o = 0;
+    t->o_off = (uint32_t)o; o = al8(o + t->off.size() * 8);
+    t->o_cnt = (uint32_t)o; o = al8(o + t->cnt.size() * 8);
+    t->o_lb = (uint32_t)o;  o = al8(o + t->level_base.size() * 8);
+    t->o_lt = (uint32_t)o;  o = al8(o + t->level_total.size() * 8);
+    t->o_cb = (uint32_t)o;  o = al8(o + (size_t)na * 8);
+    t->o_h = (uint32_t)o;   o = al8(o + (size_t)na * 4);
+    t->o_g = (uint32_t)o;   o = al8(o + (size_t)na * 8);
+    const size_t total = o;
+    t->meta_host.assign(total / 8, 0);
+    uint8_t *blob = reinterpret_cast<uint8_t *>(t->meta_host.data());
+    std::memcpy(blob + t->o_off, t->off.data(), t->off.size() * 8);
+    std::memcpy(blob + t->o_cnt, t->cnt.data(), t->cnt.size() * 8);
+    std::memcpy(blob + t->o_lb, t->level_base.data(), t->level_base.size() * 8);
+    std::memcpy(blob + t->o_lt, t->level_total.data(), t->level_total.size() * 8);
+    std::memcpy(blob + t->o_cb, t->chunk_base.data(), (size_t)na * 8);
+    std::memcpy(blob + t->o_h, t->height.data(), (size_t)na * 4);
+    std::memcpy(blob + t->o_g, gbegin.data(), (size_t)na * 8);
     CK_CUDA(cudaMallocAsync((void **)&t->nodes, (t->array_nodes + t->top_nodes) * 16, s));
-    CK_CUDA(cudaMallocAsync((void **)&t->meta, blob.size(), s));
-    CK_TRY(g_ring.copy(t->meta, blob.data(), blob.size(), s));
-    t->d_off = (const uint64_t *)(t->meta + o_off);
-    t->d_cnt = (const uint64_t *)(t->meta + o_cnt);
-    t->d_level_base = (const uint64_t *)(t->meta + o_lb);
-    t->d_level_total = (const uint64_t *)(t->meta + o_lt);
-    t->d_chunk_base = (const uint64_t *)(t->meta + o_cb);
-    t->d_height = (const uint32_t *)(t->meta + o_h);
-    t->d_gbegin = (const uint64_t *)(t->meta + o_g);
-    t->d_ticket = (unsigned *)(t->meta + o_tk);
+    CK_CUDA(cudaMallocAsync((void **)&t->meta, total, s));
+    // the blob reaches `meta` through K2 (inline parameters) or a staging copy there
+    t->d_off = (const uint64_t *)(t->meta + t->o_off);
+    t->d_cnt = (const uint64_t *)(t->meta + t->o_cnt);
+    t->d_level_base = (const uint64_t *)(t->meta + t->o_lb);
+    t->d_level_total = (const uint64_t *)(t->meta + t->o_lt);
+    t->d_chunk_base = (const uint64_t *)(t->meta + t->o_cb);
+    t->d_height = (const uint32_t *)(t->meta + t->o_h);
+    t->d_gbegin = (const uint64_t *)(t->meta + t->o_g);
     return CKPT_OK;
 }
 
 // One leaf-kernel launch over every array of every tree in `table`.
 static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t tasks,
                                  ckpt_dtype dtype, double eps, uint32_t C, cudaStream_t s, int sms) {
-    QuantParams q;
-    quant_params(eps, &q);
+    LeafParams P;
+    std::memset(&P, 0, sizeof(P));
+    quant_params(eps, &P.q);
+    P.n_arrays = (int)table.size();
+    P.n_tasks = tasks;
+    P.chunk = C;
     LeafArray *d_tab = nullptr;
-    const size_t bytes = table.size() * sizeof(LeafArray);
-    CK_CUDA(cudaMallocAsync((void **)&d_tab, bytes, s));
-    CK_TRY(g_ring.copy(d_tab, table.data(), bytes, s));
-    const int na = (int)table.size();
-    if (eps == 0.0) {
-        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(d_tab, na, tasks, C, q, s, sms)));
-        else CK_TRY((launch_leaf_dt<1, true>(d_tab, na, tasks, C, q, s, sms)));
+    if (table.size() <= (size_t)kLeafInline) {
+        for (size_t a = 0; a < table.size(); ++a) P.inl[a] = table[a];
     } else {
-        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(d_tab, na, tasks, C, q, s, sms)));
-        else CK_TRY((launch_leaf_dt<1, false>(d_tab, na, tasks, C, q, s, sms)));
+        const size_t bytes = table.size() * sizeof(LeafArray);
+        CK_CUDA(cudaMallocAsync((void **)&d_tab, bytes, s));
+        CK_TRY(g_ring.copy(d_tab, table.data(), bytes, s));
+        P.arrays = d_tab;
     }
-    CK_CUDA(cudaFreeAsync(d_tab, s));
+    if (eps == 0.0) {
+        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(P, s, sms)));
+        else CK_TRY((launch_leaf_dt<1, true>(P, s, sms)));
+    } else {
+        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(P, s, sms)));
+        else CK_TRY((launch_leaf_dt<1, false>(P, s, sms)));
+    }
+    if (d_tab) CK_CUDA(cudaFreeAsync(d_tab, s));
     return CKPT_OK;
 }
 
@@ -611,14 +650,54 @@ static ckpt_status check_pair(const ckpt_tree *a, const ckpt_tree *b) {
     return CKPT_OK;
 }
 
+// ---------------------------------------------------------------------------
+// per-(device, stream) scratch for the ordered compactions: look-back states
+// tagged with a launch epoch (never cleared) and a self-resetting ticket.
+// ---------------------------------------------------------------------------
+struct Scratch {
+    uint64_t *states = nullptr;
+    size_t cap = 0;
+    unsigned long long *ticket = nullptr;
+    uint32_t epoch = 0;
+};
+static std::mutex g_scr_mu;
+static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
+
+static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_t **states,
+                               unsigned long long **ticket, uint32_t *epoch) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    Scratch &sc = g_scr[std::make_pair(dev, s)];
+    if (!sc.ticket) {
+        CK_CUDA(cudaMallocAsync((void **)&sc.ticket, 256, s));
+        CK_CUDA(cudaMemsetAsync(sc.ticket, 0, 256, s));
+    }
+    n_states = std::max<size_t>(n_states, 1);
+    bool cleared = false;
+    if (sc.cap < n_states) {
+        if (sc.states) CK_CUDA(cudaFreeAsync(sc.states, s));
+        sc.cap = std::max<size_t>(n_states, std::max<size_t>(2 * sc.cap, 4096));
+        CK_CUDA(cudaMallocAsync((void **)&sc.states, sc.cap * 8, s));
+        CK_CUDA(cudaMemsetAsync(sc.states, 0, sc.cap * 8, s));
+        cleared = true;
+    }
+    if (++sc.epoch >= (1u << 24)) {                  // epoch wrap: clear once, restart at 1
+        if (!cleared) CK_CUDA(cudaMemsetAsync(sc.states, 0, sc.cap * 8, s));
+        sc.epoch = 1;
+    }
+    *states = sc.states;
+    *ticket = sc.ticket;
+    *epoch = sc.epoch;
+    return CKPT_OK;
+}
+
 static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, const uint8_t *flags,
                                   uint64_t n, uint64_t *out, uint64_t cap, uint64_t *count,
                                   cudaStream_t s, int sms) {
     const uint64_t n_tiles = (n + kCompactTile - 1) / kCompactTile;
-    uint64_t *scratch = nullptr;
-    CK_CUDA(cudaMallocAsync((void **)&scratch, (n_tiles + 1) * 8, s));
-    CK_CUDA(cudaMemsetAsync(scratch, 0, (n_tiles + 1) * 8, s));
+    int dev = 0;
+    CK_CUDA(cudaGetDevice(&dev));
     CompactParams p;
+    CK_TRY(get_scratch(dev, s, n_tiles, &p.states, &p.ticket, &p.epoch));
     p.leaf_a = la;
     p.leaf_b = lb;
     p.flags = flags;
@@ -626,14 +705,11 @@ static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, co
     p.out = out;
     p.cap = cap;
     p.count = count;
-    p.states = scratch + 1;
-    p.ticket = (unsigned long long *)scratch;
     const unsigned grid = (unsigned)std::min<uint64_t>(n_tiles, (uint64_t)sms * 8);
     ProfScope prof(2, s);
     if (mode == 0) compact_kernel<0><<<grid, kCompactThreads, 0, s>>>(p);
     else compact_kernel<1><<<grid, kCompactThreads, 0, s>>>(p);
     CK_LAUNCH();
-    CK_CUDA(cudaFreeAsync(scratch, s));
     return CKPT_OK;
 }
 
@@ -771,21 +847,23 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     CK_TRY(dev_info(&dev, &di));
     const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c);
     const uint64_t max_tiles = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
-    const size_t o_va = 0;
-    const size_t o_cb = align256(o_va + (size_t)na * sizeof(VerifyArray));
-    const size_t o_tk = align256(o_cb + (size_t)na * 8);
-    const size_t o_st = o_tk + 8;
-    const size_t total = align256(o_st + (max_tiles + 1) * 8);
-    uint8_t *scr = nullptr;
-    CK_CUDA(cudaMallocAsync((void **)&scr, total, s));
-    std::vector<uint8_t> tbl(o_tk, 0);
-    std::memcpy(tbl.data() + o_va, va.data(), (size_t)na * sizeof(VerifyArray));
-    std::memcpy(tbl.data() + o_cb, cb.data(), (size_t)na * 8);
-    CK_TRY(g_ring.copy(scr, tbl.data(), tbl.size(), s));
-    CK_CUDA(cudaMemsetAsync(scr + o_tk, 0, total - o_tk, s));
     VerifyParams p;
-    p.arrays = (const VerifyArray *)(scr + o_va);
-    p.chunk_base = (const uint64_t *)(scr + o_cb);
+    std::memset(&p, 0, sizeof(p));
+    uint8_t *tab = nullptr;
+    if (na <= (uint32_t)kVerifyInline) {
+        // small array tables ride in the kernel parameters: no copy, no allocation
+        for (uint32_t k = 0; k < na; ++k) { p.inl[k] = va[k]; p.inl_base[k] = cb[k]; }
+    } else {
+        const size_t o_cb = align256((size_t)na * sizeof(VerifyArray));
+        std::vector<uint8_t> tbl(o_cb + (size_t)na * 8, 0);
+        std::memcpy(tbl.data(), va.data(), (size_t)na * sizeof(VerifyArray));
+        std::memcpy(tbl.data() + o_cb, cb.data(), (size_t)na * 8);
+        CK_CUDA(cudaMallocAsync((void **)&tab, tbl.size(), s));
+        CK_TRY(g_ring.copy(tab, tbl.data(), tbl.size(), s));
+        p.arrays = (const VerifyArray *)tab;
+        p.chunk_base = (const uint64_t *)(tab + o_cb);
+    }
+    CK_TRY(get_scratch(dev, s, max_tiles, &p.states, &p.ticket, &p.epoch));
     p.n_arrays = (int)na;
     p.chunks = chunks;
     p.n_chunks_dev = n_chunks_dev;
@@ -796,8 +874,6 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     p.out = idx;
     p.cap = cap;
     p.count = n_diff_dev;
-    p.states = (uint64_t *)(scr + o_st);
-    p.ticket = (unsigned long long *)(scr + o_tk);
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * 8));
     {
         ProfScope prof(3, s);
@@ -805,7 +881,7 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
         else verify_kernel<1><<<grid, kVerifyWarps * 32, 0, s>>>(p);
     }
     CK_LAUNCH();
-    CK_CUDA(cudaFreeAsync(scr, s));
+    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
     return CKPT_OK;
 }
 
@@ -1079,5 +1155,23 @@ extern "C" ckpt_status ckpt_profile_read(int k, double *ms, uint64_t *launches) 
     }
     *ms = tot;
     *launches = n;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_profile_timeline(double *out, uint64_t cap, uint64_t *n_records) {
+    if (!n_records || (!out && cap)) return fail(CKPT_EINVAL, "NULL output");
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    *n_records = g_prof.size();
+    if (g_prof.empty()) return CKPT_OK;
+    for (auto &r : g_prof) CK_CUDA(cudaEventSynchronize(r.b));
+    cudaEvent_t base = g_prof[0].a;
+    for (size_t i = 0; i < g_prof.size() && i < cap; ++i) {
+        float s0 = 0.f, s1 = 0.f;
+        CK_CUDA(cudaEventElapsedTime(&s0, base, g_prof[i].a));
+        CK_CUDA(cudaEventElapsedTime(&s1, base, g_prof[i].b));
+        out[3 * i] = g_prof[i].k;
+        out[3 * i + 1] = s0;
+        out[3 * i + 2] = s1;
+    }
     return CKPT_OK;
 }

@@ -14,15 +14,22 @@
 namespace ckpt {
 
 constexpr unsigned kFull = 0xffffffffu;
-constexpr uint64_t kFlagA = 1ull << 62;     // tile aggregate available
-constexpr uint64_t kFlagP = 1ull << 63;     // inclusive prefix available
-constexpr uint64_t kValMask = kFlagA - 1;
+// Look-back state word: epoch (24 bits) | flag (2 bits) | value (38 bits).
+// The epoch is new for every launch that uses a scratch buffer, so states left
+// by earlier launches read as "not ready" and the buffer never needs clearing.
+constexpr int kValBits = 38;
+constexpr uint64_t kValMask = (1ull << kValBits) - 1;
+constexpr uint64_t kFlagA = 1ull << kValBits;        // tile aggregate available
+constexpr uint64_t kFlagP = 2ull << kValBits;        // inclusive prefix available
 
 __device__ __forceinline__ uint64_t ld_volatile(const uint64_t *p) {
     return *reinterpret_cast<const volatile uint64_t *>(p);
 }
 __device__ __forceinline__ void st_volatile(uint64_t *p, uint64_t v) {
     *reinterpret_cast<volatile uint64_t *>(p) = v;
+}
+__device__ __forceinline__ uint64_t state_word(uint32_t epoch, uint64_t flag, uint64_t v) {
+    return ((uint64_t)epoch << 40) | flag | (v & kValMask);
 }
 
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
@@ -42,54 +49,28 @@ __device__ __forceinline__ uint32_t warp_excl_scan_u32(uint32_t v, int lane, uin
     return x - v;
 }
 
-// Called by one full warp.  Returns the exclusive prefix of `tile`.
-__device__ uint64_t tile_lookback(uint64_t *states, uint64_t tile, uint64_t aggregate, int lane) {
-    if (tile == 0) {
-        if (lane == 0) st_volatile(&states[0], kFlagP | aggregate);
-        return 0;
-    }
-    if (lane == 0) st_volatile(&states[tile], kFlagA | aggregate);
-    uint64_t excl = 0;
-    int64_t pred = (int64_t)tile - 1;
-    for (;;) {
-        const int64_t idx = pred - lane;
-        uint64_t s;
-        do {
-            s = idx >= 0 ? ld_volatile(&states[idx]) : kFlagP;
-        } while (__any_sync(kFull, s == 0));
-        const uint32_t pm = __ballot_sync(kFull, (s & kFlagP) != 0);
-        const int stop = pm ? __ffs(pm) - 1 : 31;
-        excl += warp_sum_u64(lane <= stop ? (s & kValMask) : 0);
-        if (pm) break;
-        pred -= 32;
-    }
-    if (lane == 0) st_volatile(&states[tile], kFlagP | (excl + aggregate));
-    return excl;
-}
-
 // CTA-wide decoupled look-back: every thread inspects one predecessor per
-// round, so a round covers blockDim.x predecessors with one L2 round trip
-// (a warp-wide look-back walks 32 at a time, which is a serial chain when all
-// tiles start together).  Called by all threads; `aggregate` must be the
-// same in every thread.  Returns the tile's exclusive prefix.
+// round, so a round covers blockDim.x predecessors with one L2 round trip.
+// Called by all threads; `aggregate` must be the same in every thread.
+// Returns the tile's exclusive prefix.
 template <int NT>
-__device__ uint64_t cta_lookback(uint64_t *states, uint64_t tile, uint64_t aggregate) {
+__device__ uint64_t cta_lookback(uint64_t *states, uint64_t tile, uint64_t aggregate, uint32_t epoch) {
     constexpr int NW = NT / 32;
     __shared__ uint64_t s_sum[NW];
     __shared__ int s_min[NW];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tile == 0) {
-        if (tid == 0) st_volatile(&states[0], kFlagP | aggregate);
+        if (tid == 0) st_volatile(&states[0], state_word(epoch, kFlagP, aggregate));
         return 0;
     }
-    if (tid == 0) st_volatile(&states[tile], kFlagA | aggregate);
+    if (tid == 0) st_volatile(&states[tile], state_word(epoch, kFlagA, aggregate));
     uint64_t excl = 0;
     int64_t hi = (int64_t)tile - 1;
     for (;;) {
         const int64_t idx = hi - tid;
         uint64_t s = kFlagP;                       // before tile 0: inclusive prefix 0
         if (idx >= 0) {
-            do { s = ld_volatile(&states[idx]); } while (s == 0);
+            do { s = ld_volatile(&states[idx]); } while ((uint32_t)(s >> 40) != epoch);
         }
         int mp = (s & kFlagP) ? tid : 0x7fffffff;  // nearest predecessor with a prefix
 #pragma unroll
@@ -110,8 +91,21 @@ __device__ uint64_t cta_lookback(uint64_t *states, uint64_t tile, uint64_t aggre
         if (nearest != 0x7fffffff) break;
         hi -= NT;
     }
-    if (tid == 0) st_volatile(&states[tile], kFlagP | (excl + aggregate));
+    if (tid == 0) st_volatile(&states[tile], state_word(epoch, kFlagP, excl + aggregate));
     return excl;
+}
+
+// Persistent-CTA tile ticket.  Every CTA draws until it gets a tile >= n_tiles;
+// the CTA that draws last resets the counter for the next launch.
+__device__ __forceinline__ uint64_t draw_tile(unsigned long long *ticket, uint64_t n_tiles,
+                                              uint64_t *s_tile) {
+    if (threadIdx.x == 0) {
+        const uint64_t t = atomicAdd(ticket, 1ull);
+        if (t == n_tiles + gridDim.x - 1) *ticket = 0ull;
+        *s_tile = t;
+    }
+    __syncthreads();
+    return *s_tile;
 }
 
 // ---------------------------------------------------------------------------
@@ -131,12 +125,13 @@ struct CompactParams {
     uint64_t *out;
     uint64_t cap;
     uint64_t *count;          // device: total hits
-    uint64_t *states;         // zeroed, >= n_tiles entries
-    unsigned long long *ticket;  // zeroed
+    uint64_t *states;         // >= n_tiles entries (epoch-tagged, never cleared)
+    unsigned long long *ticket;  // 0 on entry, 0 again on exit
+    uint32_t epoch;
 };
 
 template <int MODE>
-__global__ void __launch_bounds__(kCompactThreads) compact_kernel(CompactParams p) {
+__global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_constant__ CompactParams p) {
     __shared__ uint32_t row_cnt[kCompactRows * 8];
     __shared__ uint32_t row_off[kCompactRows * 8];
     __shared__ uint64_t s_excl;
@@ -144,9 +139,7 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(CompactParams 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t n_tiles = (p.n + kCompactTile - 1) / kCompactTile;
     for (;;) {
-        if (threadIdx.x == 0) s_tile = atomicAdd(p.ticket, 1ull);
-        __syncthreads();
-        const uint64_t tile = s_tile;
+        const uint64_t tile = draw_tile(p.ticket, n_tiles, &s_tile);
         if (tile >= n_tiles) return;
         const uint64_t t0 = tile * kCompactTile;
         uint32_t bits[kCompactRows];
@@ -188,7 +181,7 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(CompactParams 
         }
         __syncthreads();
         const uint64_t total = s_excl;
-        const uint64_t excl = cta_lookback<kCompactThreads>(p.states, tile, total);
+        const uint64_t excl = cta_lookback<kCompactThreads>(p.states, tile, total, p.epoch);
         if (threadIdx.x == 0 && tile == n_tiles - 1) *p.count = excl + total;
         const uint32_t lt = (1u << lane) - 1u;
 #pragma unroll
@@ -308,9 +301,13 @@ struct VerifyArray {
     uint64_t elem_base;    // global element id of local element 0
 };
 
+constexpr int kVerifyInline = 16;   // array tables up to this size travel in the kernel params
+
 struct VerifyParams {
-    const VerifyArray *arrays;
+    const VerifyArray *arrays;    // device table (n_arrays > kVerifyInline)
     const uint64_t *chunk_base;   // [a] copy of arrays[a].chunk_base for the search
+    VerifyArray inl[kVerifyInline];
+    uint64_t inl_base[kVerifyInline];
     int n_arrays;
     const uint64_t *chunks;
     const uint64_t *n_chunks_dev; // may be null -> n_chunks_host
@@ -323,6 +320,7 @@ struct VerifyParams {
     uint64_t *count;
     uint64_t *states;
     unsigned long long *ticket;
+    uint32_t epoch;
 };
 
 // 16-byte vector of elements starting at element e (e % VEC == 0); bits of
@@ -364,7 +362,7 @@ __device__ __forceinline__ uint32_t diff_bits(const uint8_t *pa, const uint8_t *
 }
 
 template <int DT>
-__global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams p) {
+__global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(const __grid_constant__ VerifyParams p) {
     constexpr int VEC = DT == 0 ? 4 : 2;
     constexpr int ESZ = DT == 0 ? 4 : 8;
     __shared__ uint32_t w_cnt[kVerifyWarps];
@@ -380,9 +378,7 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams 
     }
     const uint32_t lt = (1u << lane) - 1u;
     for (;;) {
-        if (threadIdx.x == 0) s_tile = atomicAdd(p.ticket, 1ull);
-        __syncthreads();
-        const uint64_t tile = s_tile;
+        const uint64_t tile = draw_tile(p.ticket, n_tiles, &s_tile);
         if (tile >= n_tiles) return;
         const uint64_t q = tile * kVerifyWarps + warp;
         const bool have = q < n_chunks;
@@ -390,8 +386,9 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams 
         uint64_t e_begin = 0, len = 0, gbase = 0;
         if (have) {
             const uint64_t g = p.chunks[q];
-            const int a = find_u64(p.chunk_base, p.n_arrays, g);
-            const VerifyArray A = p.arrays[a];
+            const bool inl = p.n_arrays <= kVerifyInline;
+            const int a = find_u64(inl ? p.inl_base : p.chunk_base, p.n_arrays, g);
+            const VerifyArray A = inl ? p.inl[a] : p.arrays[a];
             const uint64_t c = g - A.chunk_base;
             e_begin = c * p.per;
             const uint64_t e_end = (e_begin + p.per) < A.n ? (e_begin + p.per) : A.n;
@@ -400,12 +397,22 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams 
             pb = A.b + e_begin * ESZ;
             gbase = A.elem_base + e_begin;
         }
-        // pass 1: count
+        // pass 1: count; chunks of up to 64/VEC warp iterations keep their hit bits in
+        // a register so pass 2 does not re-read the data
         uint32_t cnt = 0;
+        uint64_t held = 0;
         constexpr int kStep = 32 * VEC;
+        constexpr int kHeldIters = 64 / VEC;
+        const bool hold = len <= (uint64_t)kHeldIters * kStep;
+        {
+            int it = 0;
 #pragma unroll 4
-        for (uint64_t e = (uint64_t)lane * VEC; e < len; e += kStep)
-            cnt += __popc(diff_bits<DT>(pa, pb, e, len, p.eps));
+            for (uint64_t e = (uint64_t)lane * VEC; e < len; e += kStep, ++it) {
+                const uint32_t m = diff_bits<DT>(pa, pb, e, len, p.eps);
+                cnt += __popc(m);
+                if (it < kHeldIters) held |= (uint64_t)m << (it * VEC);
+            }
+        }
         cnt = (uint32_t)warp_sum_u64(cnt);
         if (lane == 0) w_cnt[warp] = cnt;
         __syncthreads();
@@ -419,14 +426,18 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(VerifyParams 
         }
         __syncthreads();
         const uint64_t tile_total = s_excl;
-        const uint64_t excl = cta_lookback<kVerifyWarps * 32>(p.states, tile, tile_total);
+        const uint64_t excl = cta_lookback<kVerifyWarps * 32>(p.states, tile, tile_total, p.epoch);
         if (threadIdx.x == 0 && tile == n_tiles - 1) *p.count = excl + tile_total;
         // pass 2: emit (only chunks with hits re-read their data)
         if (cnt) {
             uint64_t pos = excl + w_cnt[warp];
-            for (uint64_t e0 = 0; e0 < len; e0 += kStep) {
+            int it = 0;
+            for (uint64_t e0 = 0; e0 < len; e0 += kStep, ++it) {
                 const uint64_t e = e0 + (uint64_t)lane * VEC;
-                const uint32_t m = e < len ? diff_bits<DT>(pa, pb, e, len, p.eps) : 0u;
+                uint32_t m;
+                if (hold) m = (uint32_t)(held >> (it * VEC)) & ((1u << VEC) - 1u);
+                else m = e < len ? diff_bits<DT>(pa, pb, e, len, p.eps) : 0u;
+                if (__ballot_sync(kFull, m != 0) == 0) continue;
                 uint32_t total;
                 const uint32_t ex = warp_excl_scan_u32(__popc(m), lane, total);
                 uint32_t mm = m, k = 0;

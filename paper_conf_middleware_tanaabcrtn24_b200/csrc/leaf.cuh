@@ -153,6 +153,17 @@ __device__ __noinline__ void chain_tail(uint64_t &h1, uint64_t &h2, const uint8_
                    (uint64_t)w[2] | ((uint64_t)w[3] << 32), len);
 }
 
+constexpr int kLeafInline = 16;
+
+struct LeafParams {
+    const LeafArray *arrays;      // device table when n_arrays > kLeafInline
+    LeafArray inl[kLeafInline];
+    int n_arrays;
+    uint64_t n_tasks;
+    uint32_t chunk;
+    QuantParams q;
+};
+
 __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, uint64_t task) {
     int lo = 0, hi = n_arrays - 1;
     while (lo < hi) {
@@ -168,8 +179,13 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
 // scheduler two interleavable instruction streams).
 template <int DT, bool RAW, int CB>
 __global__ void __launch_bounds__(kLeafWarps * 32, CKPT_LEAF_MINB)
-leaf_kernel(const LeafArray *__restrict__ arrays, int n_arrays, uint64_t n_tasks, uint32_t chunk_rt,
-            QuantParams q) {
+leaf_kernel(const __grid_constant__ LeafParams P) {
+    // small array tables travel in the kernel parameters (no H2D copy per build)
+    const LeafArray *arrays = P.n_arrays <= kLeafInline ? P.inl : P.arrays;
+    const int n_arrays = P.n_arrays;
+    const uint64_t n_tasks = P.n_tasks;
+    const uint32_t chunk_rt = P.chunk;
+    QuantParams q = P.q;
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;

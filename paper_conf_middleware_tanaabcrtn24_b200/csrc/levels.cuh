@@ -26,20 +26,30 @@ namespace ckpt {
 constexpr int kLevelThreads = 256;
 constexpr int kLog = 9;
 constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA
-constexpr int kLevelSmemNodes = 6144;        // phase-2 shared memory in nodes (96 KiB)
+constexpr int kLevelSmemNodes = 1536;        // phase-2 shared memory in nodes (24 KiB)
 constexpr int kLevelSmem = kLevelSmemNodes * 16;
 constexpr int kMaxLevelTrees = 4;
 
+constexpr int kLevelInlineWords = 512;       // 4 KiB of tree metadata in the kernel params
+
+// Per-tree launch record.  The metadata tables live in one blob (layout below)
+// that is either inline in the kernel parameters (small trees: no H2D copy;
+// the tree's first CTA then writes it to `meta` for later BFS use) or already
+// in device memory at `meta`.
 struct LevelParams {
     uint4 *nodes;                 // whole tree storage
-    const uint64_t *off;          // [level * n_arrays + a]: node index of array a's level
-    const uint64_t *cnt;          // [level * n_arrays + a]: node count (0 above the array's root)
-    const uint64_t *gbegin;       // [a]: first group of array a (prefix of ceil(cnt[ls][a]/kGroup))
-    const uint64_t *level_base;   // [level]: node index of level (all arrays, concatenated)
-    const uint64_t *level_total;  // [level]: nodes in level (all arrays)
-    const uint32_t *height;       // [a]: number of levels of array a
+    uint8_t *meta;                // device metadata blob
+    int inl;                      // word offset of the blob in LevelBatch::blob, or -1
+    uint32_t meta_words;
+    // byte offsets in the blob:
+    uint32_t o_off;               // u64 [level * n_arrays + a]: node index of array a's level
+    uint32_t o_cnt;               // u64 [level * n_arrays + a]: node count (0 above the root)
+    uint32_t o_lb;                // u64 [level]: node index of level (all arrays)
+    uint32_t o_lt;                // u64 [level]: nodes in level (all arrays)
+    uint32_t o_h;                 // u32 [a]: number of levels of array a
+    uint32_t o_g;                 // u64 [a]: first group of array a
     uint64_t top_off;             // node index of the top tree's level 0
-    unsigned int *ticket;         // zero-initialised counter (reset by the last CTA)
+    unsigned int *ticket;         // zero on entry, reset to zero by the last CTA
     int n_arrays;
     int n_levels;                 // max height over arrays
     int ls;                       // start level of this launch
@@ -50,6 +60,18 @@ struct LevelBatch {
     LevelParams t[kMaxLevelTrees];
     unsigned int cta_begin[kMaxLevelTrees + 1];
     int n;
+    uint64_t blob[kLevelInlineWords];
+};
+
+// Resolved view of one tree's tables.
+struct LvView {
+    uint4 *nodes;
+    const uint64_t *off, *cnt, *gbegin, *level_base, *level_total;
+    const uint32_t *height;
+    uint64_t top_off;
+    unsigned int *ticket;
+    int n_arrays, n_levels, ls;
+    unsigned int n_groups;
 };
 
 __device__ __forceinline__ int find_le(const uint64_t *v, int n, uint64_t x) {
@@ -86,7 +108,7 @@ __device__ __forceinline__ uint4 warp_levels(uint4 v, int m, int k0, int k1, int
 
 // One level over all arrays, children read from `src` (indexable by node
 // index - src_base) and parents written to global and, if dst != null, to dst.
-__device__ __forceinline__ void build_level(const LevelParams &p, int l, const uint4 *src,
+__device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 *src,
                                             uint64_t src_base, uint4 *dst, bool from_global) {
     const int na = p.n_arrays;
     const uint64_t total = p.level_total[l];
@@ -112,8 +134,28 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     int ti = 0;
     while (ti + 1 < pb.n && blockIdx.x >= pb.cta_begin[ti + 1]) ++ti;
-    const LevelParams &p = pb.t[ti];
+    const LevelParams &lp = pb.t[ti];
+    const uint8_t *mb = lp.inl >= 0 ? reinterpret_cast<const uint8_t *>(pb.blob + lp.inl) : lp.meta;
+    LvView p;
+    p.nodes = lp.nodes;
+    p.off = reinterpret_cast<const uint64_t *>(mb + lp.o_off);
+    p.cnt = reinterpret_cast<const uint64_t *>(mb + lp.o_cnt);
+    p.level_base = reinterpret_cast<const uint64_t *>(mb + lp.o_lb);
+    p.level_total = reinterpret_cast<const uint64_t *>(mb + lp.o_lt);
+    p.height = reinterpret_cast<const uint32_t *>(mb + lp.o_h);
+    p.gbegin = reinterpret_cast<const uint64_t *>(mb + lp.o_g);
+    p.top_off = lp.top_off;
+    p.ticket = lp.ticket;
+    p.n_arrays = lp.n_arrays;
+    p.n_levels = lp.n_levels;
+    p.ls = lp.ls;
+    p.n_groups = lp.n_groups;
     const int na = p.n_arrays;
+    if (lp.inl >= 0 && blockIdx.x == pb.cta_begin[ti]) {
+        // publish the inline tables to device memory for later BFS launches
+        uint64_t *dst = reinterpret_cast<uint64_t *>(lp.meta);
+        for (uint32_t w = tid; w < lp.meta_words; w += kLevelThreads) dst[w] = pb.blob[lp.inl + w];
+    }
     // ------------------------------ phase 1 ------------------------------
     {
         const uint64_t gid = blockIdx.x - pb.cta_begin[ti];

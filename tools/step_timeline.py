@@ -1,0 +1,45 @@
+#!/usr/bin/env python
+"""Per-kernel timeline of bench steps (events around every library launch)."""
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_middleware_tanaabcrtn24_b200 as ck  # noqa: E402
+import synth  # noqa: E402
+
+pair = synth.c2_pair(device="cuda")
+A, B = pair.a, pair.b
+L = sum(t.numel() * 4 // 4096 for t in A)
+chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+idx = torch.empty(sum(t.numel() for t in A), dtype=torch.int64, device="cuda")
+counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+
+
+def step():
+    TA, TB = ck.tree_build_batch([A, B], 4096, 1e-6)
+    ck.tree_diff_async(TA, TB, chunks, counts[0:1])
+    ck.verify_async(A, B, chunks, counts[0:1], 4096, 1e-6, idx, counts[1:2])
+    TA.wait()
+    TB.wait()
+    return TA, TB
+
+
+for _ in range(5):
+    keep = step()
+torch.cuda.synchronize()
+ck.profile_reset()
+ck.profile_enable(True)
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record()
+for _ in range(3):
+    keep = step()
+e1.record()
+torch.cuda.synchronize()
+ck.profile_enable(False)
+print(f"3 steps: {e0.elapsed_time(e1):.3f} ms")
+prev_end = 0.0
+for k, s0, s1 in ck.profile_timeline():
+    print(f"{k:7s} start {s0 * 1e3:9.1f} us  end {s1 * 1e3:9.1f} us  dur {(s1 - s0) * 1e3:7.1f} us  gap {(s0 - prev_end) * 1e3:7.1f}")
+    prev_end = max(prev_end, s1)
