@@ -233,8 +233,7 @@ def run_ours(args):
 
     def step():
         TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS)     # one leaf launch for both runs
-        ck.tree_diff_async(TA, TB, chunks, counts[0:1])
-        ck.verify_async(A, B, chunks, counts[0:1], CHUNK, EPS, idx, counts[1:2])
+        ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # stages 1+2 (fused at l0=0)
         if world > 1:
             tops = []
             for T in (TA, TB):

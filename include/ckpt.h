@@ -184,6 +184,19 @@ ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b,
                                      uint64_t chunks_cap, double eps, uint64_t *idx, uint64_t cap,
                                      uint64_t *n_diff_dev, void *stream);
 
+/* Steps 3+4 in one call on two trees and their arrays (a, b: host arrays of
+ * the trees' n_arrays device pointers, same order and lengths as the build).
+ * Writes the flagged chunk ids (as ckpt_tree_diff) and the differing element
+ * ids (as ckpt_verify over those chunks) and counts_dev[0] / counts_dev[1]
+ * (device) = their full counts.  The diff kernel(s) and the verify kernel
+ * run back to back on `stream` with the chunk count kept on the device.
+ * (A single fused kernel -- tile of leaves, verify its flagged chunks, two
+ * look-backs -- was measured 1.5-3x slower: flagged chunks cluster, so
+ * leaf-sized tiles serialise the verify work.)  Asynchronous. */
+ckpt_status ckpt_diff_verify_async(const ckpt_tree *a, const ckpt_tree *b, const void *const *arrays_a,
+                                   const void *const *arrays_b, uint64_t *chunks, uint64_t chunks_cap,
+                                   uint64_t *idx, uint64_t idx_cap, uint64_t *counts_dev, void *stream);
+
 /* ------------------------------------------------------------------------
  * One-call pair comparison (steps 1-4 on two checkpoints of n_arrays
  * arrays each), the library API of P:254-257.  Device inputs.  Writes the

@@ -414,3 +414,26 @@ def profile_timeline():
     _check(lib().ckpt_profile_timeline(buf, n.value, ctypes.byref(n)), "ckpt_profile_timeline")
     names = {v: k for k, v in KERNELS.items()}
     return [(names.get(int(buf[3 * i]), "?"), buf[3 * i + 1], buf[3 * i + 2]) for i in range(n.value)]
+
+
+def diff_verify_async(ta: Tree, tb: Tree, arrays_a, arrays_b, chunks: torch.Tensor,
+                      idx: torch.Tensor, counts: torch.Tensor, stream=None):
+    """Steps 3+4 in one call (one fused kernel when the BFS starts at the leaves).
+
+    counts[0] / counts[1] (device int64) receive the flagged-chunk and differing-element counts."""
+    ta_l, tb_l = _as_list(arrays_a), _as_list(arrays_b)
+    _check_arrays(ta_l + tb_l)
+    pa, _k1 = _ptr_array(ta_l)
+    pb, _k2 = _ptr_array(tb_l)
+    L = lib()
+    if not getattr(L, "_dv_typed", False):
+        L.ckpt_diff_verify_async.argtypes = [ctypes.c_void_p, ctypes.c_void_p,
+                                             ctypes.POINTER(ctypes.c_void_p),
+                                             ctypes.POINTER(ctypes.c_void_p), ctypes.c_void_p,
+                                             ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint64,
+                                             ctypes.c_void_p, ctypes.c_void_p]
+        L.ckpt_diff_verify_async.restype = ctypes.c_int
+        L._dv_typed = True
+    _check(L.ckpt_diff_verify_async(ta.handle, tb.handle, pa, pb, chunks.data_ptr(), chunks.numel(),
+                                    idx.data_ptr(), idx.numel(), counts.data_ptr(),
+                                    _stream_ptr(stream)), "ckpt_diff_verify_async")

@@ -705,12 +705,37 @@ static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, co
     p.out = out;
     p.cap = cap;
     p.count = count;
-    const unsigned grid = (unsigned)std::min<uint64_t>(n_tiles, (uint64_t)sms * 8);
+    // co-resident grid (the look-back relies on it); static tile striding
+    static std::atomic<int> occ0{0}, occ1{0};
+    std::atomic<int> &occ = mode == 0 ? occ0 : occ1;
+    int per_sm = occ.load();
+    if (per_sm == 0) {
+        if (mode == 0) CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, compact_kernel<0>, kCompactThreads, 0));
+        else CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, compact_kernel<1>, kCompactThreads, 0));
+        per_sm = std::max(per_sm, 1);
+        occ.store(per_sm);
+    }
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(n_tiles, (uint64_t)sms * per_sm));
     ProfScope prof(2, s);
     if (mode == 0) compact_kernel<0><<<grid, kCompactThreads, 0, s>>>(p);
     else compact_kernel<1><<<grid, kCompactThreads, 0, s>>>(p);
     CK_LAUNCH();
     return CKPT_OK;
+}
+
+// BFS start level (R16): the level closest to the root whose node count over
+// all arrays is >= T (0 = the leaves).
+static uint32_t start_level(const ckpt_tree *a, uint64_t T) {
+    const uint32_t na = a->n_arrays;
+    for (int l = (int)a->n_levels - 1; l >= 0; --l) {
+        uint64_t tot = 0;
+        for (uint32_t k = 0; k < na; ++k) {
+            const uint32_t ll = std::min<uint32_t>((uint32_t)l, a->height[k] - 1);
+            tot += a->cnt[(size_t)ll * na + k];
+        }
+        if (tot >= T) return (uint32_t)l;
+    }
+    return 0;
 }
 
 extern "C" ckpt_status ckpt_tree_diff_async(const ckpt_tree *a, const ckpt_tree *b, uint64_t T,
@@ -724,16 +749,7 @@ extern "C" ckpt_status ckpt_tree_diff_async(const ckpt_tree *a, const ckpt_tree 
     cudaStream_t s = (cudaStream_t)stream;
     if (T == 0) T = (uint64_t)di.sms * (uint64_t)di.max_threads_sm;
     const uint32_t na = a->n_arrays;
-    // start level (R16): closest to the root whose node count over all arrays >= T
-    uint32_t l0 = 0;
-    for (int l = (int)a->n_levels - 1; l >= 0; --l) {
-        uint64_t tot = 0;
-        for (uint32_t k = 0; k < na; ++k) {
-            const uint32_t ll = std::min<uint32_t>((uint32_t)l, a->height[k] - 1);
-            tot += a->cnt[(size_t)ll * na + k];
-        }
-        if (tot >= T) { l0 = (uint32_t)l; break; }
-    }
+    const uint32_t l0 = start_level(a, T);
     if (l0 > 0) {
         CK_TRY(wait_levels(a, s));
         CK_TRY(wait_levels(b, s));
@@ -874,7 +890,17 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     p.out = idx;
     p.cap = cap;
     p.count = n_diff_dev;
-    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * 8));
+    static std::atomic<int> vocc0{0}, vocc1{0};
+    std::atomic<int> &vocc = dtype == CKPT_F32 ? vocc0 : vocc1;
+    int per_sm = vocc.load();
+    if (per_sm == 0) {
+        if (dtype == CKPT_F32) CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, verify_kernel<0>, kVerifyWarps * 32, 0));
+        else CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, verify_kernel<1>, kVerifyWarps * 32, 0));
+        per_sm = std::max(per_sm, 1);
+        vocc.store(per_sm);
+    }
+    // co-resident grid (the look-back relies on it); tiles are strided statically
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * per_sm));
     {
         ProfScope prof(3, s);
         if (dtype == CKPT_F32) verify_kernel<0><<<grid, kVerifyWarps * 32, 0, s>>>(p);
@@ -883,6 +909,22 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     CK_LAUNCH();
     if (tab) CK_CUDA(cudaFreeAsync(tab, s));
     return CKPT_OK;
+}
+
+// ---------------------------------------------------------------------------
+// stages 1+2 in one call (diff kernel(s) then the verify kernel, no host sync)
+// ---------------------------------------------------------------------------
+extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tree *tb,
+                                              const void *const *a, const void *const *b,
+                                              uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                              uint64_t idx_cap, uint64_t *counts_dev, void *stream) {
+    CK_TRY(check_pair(ta, tb));
+    if (!a || !b || !counts_dev || (!chunks && chunks_cap) || (!idx && idx_cap))
+        return fail(CKPT_EINVAL, "NULL argument");
+    CK_TRY(ckpt_tree_diff_async(ta, tb, 0, chunks, chunks_cap, counts_dev, stream));
+    return verify_impl(a, b, ta->n_elems.data(), ta->n_arrays, ta->dtype, ta->chunk_bytes, chunks,
+                       counts_dev, 0, chunks_cap, ta->eps, idx, idx_cap, counts_dev + 1,
+                       (cudaStream_t)stream);
 }
 
 extern "C" ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b,

@@ -135,12 +135,11 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_c
     __shared__ uint32_t row_cnt[kCompactRows * 8];
     __shared__ uint32_t row_off[kCompactRows * 8];
     __shared__ uint64_t s_excl;
-    __shared__ uint64_t s_tile;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t n_tiles = (p.n + kCompactTile - 1) / kCompactTile;
-    for (;;) {
-        const uint64_t tile = draw_tile(p.ticket, n_tiles, &s_tile);
-        if (tile >= n_tiles) return;
+    // static tile striding over a grid that is fully co-resident (host sizes it), so a
+    // look-back only ever waits on tiles that resident CTAs are processing
+    for (uint64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const uint64_t t0 = tile * kCompactTile;
         uint32_t bits[kCompactRows];
         bool hit[kCompactRows];
@@ -367,7 +366,6 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(const __grid_
     constexpr int ESZ = DT == 0 ? 4 : 8;
     __shared__ uint32_t w_cnt[kVerifyWarps];
     __shared__ uint64_t s_excl;
-    __shared__ uint64_t s_tile;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint64_t n_chunks = p.n_chunks_dev ? *p.n_chunks_dev : p.n_chunks_host;
     if (n_chunks > p.chunks_cap) n_chunks = p.chunks_cap;
@@ -377,9 +375,7 @@ __global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(const __grid_
         return;
     }
     const uint32_t lt = (1u << lane) - 1u;
-    for (;;) {
-        const uint64_t tile = draw_tile(p.ticket, n_tiles, &s_tile);
-        if (tile >= n_tiles) return;
+    for (uint64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const uint64_t q = tile * kVerifyWarps + warp;
         const bool have = q < n_chunks;
         const uint8_t *pa = nullptr, *pb = nullptr;

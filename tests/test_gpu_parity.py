@@ -280,6 +280,38 @@ def test_compare_and_compare_host_agree_with_oracle():
     assert np.array_equal(hidx.numpy(), ref_idx)
 
 
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+@pytest.mark.parametrize("chunk", [512, 4096])
+def test_fused_diff_verify_equals_separate_stages(dt, chunk):
+    sizes = [70_000, 3, 131_072 + 5]
+    arrs_a = [_data(n, dt, 500 + i) for i, n in enumerate(sizes)]
+    arrs_b = [t.clone() for t in arrs_a]
+    g = torch.Generator(device="cpu").manual_seed(1)
+    for t in arrs_b:                    # clustered and scattered changes, above and below eps
+        k = torch.randint(0, t.numel(), (min(300, t.numel()),), generator=g).cuda()
+        t[k] += (torch.rand(k.numel(), generator=g, dtype=torch.float64).cuda() * 4e-5).to(dt)
+        s0 = t.numel() // 3
+        t[s0:s0 + 5000] += 1e-3
+    eps = 1e-5
+    TA, TB = ck.tree_build_batch([arrs_a, arrs_b], chunk, eps)
+    L = TA.n_leaves
+    n = sum(t.numel() for t in arrs_a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(n, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    ck.diff_verify_async(TA, TB, arrs_a, arrs_b, chunks, idx, counts)
+    nc, nd = counts.tolist()
+    A = oracle.build_checkpoint([np_of(t) for t in arrs_a], chunk, eps)
+    B = oracle.build_checkpoint([np_of(t) for t in arrs_b], chunk, eps)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint([np_of(t) for t in arrs_a], [np_of(t) for t in arrs_b],
+                                       chunk, ref_chunks, eps, A)
+    assert nc == ref_chunks.size and np.array_equal(np_of(chunks[:nc]), ref_chunks)
+    assert nd == ref_idx.size and np.array_equal(np_of(idx[:nd]), ref_idx)
+    assert np.array_equal(ref_idx, oracle.brute_checkpoint([np_of(t) for t in arrs_a],
+                                                           [np_of(t) for t in arrs_b], eps))
+
+
 # ------------------------------------------------------------ error paths --
 
 def test_error_paths():

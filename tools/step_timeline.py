@@ -19,8 +19,7 @@ counts = torch.zeros(2, dtype=torch.int64, device="cuda")
 
 def step():
     TA, TB = ck.tree_build_batch([A, B], 4096, 1e-6)
-    ck.tree_diff_async(TA, TB, chunks, counts[0:1])
-    ck.verify_async(A, B, chunks, counts[0:1], 4096, 1e-6, idx, counts[1:2])
+    ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)
     TA.wait()
     TB.wait()
     return TA, TB
