@@ -265,8 +265,10 @@ def run_ours(args):
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     e0.record()
+    h0 = time.perf_counter()
     for _ in range(args.steps):
         step()
+    host_ms = (time.perf_counter() - h0) * 1e3 / args.steps   # enqueue time per step (host)
     e1.record()
     torch.cuda.synchronize()
     launches = ck.launch_count() - l0
@@ -344,7 +346,7 @@ def run_ours(args):
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_launch": leaf_bytes,
                          "avg_launch_ms": round(leaf_avg_s * 1e3, 4)},
-            "phases": phases,
+            "phases": phases, "host_enqueue_ms_per_step": round(host_ms, 4),
             "flagged_chunks_per_gpu": local_counts[0], "diff_elems_per_gpu": local_counts[1],
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
         }

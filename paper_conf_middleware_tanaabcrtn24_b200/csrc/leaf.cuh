@@ -97,7 +97,7 @@ __device__ __forceinline__ void chain_block_exact(U64p &h1, U64p &h2, uint4 v, c
 // branch); a task whose warp saw any out-of-range element is redone exactly.
 template <int DT, bool RAW>
 __device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, const QuantParams &q,
-                                                 bool &ok) {
+                                                 bool &ok, float &mx) {
     uint4 w;
     if (RAW) {
         w = v;
@@ -108,9 +108,14 @@ __device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, co
 #ifdef CKPT_RANGE_F64
         // range test on the FP64 pipe (DSETP) instead of the ALU pipe
         ok = ok & (fabs(d0) < q.r64) & (fabs(d1) < q.r64) & (fabs(d2) < q.r64) & (fabs(d3) < q.r64);
-#else
+#elif defined(CKPT_RANGE_FSETP)
         ok = ok & (fabsf(x0) < q.r32) & (fabsf(x1) < q.r32) & (fabsf(x2) < q.r32) &
              (fabsf(x3) < q.r32);
+#else
+        // running NaN-propagating max of |x| (two 3-input FMNMX3.NAN per block instead of
+        // four FSETP); compared with r32 once per task
+        asm("max.NaN.f32 %0, %1, %2, %3;" : "=f"(mx) : "f"(fabsf(x0)), "f"(fabsf(x1)), "f"(mx));
+        asm("max.NaN.f32 %0, %1, %2, %3;" : "=f"(mx) : "f"(fabsf(x2)), "f"(fabsf(x3)), "f"(mx));
 #endif
         // k mod 2^32 = low word of RD(x*inv + 1.5*2^52)   (hash.cuh)
         w.x = (uint32_t)__double2loint(__fma_rd(d0, q.inv, kMagic));
@@ -230,6 +235,7 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
                                     sp + (uint64_t)i * kChunksPerInstr * C);
             };
             bool ok = true;
+            float mx = 0.0f;
 #pragma unroll
             for (int s = 0; s < kStages - 1; ++s) {
                 if ((uint32_t)s < n_stages) issue(src + s * kSeg, s * kSlotBytes);
@@ -251,12 +257,13 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
 #pragma unroll
                     for (int j = 0; j < kCh; ++j)
                         chain_block_fast<DT, RAW>(h1[j], h2[j], lds128(row + j * 32 * kPitch + b * 16),
-                                                  q, ok);
+                                                  q, ok, mx);
                 }
                 __syncwarp();
                 slot = (slot == (kStages - 1) * kSlotBytes) ? 0u : slot + kSlotBytes;
             }
             cp_async_wait<0>();
+            if (DT == 0 && !RAW) ok = ok & (mx < q.r32);     // NaN (propagated) fails
             done = __all_sync(0xffffffffu, ok);
         }
         if (!done) {

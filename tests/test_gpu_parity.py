@@ -5,6 +5,8 @@ seeded synthetic checkpoints (synth), ragged/partial sizes, special values,
 every BFS start level, truncation and error paths.  Full-size (BASELINE
 configs[1]) checks sample leaves and recompute levels/verify with the oracle.
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -363,3 +365,25 @@ def test_config2_full_size_sampled_parity():
     bn = [np_of(t) for t in pair.b]
     truth = oracle.brute_checkpoint(an, bn, eps)
     assert n == truth.size and np.array_equal(np_of(idx), truth)
+
+
+# ------------------------------------------------ exhaustive f32 quantizer --
+
+@pytest.mark.slow
+@pytest.mark.parametrize("eps", [1e-3, 1e-6, 1e-8, 2.0 ** -10, 0.3])
+def test_quantizer_exhaustive_f32(eps):
+    """Every one of the 2^32 float32 bit patterns (NaNs, infinities, subnormals,
+    both zeros) rounded by the GPU fast/slow paths vs the oracle, per eps: with
+    16-byte chunks each leaf is Murmur3F(4 words, seed 0), so equal leaves mean
+    equal words (barring a 2^-128 collision)."""
+    slice_bits = 28
+    per = 1 << slice_bits
+    for s in range(1 << (32 - slice_bits)):
+        bits = torch.arange(s * per, (s + 1) * per, dtype=torch.int64, device="cuda")
+        x = bits.to(torch.int32).view(torch.float32)
+        t = ck.tree_build(x, 16, eps)
+        got = np_of(t.nodes()[: per // 4])
+        ref = oracle.leaves(np_of(x), 16, eps, threads=os.cpu_count() or 8)
+        bad = np.nonzero(np.any(got != ref, axis=1))[0]
+        assert bad.size == 0, (s, bad[:4], np_of(x).reshape(-1, 4)[bad[:4]])
+        del t, x, bits

@@ -31,14 +31,20 @@ torch.cuda.synchronize()
 ck.profile_reset()
 ck.profile_enable(True)
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+n_steps = int(sys.argv[1]) if len(sys.argv) > 1 else 3
 e0.record()
-for _ in range(3):
+for _ in range(n_steps):
     keep = step()
 e1.record()
 torch.cuda.synchronize()
 ck.profile_enable(False)
-print(f"3 steps: {e0.elapsed_time(e1):.3f} ms")
+print(f"{n_steps} steps: {e0.elapsed_time(e1) / n_steps:.4f} ms/step")
+tl = ck.profile_timeline()
+for kind in ("leaf", "levels", "diff", "verify"):
+    d = [(b - a) * 1e3 for k, a, b in tl if k == kind]
+    if d:
+        print(f"  {kind:7s} mean {sum(d) / len(d):8.1f} us  min {min(d):8.1f}  max {max(d):8.1f}")
 prev_end = 0.0
-for k, s0, s1 in ck.profile_timeline():
+for k, s0, s1 in tl[:8]:
     print(f"{k:7s} start {s0 * 1e3:9.1f} us  end {s1 * 1e3:9.1f} us  dur {(s1 - s0) * 1e3:7.1f} us  gap {(s0 - prev_end) * 1e3:7.1f}")
     prev_end = max(prev_end, s1)
