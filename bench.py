@@ -31,13 +31,36 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "checkpoint-pair compare GB/s (build+diff+verify) at 1/2/4/8 B200, % HBM peak"
-N_PARTICLES = 1 << 26
 CHUNK = 4096
 EPS = 1e-6
 SEED = 2
-WORKLOAD = ("configs[1]: HACC-shaped checkpoint pair, 2^26 particles x 6 float32 per GPU, "
-            "4 KiB chunks, eps=1e-6, 1% particles perturbed in 64 clusters")
 
+# --config: the bench line is configs[1] (c2) by default; c5 (verify-heavy,
+# BASELINE configs[4] per-GPU shard) and c3 (f64) are extra workloads.
+CONFIGS = {
+    "c2": dict(n=1 << 26, workload="configs[1]: HACC-shaped checkpoint pair, 2^26 particles x 6 "
+               "float32 per GPU, 4 KiB chunks, eps=1e-6, 1% particles perturbed in 64 clusters"),
+    "c5": dict(n=50 << 20, workload="configs[4] (one GPU's shard): 8 HACC ranks x 50*2^20 "
+               "particles x 6 float32, 4 KiB chunks, eps=1e-6, 10% chunks with 8 above-eps + 8 "
+               "below-eps changes, 1% chunks below-eps only"),
+    "c3": dict(n=1 << 29, workload="configs[2] (C=4 KiB, eps=1e-6 point): 2^29 float64 ~ N(0,1), "
+               "1024 geometric clusters (mean 4096) with |d|=10^U(-9,-2)"),
+}
+CFG = "c2"
+N_PARTICLES = CONFIGS[CFG]["n"]
+WORKLOAD = CONFIGS[CFG]["workload"]
+
+
+def make_pair(cfg: str, n: int, seed: int, device: str):
+    import synth
+    if cfg == "c2":
+        return synth.c2_pair(n_particles=n, seed=seed, device=device)
+    if cfg == "c5":
+        return synth.c5_pair(n_ranks=8 if n == CONFIGS["c5"]["n"] else 1, n_particles=n,
+                             seed=seed, device=device)
+    if cfg == "c3":
+        return synth.c3_pair(n=n, seed=seed, device=device)
+    raise ValueError(cfg)
 
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
@@ -115,8 +138,7 @@ def host_cores() -> int:
 # ---------------------------------------------------------------------------
 
 def oracle_pair_sample(n_particles: int, seed: int):
-    import synth
-    pair = synth.c2_pair(n_particles=n_particles, seed=seed, device="cpu")
+    pair = make_pair(CFG, n_particles, seed, "cpu")
     return [t.numpy() for t in pair.a], [t.numpy() for t in pair.b]
 
 
@@ -159,7 +181,7 @@ def cpu_baseline(target_s: float = 12.0):
     nbytes = 2 * sum(x.nbytes for x in a)
     return {"value": round(nbytes / dt / 1e9, 4), "unit": "GB/s", "cores": threads,
             "kind": "oracle",
-            "sample": f"same recipe at {n} particles x 6 f32 per run ({nbytes / 1e6:.1f} MB pair), "
+            "sample": f"same recipe ({CFG}) at {n} elements per array ({nbytes / 1e6:.1f} MB pair), "
                       f"one full step (build A+B, BFS diff, verify) in {dt:.2f} s"}
 
 
@@ -191,7 +213,7 @@ def run_reference(args):
                    "chunk_bytes": CHUNK, "eps": EPS, "parallelism": "host threads"},
         "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": threads,
                          "kind": "oracle",
-                         "sample": f"{n} particles x 6 f32 per run ({nbytes / 1e6:.1f} MB pair) per step"},
+                         "sample": f"{CFG} recipe, {n} elements per array ({nbytes / 1e6:.1f} MB pair) per step"},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -219,11 +241,11 @@ def run_ours(args):
     import synth
 
     ck.lib()
-    pair = synth.c2_pair(n_particles=N_PARTICLES, seed=SEED + 1000 * rank, device="cuda")
+    pair = make_pair(CFG, N_PARTICLES, SEED + 1000 * rank, "cuda")
     A, B = pair.a, pair.b
     bytes_pair = 2 * pair.nbytes
     n_elems = sum(t.numel() for t in A)
-    L = sum(t.numel() * 4 // CHUNK for t in A)
+    L = sum(-(-t.numel() * t.element_size() // CHUNK) for t in A)
     chunks = torch.empty(L, dtype=torch.int64, device="cuda")
     idx = torch.empty(n_elems, dtype=torch.int64, device="cuda")
     counts = torch.zeros(2, dtype=torch.int64, device="cuda")
@@ -257,7 +279,7 @@ def run_ours(args):
     sampler.start()
     time.sleep(0.2)
     ck.profile_reset()
-    ck.profile_enable(True)
+    ck.profile_enable(["leaf"])     # leaf events only: the roofline kernel (events elsewhere end PDL overlap)
     l0 = ck.launch_count()
     if world > 1:
         dist.barrier()
@@ -280,11 +302,19 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dist.barrier()
     ms_max = float(t.item())
-    phases = {}
+    leaf_ms, leaf_n = ck.profile_read("leaf")
+    ck.profile_reset()
+    # per-phase device times from a separate profiled pass (events around every family)
+    k_prof = max(3, min(args.steps, 20))
+    ck.profile_enable(True)
+    for _ in range(k_prof):
+        step()
+    torch.cuda.synchronize()
+    ck.profile_enable(False)
+    phases = {"steps": k_prof}
     for k in ("leaf", "levels", "diff", "verify"):
         pms, pn = ck.profile_read(k)
-        phases[k] = {"ms_per_step": round(pms / args.steps, 4), "launches": pn}
-    leaf_ms, leaf_n = ck.profile_read("leaf")
+        phases[k] = {"ms_per_step": round(pms / k_prof, 4), "launches": pn}
     ck.profile_reset()
     leaf_avg_s = leaf_ms / max(1, leaf_n) / 1e3
     leaf_bytes = 2 * (pair.nbytes + 16 * L)  # algorithmic per launch: read A and B, write 2L leaves
@@ -333,11 +363,12 @@ def run_ours(args):
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": round(ms_max, 4),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-            "dtype": "f32 in, f64 quantize/compare, u64 hash",
-            "data": "synthetic (seeded HACC-shaped arrays, synth.c2_pair)",
-            "config": {"workload": WORKLOAD, "particles_per_gpu": N_PARTICLES, "arrays_per_run": 6,
+            "dtype": f"{'f64' if A[0].dtype == torch.float64 else 'f32'} in, f64 quantize/compare, u64 hash",
+            "data": f"synthetic (seeded, synth {CFG} recipe)",
+            "config": {"workload": WORKLOAD, "name": CFG, "elements_per_array": N_PARTICLES,
+                       "arrays_per_run": n_arrays,
                        "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair,
-                       "l2": "inputs larger than L2 (3.2 GB per GPU per step >> 126 MB)",
+                       "l2": f"inputs larger than L2 ({bytes_pair / 1e9:.1f} GB per GPU per step >> 126 MB)",
                        "parallelism": f"dp{world} (checkpoint arrays sharded by rank)"},
             "pct_hbm_peak": round(value / (world * peak), 4),
             "roofline": {"bound": "hbm", "kernel": "leaf_kernel (K1: quantize + chained Murmur3F)",
@@ -346,7 +377,7 @@ def run_ours(args):
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_launch": leaf_bytes,
                          "avg_launch_ms": round(leaf_avg_s * 1e3, 4)},
-            "phases": phases, "host_enqueue_ms_per_step": round(host_ms, 4),
+            "phases_profiled_pass": phases, "host_enqueue_ms_per_step": round(host_ms, 4),
             "flagged_chunks_per_gpu": local_counts[0], "diff_elems_per_gpu": local_counts[1],
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
         }
@@ -364,7 +395,12 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     args = ap.parse_args()
+    global CFG, N_PARTICLES, WORKLOAD
+    CFG = args.config
+    N_PARTICLES = CONFIGS[CFG]["n"]
+    WORKLOAD = CONFIGS[CFG]["workload"]
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

@@ -263,12 +263,14 @@ uint64_t ckpt_default_bfs_threshold(void);
 uint64_t ckpt_launch_count(void);
 
 /* Kernel timing hook for benchmarks (CUDA events on the launching stream).
- * While enabled, every launch of kernel family `k` (0 = leaf hash K1,
- * 1 = tree levels K2, 2 = diff K3, 3 = verify K4) is bracketed by two
- * events.  ckpt_profile_read synchronises those events and returns the
- * summed device time in milliseconds and the launch count of family k
- * since the last reset.  Off by default. */
-void ckpt_profile_enable(int on);
+ * `mask` selects kernel families by bit: bit k enables family k (0 = leaf
+ * hash K1, 1 = tree levels K2, 2 = diff K3, 3 = verify K4); 0 disables all.
+ * Every launch of an enabled family is bracketed by two events (an event
+ * between two kernels also ends their programmatic-launch overlap, so enable
+ * only what is measured).  ckpt_profile_read synchronises those events and
+ * returns the summed device time in milliseconds and the launch count of
+ * family k since the last reset.  Off by default. */
+void ckpt_profile_enable(int mask);
 void ckpt_profile_reset(void);
 ckpt_status ckpt_profile_read(int k, double *ms, uint64_t *launches);
 /* Timeline of the recorded launches since the last reset: for record i,

@@ -390,8 +390,17 @@ def default_bfs_threshold() -> int:
 KERNELS = {"leaf": 0, "levels": 1, "diff": 2, "verify": 3}
 
 
-def profile_enable(on: bool = True):
-    lib().ckpt_profile_enable(1 if on else 0)
+def profile_enable(on=True):
+    """on: True (all kernel families), False, or a list of KERNELS names."""
+    if on is True:
+        mask = 0xF
+    elif not on:
+        mask = 0
+    else:
+        mask = 0
+        for k in on:
+            mask |= 1 << KERNELS[k]
+    lib().ckpt_profile_enable(mask)
 
 
 def profile_reset():

@@ -12,6 +12,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstddef>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <map>
@@ -55,6 +56,32 @@ static ckpt_status fail(ckpt_status s, const std::string &msg) {
             return fail(CKPT_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e_)); \
     } while (0)
 
+// Kernel launch with programmatic stream serialisation (see pdl_enter in
+// hash.cuh); CKPT_PDL=0 in the environment turns the attribute off.
+static bool pdl_on() {
+    static const bool on = [] {
+        const char *e = std::getenv("CKPT_PDL");
+        return !(e && e[0] == '0');
+    }();
+    return on;
+}
+
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                            cudaStream_t s, Args &&...args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl_on() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
 // ---------------------------------------------------------------------------
 // optional per-kernel-family event timing (ckpt_profile_*)
 // ---------------------------------------------------------------------------
@@ -68,7 +95,7 @@ struct ProfScope {
     cudaStream_t s;
     cudaEvent_t a = nullptr, b = nullptr;
     ProfScope(int k_, cudaStream_t s_) : k(k_), s(s_) {
-        if (g_prof_on.load(std::memory_order_relaxed)) {
+        if (g_prof_on.load(std::memory_order_relaxed) & (1 << k_)) {
             cudaEventCreate(&a);
             cudaEventCreate(&b);
             cudaEventRecord(a, s);
@@ -333,7 +360,7 @@ static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
     uint64_t want = (tasks + kLeafWarps - 1) / kLeafWarps;
     uint64_t grid = std::min<uint64_t>(want, (uint64_t)sms * per_sm);
     ProfScope prof(0, s);
-    k<<<(unsigned)grid, kLeafWarps * 32, kLeafSmem, s>>>(P);
+    CK_CUDA(launch_k(k, dim3((unsigned)grid), dim3(kLeafWarps * 32), kLeafSmem, s, P));
     CK_LAUNCH();
     return CKPT_OK;
 }
@@ -412,7 +439,7 @@ static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s)
         }
         b.cta_begin[b.n] = ctas;
         ProfScope prof(1, s);
-        levels_kernel<<<ctas, kLevelThreads, kLevelSmem, s>>>(b);
+        CK_CUDA(launch_k(levels_kernel, dim3(ctas), dim3(kLevelThreads), kLevelSmem, s, b));
         CK_LAUNCH();
     }
     return CKPT_OK;
@@ -659,6 +686,8 @@ struct Scratch {
     size_t cap = 0;
     unsigned long long *ticket = nullptr;
     uint32_t epoch = 0;
+    uint8_t *work = nullptr;       // K4 per-chunk counts + hit bitmasks
+    size_t work_cap = 0;
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -690,6 +719,20 @@ static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_
     return CKPT_OK;
 }
 
+// Stream-ordered work buffer of at least `bytes` (grows, never shrinks).
+static ckpt_status get_work(int dev, cudaStream_t s, size_t bytes, uint8_t **work) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    Scratch &sc = g_scr[std::make_pair(dev, s)];
+    bytes = std::max<size_t>(bytes, 256);
+    if (sc.work_cap < bytes) {
+        if (sc.work) CK_CUDA(cudaFreeAsync(sc.work, s));
+        sc.work_cap = std::max<size_t>(bytes, std::min<size_t>(2 * sc.work_cap, bytes + (64u << 20)));
+        CK_CUDA(cudaMallocAsync((void **)&sc.work, sc.work_cap, s));
+    }
+    *work = sc.work;
+    return CKPT_OK;
+}
+
 static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, const uint8_t *flags,
                                   uint64_t n, uint64_t *out, uint64_t cap, uint64_t *count,
                                   cudaStream_t s, int sms) {
@@ -717,8 +760,7 @@ static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, co
     }
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(n_tiles, (uint64_t)sms * per_sm));
     ProfScope prof(2, s);
-    if (mode == 0) compact_kernel<0><<<grid, kCompactThreads, 0, s>>>(p);
-    else compact_kernel<1><<<grid, kCompactThreads, 0, s>>>(p);
+    CK_CUDA(launch_k(mode == 0 ? compact_kernel<0> : compact_kernel<1>, dim3(grid), dim3(kCompactThreads), 0, s, p));
     CK_LAUNCH();
     return CKPT_OK;
 }
@@ -796,12 +838,16 @@ extern "C" ckpt_status ckpt_tree_diff_async(const ckpt_tree *a, const ckpt_tree 
     unsigned long long *cnts = (unsigned long long *)(scr + o_cnt);
     uint64_t *fr[2] = {(uint64_t *)(scr + o_f0), (uint64_t *)(scr + o_f1)};
     const unsigned grid_first = (unsigned)std::min<uint64_t>((n_start + 255) / 256, (uint64_t)di.sms * 8);
-    { ProfScope prof(2, s); bfs_first_kernel<<<grid_first, 256, 0, s>>>(p, fr[0], cnts); }
+    {
+        ProfScope prof(2, s);
+        CK_CUDA(launch_k(bfs_first_kernel, dim3(grid_first), dim3(256), 0, s, p, fr[0], cnts));
+    }
     CK_LAUNCH();
     for (uint32_t step = 1; step <= l0; ++step) {
         ProfScope prof(2, s);
-        bfs_step_kernel<<<(unsigned)di.sms * 8, 256, 0, s>>>(p, fr[(step - 1) & 1], cnts + step - 1,
-                                                            fr[step & 1], cnts + step);
+        CK_CUDA(launch_k(bfs_step_kernel, dim3((unsigned)di.sms * 8), dim3(256), 0, s, p,
+                         (const uint64_t *)fr[(step - 1) & 1], (const unsigned long long *)(cnts + step - 1),
+                         fr[step & 1], cnts + step));
         CK_LAUNCH();
     }
     CK_TRY(launch_compact(1, nullptr, nullptr, scr + o_flags, L, chunks, cap, n_chunks_dev, s, di.sms));
@@ -862,7 +908,6 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
     const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c);
-    const uint64_t max_tiles = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
     VerifyParams p;
     std::memset(&p, 0, sizeof(p));
     uint8_t *tab = nullptr;
@@ -879,32 +924,57 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
         p.arrays = (const VerifyArray *)tab;
         p.chunk_base = (const uint64_t *)(tab + o_cb);
     }
-    CK_TRY(get_scratch(dev, s, max_tiles, &p.states, &p.ticket, &p.epoch));
     p.n_arrays = (int)na;
     p.chunks = chunks;
     p.n_chunks_dev = n_chunks_dev;
     p.n_chunks_host = n_chunks_host;
     p.chunks_cap = chunks_cap;
     p.per = chunk_bytes / (uint32_t)esz;
+    p.groups = (uint32_t)((p.per + 1023) / 1024);   // 32 words of 32 bits per 1024 elements
     p.eps = eps;
     p.out = idx;
     p.cap = cap;
     p.count = n_diff_dev;
-    static std::atomic<int> vocc0{0}, vocc1{0};
-    std::atomic<int> &vocc = dtype == CKPT_F32 ? vocc0 : vocc1;
-    int per_sm = vocc.load();
-    if (per_sm == 0) {
-        if (dtype == CKPT_F32) CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, verify_kernel<0>, kVerifyWarps * 32, 0));
-        else CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, verify_kernel<1>, kVerifyWarps * 32, 0));
-        per_sm = std::max(per_sm, 1);
-        vocc.store(per_sm);
+    static std::atomic<int> occ[5] = {{0}, {0}, {0}, {0}, {0}};
+    const int d = dtype == CKPT_F32 ? 0 : 1;
+    if (occ[d].load() == 0) {
+        int m = 0, e = 0, sc = 0;
+        if (d == 0) {
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<0>, kVerifyThreads, 0));
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<0>, kVerifyThreads, 0));
+        } else {
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<1>, kVerifyThreads, 0));
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<1>, kVerifyThreads, 0));
+        }
+        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sc, verify_scan_kernel, kVerifyThreads, 0));
+        occ[4].store(std::max(sc, 1));
+        occ[2 + d].store(std::max(e, 1));
+        occ[d].store(std::max(m, 1));
     }
+    const uint64_t warp_ctas = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
+    const unsigned g_mark = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[d].load()));
+    const unsigned g_emit = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[2 + d].load()));
     // co-resident grid (the look-back relies on it); tiles are strided statically
-    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * per_sm));
+    const uint64_t max_tiles = (max_chunks + kVerifyScanTile - 1) / kVerifyScanTile;
+    const unsigned g_scan = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * occ[4].load()));
+    unsigned long long *ticket_unused = nullptr;
+    CK_TRY(get_scratch(dev, s, max_tiles, &p.states, &ticket_unused, &p.epoch));
+    const size_t o_off = align256((size_t)max_chunks * 4);
+    const size_t o_mask = o_off + align256((size_t)max_chunks * 8);
+    uint8_t *work = nullptr;
+    CK_TRY(get_work(dev, s, o_mask + (size_t)max_chunks * p.groups * 128, &work));
+    p.cnt = (uint32_t *)work;
+    p.off = (uint64_t *)(work + o_off);
+    p.mask = (uint32_t *)(work + o_mask);
     {
         ProfScope prof(3, s);
-        if (dtype == CKPT_F32) verify_kernel<0><<<grid, kVerifyWarps * 32, 0, s>>>(p);
-        else verify_kernel<1><<<grid, kVerifyWarps * 32, 0, s>>>(p);
+        CK_CUDA(launch_k(d == 0 ? verify_mark_kernel<0> : verify_mark_kernel<1>, dim3(g_mark),
+                         dim3(kVerifyThreads), 0, s, p));
+        CK_LAUNCH();
+        CK_CUDA(launch_k(verify_scan_kernel, dim3(g_scan), dim3(kVerifyThreads), 0, s, p));
+        CK_LAUNCH();
+        CK_CUDA(launch_k(d == 0 ? verify_emit_kernel<0> : verify_emit_kernel<1>, dim3(g_emit),
+                         dim3(kVerifyThreads), 0, s, p));
     }
     CK_LAUNCH();
     if (tab) CK_CUDA(cudaFreeAsync(tab, s));
@@ -1174,7 +1244,7 @@ extern "C" const char *ckpt_last_error(void) { return g_last_error.c_str(); }
 
 extern "C" uint32_t ckpt_version(void) { return (1u << 16) | 0u; }
 
-extern "C" void ckpt_profile_enable(int on) { g_prof_on.store(on ? 1 : 0); }
+extern "C" void ckpt_profile_enable(int mask) { g_prof_on.store(mask & 0xF); }
 
 extern "C" void ckpt_profile_reset(void) {
     std::lock_guard<std::mutex> lk(g_prof_mu);

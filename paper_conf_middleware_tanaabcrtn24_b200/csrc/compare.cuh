@@ -132,6 +132,7 @@ struct CompactParams {
 
 template <int MODE>
 __global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_constant__ CompactParams p) {
+    pdl_enter();
     __shared__ uint32_t row_cnt[kCompactRows * 8];
     __shared__ uint32_t row_off[kCompactRows * 8];
     __shared__ uint64_t s_excl;
@@ -253,6 +254,7 @@ __device__ __forceinline__ void bfs_visit(const BfsParams &p, bool valid, uint64
 }
 
 __global__ void bfs_first_kernel(BfsParams p, uint64_t *out, unsigned long long *out_cnt) {
+    pdl_enter();
     const int lane = threadIdx.x & 31;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < p.n_start; base += stride) {
@@ -270,6 +272,7 @@ __global__ void bfs_first_kernel(BfsParams p, uint64_t *out, unsigned long long 
 
 __global__ void bfs_step_kernel(BfsParams p, const uint64_t *in, const unsigned long long *in_cnt,
                                 uint64_t *out, unsigned long long *out_cnt) {
+    pdl_enter();
     const int lane = threadIdx.x & 31;
     const uint64_t n = *in_cnt;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -288,9 +291,23 @@ __global__ void bfs_step_kernel(BfsParams p, const uint64_t *in, const unsigned 
 }
 
 // ---------------------------------------------------------------------------
-// K4 verify: one warp per listed chunk, 8 chunks per tile.
+// K4 verify, three kernels:
+//   K4a verify_mark_kernel: warps walk groups of listed chunks (no inter-CTA
+//       synchronisation), stream both runs once, and write each chunk's hit
+//       count and hit bitmask (1 bit per element, element-contiguous 32-bit
+//       words) to scratch.
+//   K4b verify_scan_kernel: ordered exclusive scan of the counts (decoupled
+//       look-back over 4 bytes per chunk) -> output offset per chunk.
+//   K4c verify_emit_kernel: warps walk groups of chunks and write the element
+//       ids of each chunk with hits from its bitmask (ascending, coalesced).
+// The data pass never waits on a look-back chain.
 // ---------------------------------------------------------------------------
 constexpr int kVerifyWarps = 8;
+constexpr int kVerifyThreads = kVerifyWarps * 32;
+#ifndef CKPT_VERIFY_BATCH
+#define CKPT_VERIFY_BATCH 4
+#endif
+constexpr int kVerifyBatch = CKPT_VERIFY_BATCH;   // warp iterations whose loads are issued together
 
 struct VerifyArray {
     const uint8_t *a;
@@ -313,141 +330,299 @@ struct VerifyParams {
     uint64_t n_chunks_host;
     uint64_t chunks_cap;
     uint32_t per;                 // elements per chunk
+    uint32_t groups;              // mask words per lane per chunk
     double eps;
+    uint32_t *cnt;                // [chunks_cap] hits per listed chunk (scratch)
+    uint32_t *mask;               // [chunks_cap][groups][32] hit bits (scratch)
+    uint64_t *off;                // [chunks_cap] output position of each chunk's first hit
     uint64_t *out;
     uint64_t cap;
     uint64_t *count;
-    uint64_t *states;
-    unsigned long long *ticket;
+    uint64_t *states;             // look-back state words (K4b)
     uint32_t epoch;
 };
 
-// 16-byte vector of elements starting at element e (e % VEC == 0); bits of
-// |a-b| > eps for the elements < len.
+__device__ __forceinline__ uint64_t verify_n_chunks(const VerifyParams &p) {
+    const uint64_t n = p.n_chunks_dev ? *p.n_chunks_dev : p.n_chunks_host;
+    return n < p.chunks_cap ? n : p.chunks_cap;
+}
+
+// Locate listed chunk q: data pointers at its first element, its length and
+// the global id of its first element.
+__device__ __forceinline__ void verify_locate(const VerifyParams &p, uint64_t q, int esz,
+                                              const uint8_t *&pa, const uint8_t *&pb,
+                                              uint64_t &len, uint64_t &gbase) {
+    const uint64_t g = p.chunks[q];
+    const bool inl = p.n_arrays <= kVerifyInline;
+    const int a = find_u64(inl ? p.inl_base : p.chunk_base, p.n_arrays, g);
+    const VerifyArray A = inl ? p.inl[a] : p.arrays[a];
+    const uint64_t e_begin = (g - A.chunk_base) * p.per;
+    const uint64_t e_end = (e_begin + p.per) < A.n ? (e_begin + p.per) : A.n;
+    len = e_end > e_begin ? e_end - e_begin : 0;
+    pa = A.a + e_begin * esz;
+    pb = A.b + e_begin * esz;
+    gbase = A.elem_base + e_begin;
+}
+
+// Chunks per warp group: the largest power of two <= 32 that still gives
+// every warp of the grid a group.  The lanes of a warp locate the group's
+// chunks in parallel (one binary search each) and the warp then walks them, so
+// the dependent loads of the search are paid once per group, not per chunk.
+__device__ __forceinline__ uint32_t verify_group(uint64_t n_chunks, uint64_t n_warps) {
+    uint32_t g = 32;
+    while (g > 1 && (uint64_t)g * n_warps > n_chunks) g >>= 1;
+    return g;
+}
+
+struct ChunkLoc {
+    const uint8_t *pa, *pb;
+    uint64_t len, gbase;
+};
+
+__device__ __forceinline__ ChunkLoc shfl_loc(const ChunkLoc &l, int src) {
+    ChunkLoc o;
+    o.pa = (const uint8_t *)__shfl_sync(kFull, (unsigned long long)l.pa, src);
+    o.pb = (const uint8_t *)__shfl_sync(kFull, (unsigned long long)l.pb, src);
+    o.len = __shfl_sync(kFull, l.len, src);
+    o.gbase = __shfl_sync(kFull, l.gbase, src);
+    return o;
+}
+
+// Bits of |a-b| > eps (computed in double, reading R9) for the VEC elements
+// of one 16-byte vector pair.
 template <int DT>
-__device__ __forceinline__ uint32_t diff_bits(const uint8_t *pa, const uint8_t *pb, uint64_t e,
+__device__ __forceinline__ uint32_t diff_vec(uint4 va, uint4 vb, double eps) {
+    uint32_t m = 0;
+    if (DT == 0) {
+        m |= (fabs((double)__uint_as_float(va.x) - (double)__uint_as_float(vb.x)) > eps) ? 1u : 0u;
+        m |= (fabs((double)__uint_as_float(va.y) - (double)__uint_as_float(vb.y)) > eps) ? 2u : 0u;
+        m |= (fabs((double)__uint_as_float(va.z) - (double)__uint_as_float(vb.z)) > eps) ? 4u : 0u;
+        m |= (fabs((double)__uint_as_float(va.w) - (double)__uint_as_float(vb.w)) > eps) ? 8u : 0u;
+    } else {
+        const double a0 = __hiloint2double((int)va.y, (int)va.x), b0 = __hiloint2double((int)vb.y, (int)vb.x);
+        const double a1 = __hiloint2double((int)va.w, (int)va.z), b1 = __hiloint2double((int)vb.w, (int)vb.z);
+        m |= (fabs(a0 - b0) > eps) ? 1u : 0u;
+        m |= (fabs(a1 - b1) > eps) ? 2u : 0u;
+    }
+    return m;
+}
+
+// Scalar tail: elements e.. of a vector that crosses the chunk end.
+template <int DT>
+__device__ __forceinline__ uint32_t diff_tail(const uint8_t *pa, const uint8_t *pb, uint64_t e,
                                               uint64_t len, double eps) {
     constexpr int VEC = DT == 0 ? 4 : 2;
     uint32_t m = 0;
-    if (e + VEC <= len) {
-        const uint4 va = __ldg(reinterpret_cast<const uint4 *>(pa) + e / VEC);
-        const uint4 vb = __ldg(reinterpret_cast<const uint4 *>(pb) + e / VEC);
+    for (int v = 0; v < VEC; ++v) {
+        if (e + v >= len) break;
+        double x, y;
         if (DT == 0) {
-            m |= (fabs((double)__uint_as_float(va.x) - (double)__uint_as_float(vb.x)) > eps) ? 1u : 0u;
-            m |= (fabs((double)__uint_as_float(va.y) - (double)__uint_as_float(vb.y)) > eps) ? 2u : 0u;
-            m |= (fabs((double)__uint_as_float(va.z) - (double)__uint_as_float(vb.z)) > eps) ? 4u : 0u;
-            m |= (fabs((double)__uint_as_float(va.w) - (double)__uint_as_float(vb.w)) > eps) ? 8u : 0u;
+            x = (double)reinterpret_cast<const float *>(pa)[e + v];
+            y = (double)reinterpret_cast<const float *>(pb)[e + v];
         } else {
-            const double a0 = __hiloint2double((int)va.y, (int)va.x), b0 = __hiloint2double((int)vb.y, (int)vb.x);
-            const double a1 = __hiloint2double((int)va.w, (int)va.z), b1 = __hiloint2double((int)vb.w, (int)vb.z);
-            m |= (fabs(a0 - b0) > eps) ? 1u : 0u;
-            m |= (fabs(a1 - b1) > eps) ? 2u : 0u;
+            x = reinterpret_cast<const double *>(pa)[e + v];
+            y = reinterpret_cast<const double *>(pb)[e + v];
         }
-    } else {
-        for (int v = 0; v < VEC; ++v) {
-            if (e + v >= len) break;
-            double x, y;
-            if (DT == 0) {
-                x = (double)reinterpret_cast<const float *>(pa)[e + v];
-                y = (double)reinterpret_cast<const float *>(pb)[e + v];
-            } else {
-                x = reinterpret_cast<const double *>(pa)[e + v];
-                y = reinterpret_cast<const double *>(pb)[e + v];
-            }
-            if (fabs(x - y) > eps) m |= 1u << v;
-        }
+        if (fabs(x - y) > eps) m |= 1u << v;
     }
     return m;
 }
 
 template <int DT>
-__global__ void __launch_bounds__(kVerifyWarps * 32) verify_kernel(const __grid_constant__ VerifyParams p) {
+__global__ void __launch_bounds__(kVerifyThreads) verify_mark_kernel(const __grid_constant__ VerifyParams p) {
+    pdl_enter();
     constexpr int VEC = DT == 0 ? 4 : 2;
     constexpr int ESZ = DT == 0 ? 4 : 8;
-    __shared__ uint32_t w_cnt[kVerifyWarps];
-    __shared__ uint64_t s_excl;
+    constexpr int kStep = 32 * VEC;            // elements per warp iteration
+    constexpr int IPG = 32 / VEC;              // warp iterations per group of 32 mask words
+    constexpr int LPW = 32 / VEC;              // lanes contributing to one mask word
+    const int lane = threadIdx.x & 31;
+    const uint64_t n_chunks = verify_n_chunks(p);
+    const uint64_t n_warps = (uint64_t)gridDim.x * kVerifyWarps;
+    const uint32_t G = verify_group(n_chunks, n_warps);
+    for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + (threadIdx.x >> 5)) * G; q0 < n_chunks;
+         q0 += n_warps * G) {
+      ChunkLoc mine{nullptr, nullptr, 0, 0};
+      if (lane < (int)G && q0 + lane < n_chunks)
+          verify_locate(p, q0 + lane, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+      const uint32_t nq = (n_chunks - q0) < G ? (uint32_t)(n_chunks - q0) : G;
+      for (uint32_t j = 0; j < nq; ++j) {
+        const uint64_t q = q0 + j;
+        const ChunkLoc L = shfl_loc(mine, j);
+        const uint8_t *pa = L.pa, *pb = L.pb;
+        const uint64_t len = L.len;
+        const uint4 *qa = reinterpret_cast<const uint4 *>(pa);
+        const uint4 *qb = reinterpret_cast<const uint4 *>(pb);
+        uint32_t *mq = p.mask + q * p.groups * 32 + lane;
+        uint32_t cnt = 0, word = 0;
+        int it = 0;
+        for (uint64_t base = 0; base < len; base += (uint64_t)kVerifyBatch * kStep) {
+            uint4 va[kVerifyBatch], vb[kVerifyBatch];
+#pragma unroll
+            for (int u = 0; u < kVerifyBatch; ++u) {
+                const uint64_t e = base + (uint64_t)u * kStep + (uint64_t)lane * VEC;
+                if (e + VEC <= len) {
+                    va[u] = __ldcs(qa + e / VEC);
+                    vb[u] = __ldcs(qb + e / VEC);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kVerifyBatch; ++u) {
+                const uint64_t e0 = base + (uint64_t)u * kStep;
+                if (e0 >= len) break;                          // warp-uniform
+                const uint64_t e = e0 + (uint64_t)lane * VEC;
+                uint32_t m = 0;
+                if (e + VEC <= len) m = diff_vec<DT>(va[u], vb[u], p.eps);
+                else if (e < len) m = diff_tail<DT>(pa, pb, e, len, p.eps);
+                cnt += __popc(m);
+                // transpose to element-contiguous words: word k of this iteration
+                // (elements k*32.. of its 32*VEC) is gathered from LPW lanes and
+                // lands in lane (it % IPG) * VEC + k
+                uint32_t x = m << (VEC * (lane % LPW));
+#pragma unroll
+                for (int o = 1; o < LPW; o <<= 1) x |= __shfl_xor_sync(kFull, x, o);
+                const uint32_t y = __shfl_sync(kFull, x, (lane % VEC) * LPW);
+                if (lane / VEC == it % IPG) word = y;
+                if (++it % IPG == 0) { __stcs(mq, word); mq += 32; word = 0; }
+            }
+        }
+        if (it % IPG) __stcs(mq, word);
+        cnt = (uint32_t)warp_sum_u64(cnt);
+        if (lane == 0) p.cnt[q] = cnt;
+      }
+    }
+}
+
+// K4b: exclusive scan of the per-chunk hit counts (kVerifyScanItems chunks per
+// thread, decoupled look-back across tiles) -> p.off[q]; the last tile writes
+// the total to *p.count.
+constexpr int kVerifyScanItems = 4;
+constexpr int kVerifyScanTile = kVerifyThreads * kVerifyScanItems;
+
+__global__ void __launch_bounds__(kVerifyThreads) verify_scan_kernel(const __grid_constant__ VerifyParams p) {
+    pdl_enter();
+    __shared__ uint64_t w_tot[kVerifyWarps];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint64_t n_chunks = p.n_chunks_dev ? *p.n_chunks_dev : p.n_chunks_host;
-    if (n_chunks > p.chunks_cap) n_chunks = p.chunks_cap;
-    const uint64_t n_tiles = (n_chunks + kVerifyWarps - 1) / kVerifyWarps;
+    const uint64_t n_chunks = verify_n_chunks(p);
+    const uint64_t n_tiles = (n_chunks + kVerifyScanTile - 1) / kVerifyScanTile;
     if (n_tiles == 0) {
         if (blockIdx.x == 0 && threadIdx.x == 0) *p.count = 0;
         return;
     }
-    const uint32_t lt = (1u << lane) - 1u;
     for (uint64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-        const uint64_t q = tile * kVerifyWarps + warp;
-        const bool have = q < n_chunks;
-        const uint8_t *pa = nullptr, *pb = nullptr;
-        uint64_t e_begin = 0, len = 0, gbase = 0;
-        if (have) {
-            const uint64_t g = p.chunks[q];
-            const bool inl = p.n_arrays <= kVerifyInline;
-            const int a = find_u64(inl ? p.inl_base : p.chunk_base, p.n_arrays, g);
-            const VerifyArray A = inl ? p.inl[a] : p.arrays[a];
-            const uint64_t c = g - A.chunk_base;
-            e_begin = c * p.per;
-            const uint64_t e_end = (e_begin + p.per) < A.n ? (e_begin + p.per) : A.n;
-            len = e_end > e_begin ? e_end - e_begin : 0;
-            pa = A.a + e_begin * ESZ;
-            pb = A.b + e_begin * ESZ;
-            gbase = A.elem_base + e_begin;
+        const uint64_t q0 = tile * kVerifyScanTile + (uint64_t)threadIdx.x * kVerifyScanItems;
+        uint32_t c[kVerifyScanItems];
+        uint64_t sum = 0;
+#pragma unroll
+        for (int k = 0; k < kVerifyScanItems; ++k) {
+            c[k] = q0 + k < n_chunks ? p.cnt[q0 + k] : 0u;
+            sum += c[k];
         }
-        // pass 1: count; chunks of up to 64/VEC warp iterations keep their hit bits in
-        // a register so pass 2 does not re-read the data
-        uint32_t cnt = 0;
-        uint64_t held = 0;
-        constexpr int kStep = 32 * VEC;
-        constexpr int kHeldIters = 64 / VEC;
-        const bool hold = len <= (uint64_t)kHeldIters * kStep;
-        {
-            int it = 0;
-#pragma unroll 4
-            for (uint64_t e = (uint64_t)lane * VEC; e < len; e += kStep, ++it) {
-                const uint32_t m = diff_bits<DT>(pa, pb, e, len, p.eps);
-                cnt += __popc(m);
-                if (it < kHeldIters) held |= (uint64_t)m << (it * VEC);
-            }
+        uint64_t x = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint64_t y = __shfl_up_sync(kFull, x, o);
+            if (lane >= o) x += y;
         }
-        cnt = (uint32_t)warp_sum_u64(cnt);
-        if (lane == 0) w_cnt[warp] = cnt;
+        if (lane == 31) w_tot[warp] = x;
         __syncthreads();
-        if (warp == 0) {
-            const uint32_t v = lane < kVerifyWarps ? w_cnt[lane] : 0u;
-            uint32_t total;
-            const uint32_t ex = warp_excl_scan_u32(v, lane, total);
-            __syncwarp();
-            if (lane < kVerifyWarps) w_cnt[lane] = ex;
-            if (lane == 0) s_excl = total;
+        uint64_t before = 0, total = 0;
+#pragma unroll
+        for (int w = 0; w < kVerifyWarps; ++w) {
+            const uint64_t v = w_tot[w];
+            if (w < warp) before += v;
+            total += v;
+        }
+        const uint64_t excl = cta_lookback<kVerifyThreads>(p.states, tile, total, p.epoch);
+        if (threadIdx.x == 0 && tile == n_tiles - 1) *p.count = excl + total;
+        uint64_t pos = excl + before + x - sum;
+#pragma unroll
+        for (int k = 0; k < kVerifyScanItems; ++k) {
+            if (q0 + k < n_chunks) p.off[q0 + k] = pos;
+            pos += c[k];
         }
         __syncthreads();
-        const uint64_t tile_total = s_excl;
-        const uint64_t excl = cta_lookback<kVerifyWarps * 32>(p.states, tile, tile_total, p.epoch);
-        if (threadIdx.x == 0 && tile == n_tiles - 1) *p.count = excl + tile_total;
-        // pass 2: emit (only chunks with hits re-read their data)
-        if (cnt) {
-            uint64_t pos = excl + w_cnt[warp];
-            int it = 0;
-            for (uint64_t e0 = 0; e0 < len; e0 += kStep, ++it) {
-                const uint64_t e = e0 + (uint64_t)lane * VEC;
-                uint32_t m;
-                if (hold) m = (uint32_t)(held >> (it * VEC)) & ((1u << VEC) - 1u);
-                else m = e < len ? diff_bits<DT>(pa, pb, e, len, p.eps) : 0u;
-                if (__ballot_sync(kFull, m != 0) == 0) continue;
-                uint32_t total;
-                const uint32_t ex = warp_excl_scan_u32(__popc(m), lane, total);
-                uint32_t mm = m, k = 0;
-                while (mm) {
-                    const int bit = __ffs(mm) - 1;
-                    mm &= mm - 1;
-                    const uint64_t o = pos + ex + k++;
-                    if (o < p.cap) p.out[o] = gbase + e + bit;
-                }
-                pos += total;
-            }
-        }
-        (void)lt;
-        __syncthreads();
+    }
+}
+
+// Write the hits of one group of 32 mask words (1024 elements from e_base,
+// word l in lane l) to out[pos..).  The hit offsets are first compacted into
+// the warp's shared-memory slot (lane l after the hits of lanes < l), then
+// written out with each store instruction covering 32 consecutive output slots.
+// Returns the count.
+__device__ __forceinline__ uint32_t emit_words(uint32_t word, uint64_t e_base, uint64_t pos,
+                                               uint64_t *out, uint64_t cap, int lane,
+                                               uint16_t *s_off) {
+    if (__ballot_sync(kFull, word != 0) == 0) return 0;
+    uint32_t tot;
+    uint32_t o = warp_excl_scan_u32(__popc(word), lane, tot);
+    for (uint32_t mm = word; mm; mm &= mm - 1, ++o) s_off[o] = (uint16_t)(lane * 32 + __ffs(mm) - 1);
+    __syncwarp();
+    for (uint32_t k = lane; k < tot; k += 32)
+        if (pos + k < cap) out[pos + k] = e_base + s_off[k];
+    __syncwarp();
+    return tot;
+}
+
+// K4c: warps walk groups of listed chunks; the lanes load the group's counts,
+// offsets and locations in parallel.  Sparse chunks (<= kEmitSparse hits) are
+// emitted one per lane (the lane reads the chunk's mask words with 16-byte
+// loads and writes its ids in order); dense chunks are emitted by the whole
+// warp, one 32-word group at a time, with coalesced stores.
+constexpr uint32_t kEmitSparse = 48;
+
+template <int DT>
+__global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __grid_constant__ VerifyParams p) {
+    pdl_enter();
+    constexpr int ESZ = DT == 0 ? 4 : 8;
+    __shared__ uint16_t s_off_all[kVerifyWarps][1024];
+    const int lane = threadIdx.x & 31;
+    uint16_t *s_off = s_off_all[threadIdx.x >> 5];
+    const uint64_t n_chunks = verify_n_chunks(p);
+    const uint64_t n_warps = (uint64_t)gridDim.x * kVerifyWarps;
+    const uint32_t G = verify_group(n_chunks, n_warps);
+    const uint32_t n_words = p.groups * 32;
+    for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + (threadIdx.x >> 5)) * G; q0 < n_chunks;
+         q0 += n_warps * G) {
+      uint64_t my_off = 0, my_gb = 0;
+      uint32_t c = 0;
+      if (lane < (int)G && q0 + lane < n_chunks) {
+          c = p.cnt[q0 + lane];
+          if (c) {
+              const uint8_t *pa, *pb;
+              uint64_t len;
+              my_off = p.off[q0 + lane];
+              verify_locate(p, q0 + lane, ESZ, pa, pb, len, my_gb);
+          }
+      }
+      // sparse chunks: one lane each
+      if (c && c <= kEmitSparse) {
+          const uint4 *mw = reinterpret_cast<const uint4 *>(p.mask + (q0 + lane) * n_words);
+          uint64_t o = my_off;
+#pragma unroll 1
+          for (uint32_t w4 = 0; w4 < n_words / 4; ++w4) {
+              const uint4 v = __ldcs(mw + w4);
+              const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                  const uint64_t e = my_gb + (uint64_t)(w4 * 4 + k) * 32;
+                  for (uint32_t mm = wv[k]; mm; mm &= mm - 1, ++o)
+                      if (o < p.cap) p.out[o] = e + (__ffs(mm) - 1);
+              }
+          }
+      }
+      // dense chunks: the whole warp
+#pragma unroll 1
+      for (uint32_t todo = __ballot_sync(kFull, c > kEmitSparse); todo; todo &= todo - 1) {
+        const int j = __ffs(todo) - 1;
+        const uint64_t gbase = __shfl_sync(kFull, my_gb, j);
+        uint64_t pos = __shfl_sync(kFull, my_off, j);
+        const uint32_t *mq = p.mask + (q0 + j) * n_words + lane;
+#pragma unroll 1
+        for (uint32_t g = 0; g < p.groups; ++g)
+            pos += emit_words(__ldcs(mq + g * 32), gbase + (uint64_t)g * 1024, pos, p.out, p.cap, lane,
+                              s_off);
+      }
     }
 }
 

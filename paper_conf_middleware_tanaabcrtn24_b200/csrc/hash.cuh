@@ -21,6 +21,17 @@
 
 namespace ckpt {
 
+// Programmatic dependent launch: every kernel of the library is launched with
+// programmatic stream serialisation, waits for its stream predecessor to
+// complete (griddepcontrol.wait: full completion and memory visibility) before
+// touching memory, and lets its own successor be scheduled right away, so the
+// successor's launch and CTA rasterisation overlap this kernel's tail.  Both
+// instructions are no-ops for a kernel launched without the attribute.
+__device__ __forceinline__ void pdl_enter() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 constexpr uint64_t kC1 = 0x87c37b91114253d5ull;
 constexpr uint64_t kC2 = 0x4cf5ad432745937full;
 constexpr uint64_t kF1 = 0xff51afd7ed558ccdull;

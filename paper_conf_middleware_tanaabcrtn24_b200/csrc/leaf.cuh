@@ -185,6 +185,7 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
 template <int DT, bool RAW, int CB>
 __global__ void __launch_bounds__(kLeafWarps * 32, CKPT_LEAF_MINB)
 leaf_kernel(const __grid_constant__ LeafParams P) {
+    pdl_enter();
     // small array tables travel in the kernel parameters (no H2D copy per build)
     const LeafArray *arrays = P.n_arrays <= kLeafInline ? P.inl : P.arrays;
     const int n_arrays = P.n_arrays;

@@ -128,6 +128,7 @@ __device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 
 }
 
 __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_constant__ LevelBatch pb) {
+    pdl_enter();
     extern __shared__ __align__(16) uint4 sm[];
     __shared__ uint4 s_root[kLevelThreads / 32];
     __shared__ unsigned int s_ticket;

@@ -21,7 +21,10 @@ Recipes (DESIGN.md "Input recipe"):
       d = +-10^U(-8,-3) on all six fields.
   c3  2^29 f64 ~ N(0,1); 1024 clusters, geometric length (mean 4096),
       d = +-10^U(-9,-2).
-  c4/c5 per-rank c2-shaped arrays.
+  c4  per-rank c2-shaped arrays (rank_pair).
+  c5  8 ranks x 50*2^20 particles x 6 f32 per GPU; 10% of chunks get 8 above-eps
+      and 8 below-eps (bin-straddling) perturbations, another 1% only the
+      below-eps ones (verify-heavy, false positives by construction).
 """
 from __future__ import annotations
 
@@ -198,3 +201,57 @@ def rank_pair(rank: int, n_particles: int, seed_base: int, device="cpu", eps: fl
     a = hacc_arrays(n_particles, seed_base + rank, device)
     b, clusters = cluster_mask_perturb(a, frac, n_clusters, seed_base + 5000 + rank)
     return Pair(f"rank{rank}", a, b, chunk_bytes, eps, {"clusters": clusters})
+
+
+def c5_pair(n_ranks: int = 8, n_particles: int = 50 << 20, seed: int = 50, device="cpu",
+            eps: float = 1e-6, chunk_bytes: int = 4096, frac_true: float = 0.10,
+            frac_fp: float = 0.01, per_chunk: int = 8) -> Pair:
+    """Config 5 (per GPU): n_ranks HACC ranks x 6 f32 arrays per run.
+
+    In frac_true of the chunks of every array, `per_chunk` elements get
+    |d| ~ U[2,20]*eps (above) and `per_chunk` more straddle a multiple of eps
+    at a small magnitude (below, forced false positive); in another frac_fp of
+    the chunks only the straddlers are planted.  Straddling changes run A too
+    (a = m*eps - off, b = m*eps + off with off < eps/2)."""
+    a_list, b_list = [], []
+    rng = np.random.default_rng(seed)
+    per = chunk_bytes // 4
+    for r in range(n_ranks):
+        arrs = hacc_arrays(n_particles, seed * 100 + r, device)
+        outs = [t.clone() for t in arrs]
+        for f, (ta, tb) in enumerate(zip(arrs, outs)):
+            n = ta.numel()
+            L = n // per
+            n_true = int(round(frac_true * L))
+            n_fp = int(round(frac_fp * L))
+            ch = rng.choice(L, size=n_true + n_fp, replace=False)
+            ch_true, ch_fp = ch[:n_true], ch[n_true:]
+            # above-eps: per_chunk random elements of each true chunk
+            if n_true:
+                off = rng.integers(0, per, size=(n_true, per_chunk))
+                idx = (ch_true[:, None] * per + off).reshape(-1)
+                idx = np.unique(idx)
+                sgn = np.where(rng.random(idx.size) < 0.5, -1.0, 1.0)
+                mag = rng.uniform(2.0, 20.0, idx.size) * eps * sgn
+                it = torch.as_tensor(idx, dtype=torch.int64, device=device)
+                x = tb[it].to(torch.float64)
+                md = torch.as_tensor(mag, device=device)
+                # at least ~2 ulps of x so the change survives rounding to f32
+                md = torch.sign(md) * torch.maximum(md.abs(), x.abs() * 2.0 ** -22)
+                tb[it] = (x + md).to(tb.dtype)
+            # below-eps bin straddlers in true and fp chunks
+            chs = np.concatenate([ch_true, ch_fp])
+            if chs.size:
+                off = rng.integers(0, per, size=(chs.size, per_chunk))
+                idx = np.unique((chs[:, None] * per + off).reshape(-1))
+                m = rng.integers(-500, 500, idx.size).astype(np.float64)
+                d = rng.uniform(0.02, 0.2, idx.size) * eps
+                va = torch.as_tensor(m * eps - d, dtype=torch.float32, device=device)
+                vb = torch.as_tensor(m * eps + d, dtype=torch.float32, device=device)
+                it = torch.as_tensor(idx, dtype=torch.int64, device=device)
+                ta[it] = va
+                tb[it] = vb
+        a_list += arrs
+        b_list += outs
+    return Pair("c5", a_list, b_list, chunk_bytes, eps,
+                {"n_ranks": n_ranks, "n_particles": n_particles})

@@ -387,3 +387,30 @@ def test_quantizer_exhaustive_f32(eps):
         bad = np.nonzero(np.any(got != ref, axis=1))[0]
         assert bad.size == 0, (s, bad[:4], np_of(x).reshape(-1, 4)[bad[:4]])
         del t, x, bits
+
+
+def test_config5_shape_verify_heavy_bfs_path():
+    """configs[4] shape at reduced size: many arrays, 10% of chunks with true differences and
+    planted false positives; T small enough that the BFS starts above the leaves."""
+    pair = synth.c5_pair(n_ranks=2, n_particles=1 << 16, seed=7, device="cuda")
+    C, eps = pair.chunk_bytes, pair.eps
+    TA, TB = ck.tree_build_batch([pair.a, pair.b], C, eps)
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    A = oracle.build_checkpoint(an, C, eps)
+    B = oracle.build_checkpoint(bn, C, eps)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, C, ref_chunks, eps, A)
+    assert np.array_equal(ref_idx, oracle.brute_checkpoint(an, bn, eps))
+    for T in (0, 7, 1000):                  # default (leaf start) and mid-level starts
+        chunks = torch.empty(TA.n_leaves, dtype=torch.int64, device="cuda")
+        cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+        ck.tree_diff_async(TA, TB, chunks, cnt[0:1], T=T)
+        idx = torch.empty(sum(t.numel() for t in pair.a), dtype=torch.int64, device="cuda")
+        ck.verify_async(pair.a, pair.b, chunks, cnt[0:1], C, eps, idx, cnt[1:2])
+        nc, nd = cnt.tolist()
+        assert np.array_equal(np_of(chunks[:nc]), ref_chunks), T
+        assert np.array_equal(np_of(idx[:nd]), ref_idx), T
+    # false positives exist (flagged chunks without a verified difference)
+    per = C // 4
+    assert np.setdiff1d(ref_chunks, np.unique(ref_idx // per)).size > 0
