@@ -254,8 +254,12 @@ def run_ours(args):
     keep = []
 
     def step():
-        TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS)     # one leaf launch for both runs
-        ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # stages 1+2 (fused at l0=0)
+        if args.path == "fused":
+            # one leaf launch hashes both runs, compares the digests and marks the flagged chunks
+            TA, TB = ck.compare_pair_async(A, B, CHUNK, EPS, chunks, idx, counts)
+        else:
+            TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS)     # one leaf launch for both runs
+            ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # BFS diff, then verify
         if world > 1:
             tops = []
             for T in (TA, TB):
@@ -369,7 +373,8 @@ def run_ours(args):
                        "arrays_per_run": n_arrays,
                        "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair,
                        "l2": f"inputs larger than L2 ({bytes_pair / 1e9:.1f} GB per GPU per step >> 126 MB)",
-                       "parallelism": f"dp{world} (checkpoint arrays sharded by rank)"},
+                       "parallelism": f"dp{world} (checkpoint arrays sharded by rank)",
+                       "path": args.path},
             "pct_hbm_peak": round(value / (world * peak), 4),
             "roofline": {"bound": "hbm", "kernel": "leaf_kernel (K1: quantize + chained Murmur3F)",
                          "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
@@ -396,6 +401,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--path", default="fused", choices=["fused", "unfused"],
+                    help="fused: ckpt_compare_pair_async; unfused: build_batch + diff_verify_async")
     args = ap.parse_args()
     global CFG, N_PARTICLES, WORKLOAD
     CFG = args.config

@@ -197,6 +197,35 @@ ckpt_status ckpt_diff_verify_async(const ckpt_tree *a, const ckpt_tree *b, const
                                    const void *const *arrays_b, uint64_t *chunks, uint64_t chunks_cap,
                                    uint64_t *idx, uint64_t idx_cap, uint64_t *counts_dev, void *stream);
 
+/* ----------------------------------------------------------------------
+ * Fused pair compare: steps 1-4 for two checkpoints of identical shape in
+ * one call -- the device-resident form of the paper's online comparison
+ * (SURVEY 8(f) rank 1).  One leaf-kernel launch hashes A and B
+ * (Alg. 1); whichever warp finishes the second half of a 32-chunk
+ * pair-task compares the two runs' leaf digests in-kernel and writes a flag
+ * byte per chunk -- the BFS of P:555-566 at start level 0 (a chunk is flagged
+ * iff its leaves differ), with no pass over the leaves afterwards.  The
+ * flags are compacted into the ascending chunk list and the verify kernels
+ * write the ascending element ids.  Both trees are built in full
+ * (interior levels on a side stream, as ckpt_tree_build_batch) and returned
+ * in *out_a / *out_b (owned by the caller, free with ckpt_tree_free).
+ *   a, b        (host) arrays of n_arrays device pointers, 16-byte aligned
+ *   n           (host) element counts, shared by A and B
+ *   chunks      device, chunks_cap entries: flagged chunk ids, ascending
+ *   idx         device, idx_cap entries: differing element ids (global
+ *               numbering over the arrays in order), ascending
+ *   counts_dev  device uint64[2]: full chunk count; element count over the
+ *               listed (first chunks_cap) chunks
+ * Results equal ckpt_tree_build_batch + ckpt_tree_diff + ckpt_verify (the
+ * BFS finds the same chunks from any start level).  Scratch: one byte per
+ * chunk plus the verify work buffer.  Errors: EINVAL, ENOMEM, ECUDA.
+ * Asynchronous (no host synchronisation). */
+ckpt_status ckpt_compare_pair_async(const void *const *a, const void *const *b, const uint64_t *n,
+                                    uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                    double eps, uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                    uint64_t idx_cap, uint64_t *counts_dev, void *stream,
+                                    ckpt_tree **out_a, ckpt_tree **out_b);
+
 /* ------------------------------------------------------------------------
  * One-call pair comparison (steps 1-4 on two checkpoints of n_arrays
  * arrays each), the library API of P:254-257.  Device inputs.  Writes the

@@ -446,3 +446,36 @@ def diff_verify_async(ta: Tree, tb: Tree, arrays_a, arrays_b, chunks: torch.Tens
     _check(L.ckpt_diff_verify_async(ta.handle, tb.handle, pa, pb, chunks.data_ptr(), chunks.numel(),
                                     idx.data_ptr(), idx.numel(), counts.data_ptr(),
                                     _stream_ptr(stream)), "ckpt_diff_verify_async")
+
+
+def compare_pair_async(arrays_a, arrays_b, chunk_bytes: int, eps: float, chunks: torch.Tensor,
+                       idx: torch.Tensor, counts: torch.Tensor, stream=None) -> Tuple[Tree, Tree]:
+    """Fused pair compare (ckpt_compare_pair_async): steps 1-4 for two checkpoints of identical
+    shape with the leaf-digest comparison and the element marking inside the leaf kernel.
+
+    Writes the flagged chunk ids to ``chunks``, the differing element ids to ``idx`` and the two
+    full counts to ``counts[0:2]`` (device int64); returns both trees."""
+    la, lb = _as_list(arrays_a), _as_list(arrays_b)
+    if len(la) != len(lb) or any(x.numel() != y.numel() for x, y in zip(la, lb)):
+        raise ValueError("A and B must have the same arrays and lengths")
+    code = _check_arrays(la + lb)
+    pa, _k1 = _ptr_array(la)
+    pb, _k2 = _ptr_array(lb)
+    pn, _k3 = _u64_array([t.numel() for t in la])
+    L = lib()
+    if not getattr(L, "_cp_typed", False):
+        vp, u64 = ctypes.c_void_p, ctypes.c_uint64
+        L.ckpt_compare_pair_async.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                              ctypes.POINTER(u64), ctypes.c_uint32, ctypes.c_int,
+                                              ctypes.c_uint32, ctypes.c_double, vp, u64, vp, u64,
+                                              vp, vp, ctypes.POINTER(vp), ctypes.POINTER(vp)]
+        L.ckpt_compare_pair_async.restype = ctypes.c_int
+        L._cp_typed = True
+    ta, tb = ctypes.c_void_p(), ctypes.c_void_p()
+    sp = _stream_ptr(stream)
+    _check(L.ckpt_compare_pair_async(pa, pb, pn, len(la), code, chunk_bytes, float(eps),
+                                     chunks.data_ptr(), chunks.numel(), idx.data_ptr(), idx.numel(),
+                                     counts.data_ptr(), sp, ctypes.byref(ta), ctypes.byref(tb)),
+           "ckpt_compare_pair_async")
+    return (Tree(ta.value, la, code, chunk_bytes, float(eps), sp),
+            Tree(tb.value, lb, code, chunk_bytes, float(eps), sp))

@@ -343,10 +343,10 @@ static ckpt_status check_common(ckpt_dtype dtype, uint32_t chunk_bytes, double e
     return CKPT_OK;
 }
 
-template <int DT, bool RAW, int CB>
+template <int DT, bool RAW, int CB, bool PAIR>
 static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
     const uint64_t tasks = P.n_tasks;
-    auto k = leaf_kernel<DT, RAW, CB>;
+    auto k = leaf_kernel<DT, RAW, CB, PAIR>;
     static std::atomic<int> cached_per_sm{0};
     int per_sm = cached_per_sm.load(std::memory_order_relaxed);
     if (per_sm == 0) {
@@ -366,22 +366,28 @@ static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
 }
 
 template <int DT, bool RAW>
-static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms) {
+static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms, bool pair) {
     const uint32_t C = P.chunk;
+    if (pair) {   // fused pair mode: the bench chunk size specialised, others generic
+        if constexpr (!RAW) {
+            if (C == 4096) return launch_leaf_t<DT, RAW, 4096, true>(P, s, sms);
+        }
+        return launch_leaf_t<DT, RAW, 0, true>(P, s, sms);
+    }
     if (!RAW) {
         switch (C) {
-            case 512: return launch_leaf_t<DT, RAW, 512>(P, s, sms);
-            case 1024: return launch_leaf_t<DT, RAW, 1024>(P, s, sms);
-            case 2048: return launch_leaf_t<DT, RAW, 2048>(P, s, sms);
-            case 4096: return launch_leaf_t<DT, RAW, 4096>(P, s, sms);
-            case 8192: return launch_leaf_t<DT, RAW, 8192>(P, s, sms);
-            case 16384: return launch_leaf_t<DT, RAW, 16384>(P, s, sms);
-            case 32768: return launch_leaf_t<DT, RAW, 32768>(P, s, sms);
-            case 65536: return launch_leaf_t<DT, RAW, 65536>(P, s, sms);
+            case 512: return launch_leaf_t<DT, RAW, 512, false>(P, s, sms);
+            case 1024: return launch_leaf_t<DT, RAW, 1024, false>(P, s, sms);
+            case 2048: return launch_leaf_t<DT, RAW, 2048, false>(P, s, sms);
+            case 4096: return launch_leaf_t<DT, RAW, 4096, false>(P, s, sms);
+            case 8192: return launch_leaf_t<DT, RAW, 8192, false>(P, s, sms);
+            case 16384: return launch_leaf_t<DT, RAW, 16384, false>(P, s, sms);
+            case 32768: return launch_leaf_t<DT, RAW, 32768, false>(P, s, sms);
+            case 65536: return launch_leaf_t<DT, RAW, 65536, false>(P, s, sms);
             default: break;
         }
     }
-    return launch_leaf_t<DT, RAW, 0>(P, s, sms);
+    return launch_leaf_t<DT, RAW, 0, false>(P, s, sms);
 }
 
 // K2 for up to kMaxLevelTrees trees in one launch.
@@ -490,10 +496,14 @@ static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
 
 // One leaf-kernel launch over every array of every tree in `table`.
 static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t tasks,
-                                 ckpt_dtype dtype, double eps, uint32_t C, cudaStream_t s, int sms) {
+                                 ckpt_dtype dtype, double eps, uint32_t C, cudaStream_t s, int sms,
+                                 const PairParams *pair = nullptr,
+                                 unsigned long long *ticket = nullptr) {
     LeafParams P;
     std::memset(&P, 0, sizeof(P));
     quant_params(eps, &P.q);
+    if (pair) P.pr = *pair;
+    P.ticket = ticket;
     P.n_arrays = (int)table.size();
     P.n_tasks = tasks;
     P.chunk = C;
@@ -506,21 +516,78 @@ static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t t
         CK_TRY(g_ring.copy(d_tab, table.data(), bytes, s));
         P.arrays = d_tab;
     }
+    const bool pm = pair != nullptr;
     if (eps == 0.0) {
-        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(P, s, sms)));
-        else CK_TRY((launch_leaf_dt<1, true>(P, s, sms)));
+        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(P, s, sms, pm)));
+        else CK_TRY((launch_leaf_dt<1, true>(P, s, sms, pm)));
     } else {
-        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(P, s, sms)));
-        else CK_TRY((launch_leaf_dt<1, false>(P, s, sms)));
+        if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(P, s, sms, pm)));
+        else CK_TRY((launch_leaf_dt<1, false>(P, s, sms, pm)));
     }
     if (d_tab) CK_CUDA(cudaFreeAsync(d_tab, s));
     return CKPT_OK;
 }
 
-extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint64_t *n,
-                                             const uint32_t *arrays_per_tree, uint32_t n_trees,
-                                             ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
-                                             void *stream, ckpt_tree **out) {
+struct Scratch {
+    uint64_t *states = nullptr;
+    size_t cap = 0;
+    unsigned long long *ticket = nullptr;
+    uint32_t epoch = 0;
+    uint8_t *work = nullptr;       // K4 per-chunk counts + hit bitmasks
+    size_t work_cap = 0;
+    unsigned int *pair_ctr = nullptr;   // fused pair mode: one self-resetting counter per pair-task
+    size_t pair_cap = 0;
+    uint8_t *pair_flags = nullptr;      // fused pair mode: one flag byte per chunk
+    size_t flags_cap = 0;
+};
+static std::mutex g_scr_mu;
+static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
+
+static ckpt_status get_pair_flags(int dev, cudaStream_t s, size_t n, uint8_t **flags) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    Scratch &sc = g_scr[std::make_pair(dev, s)];
+    n = std::max<size_t>(n, 256);
+    if (sc.flags_cap < n) {
+        if (sc.pair_flags) CK_CUDA(cudaFreeAsync(sc.pair_flags, s));
+        sc.flags_cap = std::max<size_t>(n, 2 * sc.flags_cap);
+        CK_CUDA(cudaMallocAsync((void **)&sc.pair_flags, sc.flags_cap, s));
+    }
+    *flags = sc.pair_flags;
+    return CKPT_OK;
+}
+
+constexpr int kLeafTicketSlot = 16;   // 8-byte slot of the per-stream ticket block used by K1
+
+// CKPT_LEAF_STATIC=1: K1 warps stride over tasks statically (A/B measurement only).
+static bool leaf_static_tasks() {
+    static const bool on = [] {
+        const char *e = std::getenv("CKPT_LEAF_STATIC");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
+// Zero-initialised pair-task counters (they return to 0 after every launch).
+static ckpt_status get_pair_ctr(int dev, cudaStream_t s, size_t n, unsigned int **ctr) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    Scratch &sc = g_scr[std::make_pair(dev, s)];
+    n = std::max<size_t>(n, 1);
+    if (sc.pair_cap < n) {
+        if (sc.pair_ctr) CK_CUDA(cudaFreeAsync(sc.pair_ctr, s));
+        sc.pair_cap = std::max<size_t>(n, 2 * sc.pair_cap);
+        CK_CUDA(cudaMallocAsync((void **)&sc.pair_ctr, sc.pair_cap * 4, s));
+        CK_CUDA(cudaMemsetAsync(sc.pair_ctr, 0, sc.pair_cap * 4, s));
+    }
+    *ctr = sc.pair_ctr;
+    return CKPT_OK;
+}
+
+// Trees of several checkpoints with one leaf-kernel launch.  `pair` != NULL:
+// fused pair mode (two checkpoints of identical shape; see PairParams).
+static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
+                                    const uint32_t *arrays_per_tree, uint32_t n_trees,
+                                    ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                    void *stream, ckpt_tree **out, const PairParams *pair) {
     if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
     for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
     if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
@@ -568,12 +635,27 @@ extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint
             e.n_full = e.nbytes / chunk_bytes;
             e.task_begin = task;
             e.out = t->nodes + t->off[a];      // level 0 of array a
+            e.chunk_base = t->chunk_base[a];
             table.push_back(e);
             task += (leaves[a] + kRows - 1) / kRows;
         }
         a0 += na;
     }
-    if (st == CKPT_OK) st = launch_leaves(table, task, dtype, eps, chunk_bytes, s, di.sms);
+    PairParams pp;
+    unsigned long long *ticket = nullptr;
+    if (pair) {
+        pp = *pair;
+        pp.n_pair = task / 2;                  // A's tasks; B's are the same count
+        st = get_pair_ctr(dev, s, pp.n_pair, &pp.ctr);
+    }
+    if (st == CKPT_OK && !leaf_static_tasks()) {   // in-order dynamic tasks (no tail imbalance)
+        uint64_t *unused_states;
+        uint32_t unused_epoch;
+        st = get_scratch(dev, s, 0, &unused_states, &ticket, &unused_epoch);
+        ticket += kLeafTicketSlot;
+    }
+    if (st == CKPT_OK)
+        st = launch_leaves(table, task, dtype, eps, chunk_bytes, s, di.sms, pair ? &pp : nullptr, ticket);
     if (st == CKPT_OK) {
         // K2 on the side stream, after the leaves; each tree records its own event
         cudaStream_t ss = nullptr;
@@ -596,6 +678,14 @@ extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint
         return st;
     }
     return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint64_t *n,
+                                             const uint32_t *arrays_per_tree, uint32_t n_trees,
+                                             ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                             void *stream, ckpt_tree **out) {
+    return build_batch_impl(data, n, arrays_per_tree, n_trees, dtype, chunk_bytes, eps, stream, out,
+                            nullptr);
 }
 
 extern "C" ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n,
@@ -681,16 +771,6 @@ static ckpt_status check_pair(const ckpt_tree *a, const ckpt_tree *b) {
 // per-(device, stream) scratch for the ordered compactions: look-back states
 // tagged with a launch epoch (never cleared) and a self-resetting ticket.
 // ---------------------------------------------------------------------------
-struct Scratch {
-    uint64_t *states = nullptr;
-    size_t cap = 0;
-    unsigned long long *ticket = nullptr;
-    uint32_t epoch = 0;
-    uint8_t *work = nullptr;       // K4 per-chunk counts + hit bitmasks
-    size_t work_cap = 0;
-};
-static std::mutex g_scr_mu;
-static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
 
 static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_t **states,
                                unsigned long long **ticket, uint32_t *epoch) {
@@ -995,6 +1075,61 @@ extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tr
     return verify_impl(a, b, ta->n_elems.data(), ta->n_arrays, ta->dtype, ta->chunk_bytes, chunks,
                        counts_dev, 0, chunks_cap, ta->eps, idx, idx_cap, counts_dev + 1,
                        (cudaStream_t)stream);
+}
+
+// ---------------------------------------------------------------------------
+// fused pair compare: K1 in pair mode (digest compare and
+// element marking in-kernel), then the ordered chunk list and the element ids
+// ---------------------------------------------------------------------------
+extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void *const *b,
+                                               const uint64_t *n, uint32_t n_arrays,
+                                               ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                               uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                               uint64_t idx_cap, uint64_t *counts_dev, void *stream,
+                                               ckpt_tree **out_a, ckpt_tree **out_b) {
+    if (out_a) *out_a = nullptr;
+    if (out_b) *out_b = nullptr;
+    if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
+    if (!out_a || !out_b) return fail(CKPT_EINVAL, "NULL tree outputs");
+    if (!counts_dev || (!chunks && chunks_cap) || (!idx && idx_cap))
+        return fail(CKPT_EINVAL, "NULL argument");
+    if (n_arrays >= (1u << 20)) return fail(CKPT_EINVAL, "too many arrays");
+    CK_TRY(check_common(dtype, chunk_bytes, eps));
+    const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
+    uint64_t L = 0;
+    for (uint32_t k = 0; k < n_arrays; ++k) L += (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    cudaStream_t s = (cudaStream_t)stream;
+    PairParams pp;
+    std::memset(&pp, 0, sizeof(pp));
+    pp.m = (int)n_arrays;
+    // flag bytes live in their own per-stream buffer (verify's work buffer may regrow)
+    CK_TRY(get_pair_flags(dev, s, L, &pp.flags));
+    std::vector<const void *> data(2 * (size_t)n_arrays);
+    std::vector<uint64_t> nn(2 * (size_t)n_arrays);
+    for (uint32_t k = 0; k < n_arrays; ++k) {
+        data[k] = a[k];
+        data[n_arrays + k] = b[k];
+        nn[k] = nn[n_arrays + k] = n[k];
+    }
+    const uint32_t apt[2] = {n_arrays, n_arrays};
+    ckpt_tree *trees[2] = {nullptr, nullptr};
+    CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, stream, trees, &pp));
+    ckpt_status st = launch_compact(1, nullptr, nullptr, pp.flags, L, chunks, chunks_cap, counts_dev, s,
+                                    di.sms);
+    if (st == CKPT_OK)
+        st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
+                         idx, idx_cap, counts_dev + 1, s);
+    if (st != CKPT_OK) {
+        ckpt_tree_free_on(trees[0], stream);
+        ckpt_tree_free_on(trees[1], stream);
+        return st;
+    }
+    *out_a = trees[0];
+    *out_b = trees[1];
+    return CKPT_OK;
 }
 
 extern "C" ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b,

@@ -10,6 +10,7 @@
 #include <cstdint>
 
 #include "hash.cuh"
+#include "mark.cuh"
 
 namespace ckpt {
 
@@ -304,10 +305,6 @@ __global__ void bfs_step_kernel(BfsParams p, const uint64_t *in, const unsigned 
 // ---------------------------------------------------------------------------
 constexpr int kVerifyWarps = 8;
 constexpr int kVerifyThreads = kVerifyWarps * 32;
-#ifndef CKPT_VERIFY_BATCH
-#define CKPT_VERIFY_BATCH 4
-#endif
-constexpr int kVerifyBatch = CKPT_VERIFY_BATCH;   // warp iterations whose loads are issued together
 
 struct VerifyArray {
     const uint8_t *a;
@@ -388,54 +385,10 @@ __device__ __forceinline__ ChunkLoc shfl_loc(const ChunkLoc &l, int src) {
     return o;
 }
 
-// Bits of |a-b| > eps (computed in double, reading R9) for the VEC elements
-// of one 16-byte vector pair.
-template <int DT>
-__device__ __forceinline__ uint32_t diff_vec(uint4 va, uint4 vb, double eps) {
-    uint32_t m = 0;
-    if (DT == 0) {
-        m |= (fabs((double)__uint_as_float(va.x) - (double)__uint_as_float(vb.x)) > eps) ? 1u : 0u;
-        m |= (fabs((double)__uint_as_float(va.y) - (double)__uint_as_float(vb.y)) > eps) ? 2u : 0u;
-        m |= (fabs((double)__uint_as_float(va.z) - (double)__uint_as_float(vb.z)) > eps) ? 4u : 0u;
-        m |= (fabs((double)__uint_as_float(va.w) - (double)__uint_as_float(vb.w)) > eps) ? 8u : 0u;
-    } else {
-        const double a0 = __hiloint2double((int)va.y, (int)va.x), b0 = __hiloint2double((int)vb.y, (int)vb.x);
-        const double a1 = __hiloint2double((int)va.w, (int)va.z), b1 = __hiloint2double((int)vb.w, (int)vb.z);
-        m |= (fabs(a0 - b0) > eps) ? 1u : 0u;
-        m |= (fabs(a1 - b1) > eps) ? 2u : 0u;
-    }
-    return m;
-}
-
-// Scalar tail: elements e.. of a vector that crosses the chunk end.
-template <int DT>
-__device__ __forceinline__ uint32_t diff_tail(const uint8_t *pa, const uint8_t *pb, uint64_t e,
-                                              uint64_t len, double eps) {
-    constexpr int VEC = DT == 0 ? 4 : 2;
-    uint32_t m = 0;
-    for (int v = 0; v < VEC; ++v) {
-        if (e + v >= len) break;
-        double x, y;
-        if (DT == 0) {
-            x = (double)reinterpret_cast<const float *>(pa)[e + v];
-            y = (double)reinterpret_cast<const float *>(pb)[e + v];
-        } else {
-            x = reinterpret_cast<const double *>(pa)[e + v];
-            y = reinterpret_cast<const double *>(pb)[e + v];
-        }
-        if (fabs(x - y) > eps) m |= 1u << v;
-    }
-    return m;
-}
-
 template <int DT>
 __global__ void __launch_bounds__(kVerifyThreads) verify_mark_kernel(const __grid_constant__ VerifyParams p) {
     pdl_enter();
-    constexpr int VEC = DT == 0 ? 4 : 2;
     constexpr int ESZ = DT == 0 ? 4 : 8;
-    constexpr int kStep = 32 * VEC;            // elements per warp iteration
-    constexpr int IPG = 32 / VEC;              // warp iterations per group of 32 mask words
-    constexpr int LPW = 32 / VEC;              // lanes contributing to one mask word
     const int lane = threadIdx.x & 31;
     const uint64_t n_chunks = verify_n_chunks(p);
     const uint64_t n_warps = (uint64_t)gridDim.x * kVerifyWarps;
@@ -451,43 +404,7 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_mark_kernel(const __gri
         const ChunkLoc L = shfl_loc(mine, j);
         const uint8_t *pa = L.pa, *pb = L.pb;
         const uint64_t len = L.len;
-        const uint4 *qa = reinterpret_cast<const uint4 *>(pa);
-        const uint4 *qb = reinterpret_cast<const uint4 *>(pb);
-        uint32_t *mq = p.mask + q * p.groups * 32 + lane;
-        uint32_t cnt = 0, word = 0;
-        int it = 0;
-        for (uint64_t base = 0; base < len; base += (uint64_t)kVerifyBatch * kStep) {
-            uint4 va[kVerifyBatch], vb[kVerifyBatch];
-#pragma unroll
-            for (int u = 0; u < kVerifyBatch; ++u) {
-                const uint64_t e = base + (uint64_t)u * kStep + (uint64_t)lane * VEC;
-                if (e + VEC <= len) {
-                    va[u] = __ldcs(qa + e / VEC);
-                    vb[u] = __ldcs(qb + e / VEC);
-                }
-            }
-#pragma unroll
-            for (int u = 0; u < kVerifyBatch; ++u) {
-                const uint64_t e0 = base + (uint64_t)u * kStep;
-                if (e0 >= len) break;                          // warp-uniform
-                const uint64_t e = e0 + (uint64_t)lane * VEC;
-                uint32_t m = 0;
-                if (e + VEC <= len) m = diff_vec<DT>(va[u], vb[u], p.eps);
-                else if (e < len) m = diff_tail<DT>(pa, pb, e, len, p.eps);
-                cnt += __popc(m);
-                // transpose to element-contiguous words: word k of this iteration
-                // (elements k*32.. of its 32*VEC) is gathered from LPW lanes and
-                // lands in lane (it % IPG) * VEC + k
-                uint32_t x = m << (VEC * (lane % LPW));
-#pragma unroll
-                for (int o = 1; o < LPW; o <<= 1) x |= __shfl_xor_sync(kFull, x, o);
-                const uint32_t y = __shfl_sync(kFull, x, (lane % VEC) * LPW);
-                if (lane / VEC == it % IPG) word = y;
-                if (++it % IPG == 0) { __stcs(mq, word); mq += 32; word = 0; }
-            }
-        }
-        if (it % IPG) __stcs(mq, word);
-        cnt = (uint32_t)warp_sum_u64(cnt);
+        const uint32_t cnt = mark_chunk<DT>(pa, pb, len, p.eps, p.mask + q * p.groups * 32, lane);
         if (lane == 0) p.cnt[q] = cnt;
       }
     }
@@ -584,10 +501,11 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
     const uint32_t n_words = p.groups * 32;
     for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + (threadIdx.x >> 5)) * G; q0 < n_chunks;
          q0 += n_warps * G) {
-      uint64_t my_off = 0, my_gb = 0;
+      uint64_t my_off = 0, my_gb = 0, my_key = 0;
       uint32_t c = 0;
       if (lane < (int)G && q0 + lane < n_chunks) {
-          c = p.cnt[q0 + lane];
+          my_key = q0 + lane;
+          c = p.cnt[my_key];
           if (c) {
               const uint8_t *pa, *pb;
               uint64_t len;
@@ -597,7 +515,7 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
       }
       // sparse chunks: one lane each
       if (c && c <= kEmitSparse) {
-          const uint4 *mw = reinterpret_cast<const uint4 *>(p.mask + (q0 + lane) * n_words);
+          const uint4 *mw = reinterpret_cast<const uint4 *>(p.mask + my_key * n_words);
           uint64_t o = my_off;
 #pragma unroll 1
           for (uint32_t w4 = 0; w4 < n_words / 4; ++w4) {
@@ -617,7 +535,7 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
         const int j = __ffs(todo) - 1;
         const uint64_t gbase = __shfl_sync(kFull, my_gb, j);
         uint64_t pos = __shfl_sync(kFull, my_off, j);
-        const uint32_t *mq = p.mask + (q0 + j) * n_words + lane;
+        const uint32_t *mq = p.mask + __shfl_sync(kFull, my_key, j) * n_words + lane;
 #pragma unroll 1
         for (uint32_t g = 0; g < p.groups; ++g)
             pos += emit_words(__ldcs(mq + g * 32), gbase + (uint64_t)g * 1024, pos, p.out, p.cap, lane,

@@ -28,6 +28,7 @@ struct LeafArray {            // one array of the checkpoint (device table)
     uint64_t n_full;          // nbytes / C  (chunks of exactly C bytes)
     uint64_t task_begin;      // first global task id of this array
     uint4 *out;               // this array's leaf 0 in its tree's node storage
+    uint64_t chunk_base;      // global chunk id of this array's chunk 0 in its tree
 };
 
 #ifndef CKPT_LEAF_SEG
@@ -160,6 +161,22 @@ __device__ __noinline__ void chain_tail(uint64_t &h1, uint64_t &h2, const uint8_
 
 constexpr int kLeafInline = 16;
 
+// Fused pair mode: the table holds checkpoint A's m
+// arrays then B's m arrays (identical shapes); warp task t < n_pair is A's
+// task t, t >= n_pair is B's task t - n_pair (the usual batch order, so the
+// warps in flight stream one checkpoint at a time).  Whichever of the two
+// warps of a pair-task finishes second (a self-resetting atomicInc counter per
+// pair-task) compares the 32 leaf digests and writes one flag byte per chunk:
+// the diff at start level 0 happens inside K1.  (Marking the flagged chunks'
+// elements here as well was measured slower than K4a: flagged chunks cluster,
+// so the marking serialises in the few warps that own them.)
+struct PairParams {
+    uint8_t *flags;               // [L] 1 if the chunk's leaf digests differ
+    unsigned int *ctr;            // [n_pair] 0 between launches (atomicInc wraps 1 -> 0)
+    uint64_t n_pair;              // pair-tasks (A's warp tasks)
+    int m;                        // arrays per checkpoint
+};
+
 struct LeafParams {
     const LeafArray *arrays;      // device table when n_arrays > kLeafInline
     LeafArray inl[kLeafInline];
@@ -167,6 +184,10 @@ struct LeafParams {
     uint64_t n_tasks;
     uint32_t chunk;
     QuantParams q;
+    PairParams pr;
+    // non-null: warps draw tasks in order from this counter (0 at launch; the
+    // final draw resets it), so a warp held up by marking takes fewer tasks
+    unsigned long long *ticket;
 };
 
 __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, uint64_t task) {
@@ -182,7 +203,7 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
 // A task is kRows = 32*kCh consecutive chunks of one array; lane l owns the
 // chains of rows l, l+32, ... (kCh independent chains per lane give the
 // scheduler two interleavable instruction streams).
-template <int DT, bool RAW, int CB>
+template <int DT, bool RAW, int CB, bool PAIR>
 __global__ void __launch_bounds__(kLeafWarps * 32, CKPT_LEAF_MINB)
 leaf_kernel(const __grid_constant__ LeafParams P) {
     pdl_enter();
@@ -214,8 +235,17 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
         q.m2 = *reinterpret_cast<volatile uint64_t *>(cst + 1);
     }
 
-    for (uint64_t task = (uint64_t)blockIdx.x * kLeafWarps + warp; task < n_tasks;
-         task += (uint64_t)gridDim.x * kLeafWarps) {
+    const uint64_t n_warps_grid = (uint64_t)gridDim.x * kLeafWarps;
+    auto draw = [&]() -> uint64_t {
+        unsigned long long t = 0;
+        if (lane == 0) {
+            t = atomicAdd(P.ticket, 1ull);
+            if (t == n_tasks + n_warps_grid - 1) *P.ticket = 0ull;   // the last draw of the launch
+        }
+        return __shfl_sync(0xffffffffu, t, 0);
+    };
+    for (uint64_t task = P.ticket ? draw() : (uint64_t)blockIdx.x * kLeafWarps + warp; task < n_tasks;
+         task = P.ticket ? draw() : task + n_warps_grid) {
         const int a = find_array(arrays, n_arrays, task);
         const LeafArray A = arrays[a];
         const uint64_t c0 = (task - A.task_begin) * kRows;   // first local chunk of the task
@@ -336,6 +366,27 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
         for (int j = 0; j < kCh; ++j) {
             const uint64_t c = c0 + 32 * j + lane;
             if (c < A.n_leaves) A.out[c] = make_uint4(h1[j].lo, h1[j].hi, h2[j].lo, h2[j].hi);
+        }
+        if (PAIR) {
+            static_assert(!PAIR || kCh == 1, "pair mode assumes one chain per lane");
+            const int side = a >= P.pr.m ? 1 : 0;
+            const uint64_t pt = task - (side ? P.pr.n_pair : 0);
+            // publish my leaves, then count in; the second of the pair does the compare
+            __threadfence();
+            unsigned int order = 0;
+            if (lane == 0) order = atomicInc(&P.pr.ctr[pt], 1u);
+            order = __shfl_sync(0xffffffffu, order, 0);
+            if (order == 1) {
+                __threadfence();
+                const LeafArray Pa = arrays[side ? a - P.pr.m : a + P.pr.m];   // the other run
+                const uint64_t c = c0 + lane;
+                if (c < A.n_leaves) {
+                    const uint4 o = __ldcg(Pa.out + c);
+                    const bool differ = (o.x != h1[0].lo) | (o.y != h1[0].hi) | (o.z != h2[0].lo) |
+                                        (o.w != h2[0].hi);
+                    P.pr.flags[A.chunk_base + c] = differ ? 1 : 0;
+                }
+            }
         }
         __syncwarp();
     }

@@ -414,3 +414,87 @@ def test_config5_shape_verify_heavy_bfs_path():
     # false positives exist (flagged chunks without a verified difference)
     per = C // 4
     assert np.setdiff1d(ref_chunks, np.unique(ref_idx // per)).size > 0
+
+
+# ------------------------------------------------- fused pair compare path --
+
+def _pair_cases():
+    return [
+        ("c1", lambda: synth.c1_pair(n=1 << 20, seed=21, device="cuda")),
+        ("c1_tail", lambda: synth.c1_pair(n=1_000_003, seed=22, device="cuda")),
+        ("c2_small", lambda: synth.c2_pair(n_particles=(1 << 18) + 77, seed=23, device="cuda")),
+        ("c5_small", lambda: synth.c5_pair(n_ranks=2, n_particles=1 << 16, seed=24, device="cuda")),
+        ("c3_small", lambda: synth.c3_pair(n=(1 << 20) + 5, seed=25, device="cuda", n_clusters=16,
+                                           mean_len=512)),
+    ]
+
+
+@pytest.mark.parametrize("name,make", _pair_cases(), ids=[c[0] for c in _pair_cases()])
+@pytest.mark.parametrize("chunk", [4096, 512, 48])
+def test_compare_pair_matches_oracle(name, make, chunk):
+    pair = make()
+    eps = pair.eps
+    if name.startswith("c3") and chunk == 48:
+        chunk = 64                                # f64: keep C a multiple of 16 and of 8
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    L = sum(-(-t.numel() * t.element_size() // chunk) for t in pair.a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(sum(t.numel() for t in pair.a), dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(pair.a, pair.b, chunk, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    torch.cuda.synchronize()
+    A = oracle.build_checkpoint(an, chunk, eps, threads=8)
+    B = oracle.build_checkpoint(bn, chunk, eps, threads=8)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, chunk, ref_chunks, eps, A)
+    nc, nd = counts.tolist()
+    assert np.array_equal(np_of(chunks[:nc]), ref_chunks)
+    assert np.array_equal(np_of(idx[:nd]), ref_idx)
+    # both trees are complete and equal the oracle's, array by array
+    for k in range(len(an)):
+        assert np.array_equal(gpu_tree_nodes(TA, k), A.trees[k]), k
+        assert np.array_equal(gpu_tree_nodes(TB, k), B.trees[k]), k
+    assert TA.root() == A.root and TB.root() == B.root
+
+
+def test_compare_pair_equals_unfused_path_and_raw_mode():
+    pair = synth.c2_pair(n_particles=(1 << 17) + 3, seed=31, device="cuda")
+    for eps in (pair.eps, 0.0):
+        L = sum(-(-t.numel() * 4 // 4096) for t in pair.a)
+        n = sum(t.numel() for t in pair.a)
+        outs = []
+        for fused in (True, False):
+            chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+            idx = torch.empty(n, dtype=torch.int64, device="cuda")
+            counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+            if fused:
+                TA, TB = ck.compare_pair_async(pair.a, pair.b, 4096, eps, chunks, idx, counts)
+            else:
+                TA, TB = ck.tree_build_batch([pair.a, pair.b], 4096, eps)
+                ck.diff_verify_async(TA, TB, pair.a, pair.b, chunks, idx, counts)
+            TA.wait(); TB.wait()
+            nc, nd = counts.tolist()
+            outs.append((np_of(chunks[:nc]), np_of(idx[:nd]), TA.root(), TB.root()))
+        for x, y in zip(outs[0], outs[1]):
+            assert np.array_equal(np.asarray(x), np.asarray(y)) if not isinstance(x, bytes) else x == y
+
+
+def test_compare_pair_identical_and_truncated():
+    a = [synth.uniform(41, 100_000, "cuda"), synth.uniform(42, 5_000, "cuda")]
+    b = [t.clone() for t in a]
+    chunks = torch.empty(200, dtype=torch.int64, device="cuda")
+    idx = torch.empty(64, dtype=torch.int64, device="cuda")
+    counts = torch.full((2,), 7, dtype=torch.int64, device="cuda")
+    ck.compare_pair_async(a, b, 4096, 1e-6, chunks, idx, counts)
+    assert counts.tolist() == [0, 0]
+    b[0][::1000] += 1.0                                        # 100 elements
+    ck.compare_pair_async(a, b, 4096, 1e-6, chunks, idx, counts)
+    nc, nd = counts.tolist()
+    ref = np.nonzero(np.abs(np_of(a[0]).astype(np.float64) - np_of(b[0]).astype(np.float64)) > 1e-6)[0]
+    assert nc == np.unique(ref // 1024).size and nd == ref.size == 100   # full count past the cap
+    assert np.array_equal(np_of(chunks[:nc]), np.unique(ref // 1024))
+    assert np.array_equal(np_of(idx), ref[:64])
+    with pytest.raises(ValueError):
+        ck.compare_pair_async(a, [b[0]], 4096, 1e-6, chunks, idx, counts)

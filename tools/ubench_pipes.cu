@@ -72,6 +72,18 @@ __global__ void k(uint32_t *out, uint32_t seed) {
 #define S(x) asm volatile("{.reg .u64 p, q; mov.b64 q, {%1, %2}; mad.wide.u32 p, %0, 5, q; cvt.u32.u64 %0, p;}" : "+r"(x) : "r"(b), "r"(c));
             CHAIN8(S)
 #undef S
+        } else if (OP == 14) {  // 64-bit add as IMAD.WIDE.U32 x*1 + pair (FMA pipe)
+#define S(x) asm volatile("{.reg .u64 p, q; mov.b64 q, {%1, %2}; mad.wide.u32 p, %0, 1, q; mov.b64 {%0, %1}, p;}" : "+r"(x), "+r"(b) : "r"(c));
+            CHAIN8(S)
+#undef S
+        } else if (OP == 15) {  // mad.lo x*2^k + y (IMAD.SHL-style shift-add)
+#define S(x) asm volatile("mad.lo.u32 %0, %0, 32, %1;" : "+r"(x) : "r"(b));
+            CHAIN8(S)
+#undef S
+        } else if (OP == 16) {  // PRMT
+#define S(x) asm volatile("prmt.b32 %0, %0, %1, 0x3210;" : "+r"(x) : "r"(b));
+            CHAIN8(S)
+#undef S
         } else if (OP == 13) {  // FFMA (reference)
 #define S(x) asm volatile("fma.rn.f32 %0, %0, 1.0001, 0.5;" : "+f"(f##x));
             S(0) S(1) S(2) S(3) S(4) S(5) S(6) S(7)
@@ -123,5 +135,8 @@ int main() {
     run<8>("F2F.F64.F32 + DADD (2)", sms, out, 2);
     run<9>("DFMA.RM", sms, out, 1);
     run<13>("FFMA", sms, out, 1);
+    run<14>("IMAD.WIDE x*1+pair (64b add)", sms, out, 1);
+    run<15>("IMAD x*32+y", sms, out, 1);
+    run<16>("PRMT", sms, out, 1);
     return 0;
 }
