@@ -47,6 +47,7 @@ CONFIGS = {
                "1024 geometric clusters (mean 4096) with |d|=10^U(-9,-2)"),
 }
 CFG = "c2"
+HASH_BLOCK = 16
 N_PARTICLES = CONFIGS[CFG]["n"]
 WORKLOAD = CONFIGS[CFG]["workload"]
 
@@ -145,8 +146,8 @@ def oracle_pair_sample(n_particles: int, seed: int):
 def oracle_step(a_list, b_list, threads: int):
     """The oracle as it stands: build A, build B, BFS diff, verify (all arrays)."""
     import oracle
-    A = oracle.build_checkpoint(a_list, CHUNK, EPS, threads=threads)
-    B = oracle.build_checkpoint(b_list, CHUNK, EPS, threads=threads)
+    A = oracle.build_checkpoint(a_list, CHUNK, EPS, threads=threads, hash_block=HASH_BLOCK)
+    B = oracle.build_checkpoint(b_list, CHUNK, EPS, threads=threads, hash_block=HASH_BLOCK)
     ch = oracle.diff_checkpoint(A, B)
     idx = oracle.verify_checkpoint(a_list, b_list, CHUNK, ch, EPS, A)
     return ch.size, idx.size
@@ -256,9 +257,10 @@ def run_ours(args):
     def step():
         if args.path == "fused":
             # one leaf launch hashes both runs, compares the digests and marks the flagged chunks
-            TA, TB = ck.compare_pair_async(A, B, CHUNK, EPS, chunks, idx, counts)
+            TA, TB = ck.compare_pair_async(A, B, CHUNK, EPS, chunks, idx, counts,
+                                           hash_block=args.hash_block)
         else:
-            TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS)     # one leaf launch for both runs
+            TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS, hash_block=args.hash_block)
             ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # BFS diff, then verify
         if world > 1:
             tops = []
@@ -374,7 +376,8 @@ def run_ours(args):
                        "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair,
                        "l2": f"inputs larger than L2 ({bytes_pair / 1e9:.1f} GB per GPU per step >> 126 MB)",
                        "parallelism": f"dp{world} (checkpoint arrays sharded by rank)",
-                       "path": args.path},
+                       "path": args.path,
+                       "hash_block": args.hash_block if args.hash_block else "chunk"},
             "pct_hbm_peak": round(value / (world * peak), 4),
             "roofline": {"bound": "hbm", "kernel": "leaf_kernel (K1: quantize + chained Murmur3F)",
                          "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
@@ -403,9 +406,13 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--path", default="fused", choices=["fused", "unfused"],
                     help="fused: ckpt_compare_pair_async; unfused: build_batch + diff_verify_async")
+    ap.add_argument("--hash-block", type=int, default=16,
+                    help="bytes per chained Murmur3F call: 16 = the paper's 128-bit blocks "
+                         "(P:610, default); 0 = whole chunk (P:615-618 variant, R23)")
     args = ap.parse_args()
-    global CFG, N_PARTICLES, WORKLOAD
+    global CFG, N_PARTICLES, WORKLOAD, HASH_BLOCK
     CFG = args.config
+    HASH_BLOCK = args.hash_block
     N_PARTICLES = CONFIGS[CFG]["n"]
     WORKLOAD = CONFIGS[CFG]["workload"]
     if args.impl == "reference":

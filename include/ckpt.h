@@ -119,6 +119,24 @@ ckpt_status ckpt_tree_build_batch(const void *const *data, const uint64_t *n,
                                   ckpt_dtype dtype, uint32_t chunk_bytes, double eps, void *stream,
                                   ckpt_tree **out);
 
+/* Hash-block variant (reading R23).  The paper hashes 128-bit blocks
+ * and notes that "the block size is variable and can be adjusted":
+ * the chain of the leaf runs over blocks of hash_block bytes, each block one
+ * complete Murmur3F call seeded with the previous digest; a chunk's last block
+ * holds the bytes that remain and is hashed with its own length.
+ *   hash_block  16 = the default of every other entry point; any positive
+ *               multiple of 16; 0 (or >= chunk_bytes) = the whole chunk in one
+ *               Murmur3F call, seed 0.
+ * Larger blocks finalise less often (fewer instructions per byte); the
+ * quantizer, the tree levels, diff and verify are unchanged, and the set of
+ * flagged chunks is the same (barring 2^-128 collisions).  Trees of different
+ * hash_block are incompatible (CKPT_EMISMATCH in diff).  Errors as
+ * ckpt_tree_build_batch, plus CKPT_EINVAL when hash_block % 16 != 0. */
+ckpt_status ckpt_tree_build_batch_ex(const void *const *data, const uint64_t *n,
+                                     const uint32_t *arrays_per_tree, uint32_t n_trees,
+                                     ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                     uint32_t hash_block, void *stream, ckpt_tree **out);
+
 /* Tree over caller-supplied 16-byte digests used as leaves (no data
  * hashing).  Used to form the top levels over the subtree roots gathered
  * from all GPUs (R15; the multi-GPU path).  digests16: device, count*16
@@ -225,6 +243,13 @@ ckpt_status ckpt_compare_pair_async(const void *const *a, const void *const *b, 
                                     double eps, uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
                                     uint64_t idx_cap, uint64_t *counts_dev, void *stream,
                                     ckpt_tree **out_a, ckpt_tree **out_b);
+/* Same with a hash block size (see ckpt_tree_build_batch_ex). */
+ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *const *b, const uint64_t *n,
+                                 uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                 double eps, uint32_t hash_block, uint64_t *chunks,
+                                 uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                                 uint64_t *counts_dev, void *stream, ckpt_tree **out_a,
+                                 ckpt_tree **out_b);
 
 /* ------------------------------------------------------------------------
  * One-call pair comparison (steps 1-4 on two checkpoints of n_arrays
@@ -251,6 +276,54 @@ ckpt_status ckpt_compare_host(const void *const *a, const void *const *b, const 
                               uint64_t *n_diff, uint8_t *root_a16, uint8_t *root_b16);
 
 /* ------------------------------------------------------------------------
+ * Tree persistence.  The tree is built at capture time
+ * and stored next to the checkpoint (metadata ~0.8% of the data
+ * at 4 KB chunks); a later comparison loads it instead of re-hashing that run
+ * and reads only the flagged chunks of the stored data (P:899-904,
+ * P:1412-1416).
+ *
+ * Format (little-endian): "CKPTTRE1" | u32 version=1 | u32 dtype |
+ * u32 chunk_bytes | u32 hash_block | f64 eps | u32 n_arrays | u32 0 |
+ * u64 n_elems[n_arrays] | u64 node_count | 16-byte checkpoint root |
+ * node_count x 16-byte nodes in the device layout (level-major across arrays,
+ * then the top tree over the array roots; R13, R15).
+ * ---------------------------------------------------------------------- */
+
+/* (host) *bytes = size of the serialised tree.  CKPT_EINVAL for NULL or a
+ * tree built from digests. */
+ckpt_status ckpt_tree_serialized_size(const ckpt_tree *t, uint64_t *bytes);
+
+/* Write the tree to dst (host, cap bytes; *written (host) = the size).  Waits
+ * for the tree's levels and synchronises `stream`.  CKPT_EINVAL when cap is
+ * smaller than ckpt_tree_serialized_size. */
+ckpt_status ckpt_tree_serialize(const ckpt_tree *t, void *dst, uint64_t cap, uint64_t *written,
+                                void *stream);
+
+/* Load a serialised tree (src: host, `bytes` long) onto the current device.
+ * The header is validated on the host before any device work: CKPT_EINVAL for
+ * a bad magic/version, invalid parameters, a size that does not match the
+ * header, or a stored root that differs from the last node.  Synchronises
+ * `stream` (src may be reused on return).  The tree supports every tree
+ * entry point (diff, roots, nodes, params, serialize). */
+ckpt_status ckpt_tree_deserialize(const void *src, uint64_t bytes, void *stream, ckpt_tree **out);
+
+/* Compare a live checkpoint (run B) with a stored run A: A's tree is loaded
+ * from saved_a (host, saved_bytes; as ckpt_tree_deserialize), B's tree is
+ * built with A's dtype / chunk_bytes / eps / hash_block, then steps 3+4 run
+ * as ckpt_diff_verify_async.  a_data (host array of n_arrays pointers) are
+ * run A's arrays: device pointers, or host memory the device can address
+ * (pinned / registered, through unified addressing) -- the verify kernels
+ * read only the flagged chunks of A.  b: device arrays; n (host): element
+ * counts, which must equal the stored ones (else CKPT_EMISMATCH).  Outputs as
+ * ckpt_compare_pair_async; both trees are returned (*out_a, *out_b).
+ * Asynchronous after the tree upload. */
+ckpt_status ckpt_compare_saved(const void *saved_a, uint64_t saved_bytes, const void *const *a_data,
+                               const void *const *b, const uint64_t *n, uint32_t n_arrays,
+                               uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                               uint64_t idx_cap, uint64_t *counts_dev, void *stream,
+                               ckpt_tree **out_a, ckpt_tree **out_b);
+
+/* ------------------------------------------------------------------------
  * Accessors (parity tests, multi-GPU driver)
  * ---------------------------------------------------------------------- */
 
@@ -266,6 +339,12 @@ ckpt_status ckpt_tree_wait(const ckpt_tree *t, void *stream);
  * (all arrays, all levels; excludes the top tree over array roots). */
 ckpt_status ckpt_tree_info(const ckpt_tree *t, uint32_t *n_arrays, uint64_t *n_leaves,
                            uint32_t *n_levels, uint64_t *n_nodes);
+
+/* (host outputs, any may be NULL) the hashing parameters of a built tree:
+ * dtype, chunk_bytes, eps and the effective hash block in bytes (16, ...,
+ * chunk_bytes = whole chunk).  CKPT_EINVAL for trees built from digests. */
+ckpt_status ckpt_tree_params(const ckpt_tree *t, ckpt_dtype *dtype, uint32_t *chunk_bytes,
+                             double *eps, uint32_t *hash_block);
 
 /* (host) 16-byte checkpoint root = root of the tree over the array roots
  * (equal to the array root when n_arrays == 1).  Synchronises `stream`. */

@@ -69,6 +69,8 @@ def lib():
         L.orc_n_chunks.restype = u64
         L.orc_leaves.argtypes = [vp, u64, i32, u32, dbl, i32, vp]
         L.orc_leaves.restype = i32
+        L.orc_leaves_blk.argtypes = [vp, u64, i32, u32, dbl, u32, i32, vp]
+        L.orc_leaves_blk.restype = i32
         L.orc_n_levels.argtypes = [u64]
         L.orc_n_levels.restype = u32
         L.orc_n_nodes.argtypes = [u64]
@@ -139,12 +141,17 @@ def n_chunks(n: int, dtype_code: int, chunk_bytes: int) -> int:
     return lib().orc_n_chunks(n, dtype_code, chunk_bytes)
 
 
-def leaves(a: np.ndarray, chunk_bytes: int, eps: float, threads: int = 1) -> np.ndarray:
-    """(L, 16) uint8 leaf digests of one array (Alg. 1)."""
+def leaves(a: np.ndarray, chunk_bytes: int, eps: float, threads: int = 1,
+           hash_block: int = 16) -> np.ndarray:
+    """(L, 16) uint8 leaf digests of one array (Alg. 1).
+
+    hash_block: bytes per chained Murmur3F call (16 = the paper's 128-bit
+    blocks; any multiple of 16; 0 = the whole chunk, R23)."""
     a = np.ascontiguousarray(a).reshape(-1)
     L = n_chunks(a.size, _dtype_code(a), chunk_bytes)
     out = np.zeros((L, 16), np.uint8)
-    rc = lib().orc_leaves(_ptr(a), a.size, _dtype_code(a), chunk_bytes, eps, threads, _ptr(out))
+    rc = lib().orc_leaves_blk(_ptr(a), a.size, _dtype_code(a), chunk_bytes, eps, hash_block,
+                              threads, _ptr(out))
     if rc != 0:
         raise ValueError("invalid arguments to oracle leaves()")
     return out
@@ -224,11 +231,11 @@ class Checkpoint:
 
 
 def build_checkpoint(arrays: Sequence[np.ndarray], chunk_bytes: int, eps: float,
-                     threads: int = 1) -> Checkpoint:
+                     threads: int = 1, hash_block: int = 16) -> Checkpoint:
     trees, nl, cb, eb = [], [], [], []
     c = e = 0
     for a in arrays:
-        lv = leaves(a, chunk_bytes, eps, threads)
+        lv = leaves(a, chunk_bytes, eps, threads, hash_block)
         trees.append(levels(lv))
         nl.append(lv.shape[0])
         cb.append(c)

@@ -110,18 +110,20 @@ def words(values, is_f32: bool, eps: float) -> bytes:
     return bytes(out)
 
 
-def leaf(values, is_f32: bool, eps: float) -> bytes:
+def leaf(values, is_f32: bool, eps: float, block: int = 16) -> bytes:
+    """block: hash block bytes (16 = P:610; 0 = the whole chunk)."""
     w = words(values, is_f32, eps)
+    step = block if block else max(1, len(w))
     h1 = h2 = 0
-    for off in range(0, len(w), 16):
-        h1, h2 = murmur3f_state(w[off:off + 16], h1, h2)
+    for off in range(0, len(w), step):
+        h1, h2 = murmur3f_state(w[off:off + step], h1, h2)
     return struct.pack("<QQ", h1, h2)
 
 
-def leaves(values, is_f32: bool, chunk_bytes: int, eps: float) -> list[bytes]:
+def leaves(values, is_f32: bool, chunk_bytes: int, eps: float, block: int = 16) -> list[bytes]:
     per = chunk_bytes // (4 if is_f32 else 8)
     vals = list(values)
-    return [leaf(vals[i:i + per], is_f32, eps) for i in range(0, len(vals), per)]
+    return [leaf(vals[i:i + per], is_f32, eps, block) for i in range(0, len(vals), per)]
 
 
 def levels(leaf_list: list[bytes]) -> list[list[bytes]]:

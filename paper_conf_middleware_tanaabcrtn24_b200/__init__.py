@@ -29,6 +29,7 @@ from . import _build
 __all__ = [
     "CkptError", "Tree", "lib", "tree_build", "tree_from_digests", "tree_diff", "tree_diff_async",
     "verify", "verify_async", "compare", "compare_host", "launch_count", "default_bfs_threshold",
+    "tree_deserialize", "tree_load", "compare_saved", "compare_pair_async", "tree_build_batch",
     "F32", "F64",
 ]
 
@@ -64,6 +65,16 @@ def lib():
     L.ckpt_tree_build.argtypes = [vp, u64, i32, u32, dbl, vp, pp]
     L.ckpt_tree_build_arrays.argtypes = [pp, pu64, u32, i32, u32, dbl, vp, pp]
     L.ckpt_tree_build_batch.argtypes = [pp, pu64, ctypes.POINTER(u32), u32, i32, u32, dbl, vp, pp]
+    L.ckpt_tree_build_batch_ex.argtypes = [pp, pu64, ctypes.POINTER(u32), u32, i32, u32, dbl, u32,
+                                           vp, pp]
+    L.ckpt_compare_pair_ex.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, u32, vp, u64, vp, u64, vp,
+                                       vp, pp, pp]
+    L.ckpt_tree_serialized_size.argtypes = [vp, pu64]
+    L.ckpt_tree_serialize.argtypes = [vp, vp, u64, pu64, vp]
+    L.ckpt_tree_deserialize.argtypes = [vp, u64, vp, pp]
+    L.ckpt_compare_saved.argtypes = [vp, u64, pp, pp, pu64, u32, vp, u64, vp, u64, vp, vp, pp, pp]
+    L.ckpt_tree_params.argtypes = [vp, ctypes.POINTER(i32), ctypes.POINTER(u32),
+                                   ctypes.POINTER(dbl), ctypes.POINTER(u32)]
     L.ckpt_tree_from_digests.argtypes = [vp, u64, vp, pp]
     L.ckpt_tree_free.argtypes = [vp]
     L.ckpt_tree_free.restype = None
@@ -97,6 +108,9 @@ def lib():
     L.ckpt_last_error.restype = ctypes.c_char_p
     L.ckpt_version.restype = u32
     for name in ("ckpt_tree_build", "ckpt_tree_build_arrays", "ckpt_tree_build_batch",
+                 "ckpt_tree_build_batch_ex", "ckpt_compare_pair_ex", "ckpt_tree_params",
+                 "ckpt_tree_serialized_size", "ckpt_tree_serialize", "ckpt_tree_deserialize",
+                 "ckpt_compare_saved",
                  "ckpt_tree_from_digests",
                  "ckpt_tree_diff", "ckpt_tree_diff_async", "ckpt_verify",
                  "ckpt_verify_arrays_async", "ckpt_compare", "ckpt_compare_host",
@@ -200,6 +214,27 @@ class Tree:
                "ckpt_tree_array_roots")
         return dst
 
+    def params(self) -> Tuple[int, int, float, int]:
+        """(dtype code, chunk_bytes, eps, effective hash block bytes) as stored in the tree."""
+        d, c, e, h = ctypes.c_int(), ctypes.c_uint32(), ctypes.c_double(), ctypes.c_uint32()
+        _check(lib().ckpt_tree_params(self.handle, ctypes.byref(d), ctypes.byref(c), ctypes.byref(e),
+                                      ctypes.byref(h)), "ckpt_tree_params")
+        return d.value, c.value, e.value, h.value
+
+    def serialize(self, stream=None) -> bytes:
+        """The tree in the documented on-disk format (ckpt_tree_serialize)."""
+        n = ctypes.c_uint64()
+        _check(lib().ckpt_tree_serialized_size(self.handle, ctypes.byref(n)), "ckpt_tree_serialized_size")
+        buf = (ctypes.c_uint8 * n.value)()
+        w = ctypes.c_uint64()
+        _check(lib().ckpt_tree_serialize(self.handle, ctypes.cast(buf, ctypes.c_void_p), n.value,
+                                         ctypes.byref(w), _stream_ptr(stream)), "ckpt_tree_serialize")
+        return bytes(buf)
+
+    def save(self, path: str, stream=None) -> None:
+        with open(path, "wb") as f:
+            f.write(self.serialize(stream))
+
     def array_info(self, array: int) -> Tuple[int, int]:
         nl, nn = ctypes.c_uint64(), ctypes.c_uint64()
         _check(lib().ckpt_tree_array_info(self.handle, array, ctypes.byref(nl), ctypes.byref(nn)),
@@ -228,8 +263,12 @@ class Tree:
 
 
 def tree_build(arrays: Union[torch.Tensor, Sequence[torch.Tensor]], chunk_bytes: int, eps: float,
-               stream=None) -> Tree:
-    """Steps 1-2: leaves (quantize + chained Murmur3F) and all levels, asynchronously."""
+               stream=None, hash_block: int = 16) -> Tree:
+    """Steps 1-2: leaves (quantize + chained Murmur3F) and all levels, asynchronously.
+
+    hash_block: bytes per chained Murmur3F call (16 = P:610; 0 = whole chunk; R23)."""
+    if hash_block != 16:
+        return tree_build_batch([arrays], chunk_bytes, eps, stream, hash_block)[0]
     ts = _as_list(arrays)
     code = _check_arrays(ts)
     pp, _k1 = _ptr_array(ts)
@@ -242,8 +281,8 @@ def tree_build(arrays: Union[torch.Tensor, Sequence[torch.Tensor]], chunk_bytes:
 
 
 def tree_build_batch(checkpoints: Sequence[Sequence[torch.Tensor]], chunk_bytes: int, eps: float,
-                     stream=None) -> List[Tree]:
-    """Several checkpoints' trees with one leaf-kernel launch (ckpt_tree_build_batch)."""
+                     stream=None, hash_block: int = 16) -> List[Tree]:
+    """Several checkpoints' trees with one leaf-kernel launch (ckpt_tree_build_batch[_ex])."""
     cks = [_as_list(c) for c in checkpoints]
     flat = [t for c in cks for t in c]
     code = _check_arrays(flat)
@@ -252,9 +291,10 @@ def tree_build_batch(checkpoints: Sequence[Sequence[torch.Tensor]], chunk_bytes:
     per = (ctypes.c_uint32 * len(cks))(*[len(c) for c in cks])
     outs = (ctypes.c_void_p * len(cks))()
     sp = _stream_ptr(stream)
-    _check(lib().ckpt_tree_build_batch(pp, pn, per, len(cks), code, chunk_bytes, float(eps), sp,
-                                       ctypes.cast(outs, ctypes.POINTER(ctypes.c_void_p))),
-           "ckpt_tree_build_batch")
+    _check(lib().ckpt_tree_build_batch_ex(pp, pn, per, len(cks), code, chunk_bytes, float(eps),
+                                          hash_block, sp,
+                                          ctypes.cast(outs, ctypes.POINTER(ctypes.c_void_p))),
+           "ckpt_tree_build_batch_ex")
     return [Tree(outs[k], cks[k], code, chunk_bytes, float(eps), sp) for k in range(len(cks))]
 
 
@@ -268,6 +308,56 @@ def tree_from_digests(digests: torch.Tensor, stream=None) -> Tree:
     _check(lib().ckpt_tree_from_digests(d.data_ptr(), d.shape[0], sp, ctypes.byref(out)),
            "ckpt_tree_from_digests")
     return Tree(out.value, [d], F32, 16, 0.0, sp)
+
+
+def tree_deserialize(data: bytes, stream=None) -> Tree:
+    """Load a serialised tree onto the current device (ckpt_tree_deserialize)."""
+    buf = ctypes.create_string_buffer(bytes(data), len(data))
+    out = ctypes.c_void_p()
+    sp = _stream_ptr(stream)
+    _check(lib().ckpt_tree_deserialize(ctypes.cast(buf, ctypes.c_void_p), len(data), sp,
+                                       ctypes.byref(out)), "ckpt_tree_deserialize")
+    t = Tree(out.value, [], F32, 0, 0.0, sp)
+    t.dtype, t.chunk_bytes, t.eps, _ = t.params()
+    return t
+
+
+def tree_load(path: str, stream=None) -> Tree:
+    with open(path, "rb") as f:
+        return tree_deserialize(f.read(), stream)
+
+
+def compare_saved(saved_a: bytes, arrays_a, arrays_b, chunks: torch.Tensor, idx: torch.Tensor,
+                  counts: torch.Tensor, stream=None) -> Tuple[Tree, Tree]:
+    """Compare live run B (device) with stored run A: A's tree from ``saved_a`` (serialised), A's
+    data as device tensors or pinned host tensors (only flagged chunks are read), ckpt_compare_saved.
+
+    Writes chunk ids, element ids and counts[0:2] (device) like compare_pair_async."""
+    la, lb = _as_list(arrays_a), _as_list(arrays_b)
+    if len(la) != len(lb) or any(x.numel() != y.numel() for x, y in zip(la, lb)):
+        raise ValueError("A and B must have the same arrays and lengths")
+    for t in la:
+        if not t.is_cuda and not t.is_pinned():
+            raise ValueError("host arrays of run A must be pinned (device-addressable)")
+        if not t.is_contiguous():
+            raise ValueError("arrays must be contiguous")
+    code = _check_arrays(lb)
+    if len(saved_a) >= 16 and int.from_bytes(bytes(saved_a[12:16]), "little") != code:
+        raise ValueError("run B's dtype differs from the stored tree's")
+    pa, _k1 = _ptr_array(la)
+    pb, _k2 = _ptr_array(lb)
+    pn, _k3 = _u64_array([t.numel() for t in lb])
+    buf = ctypes.create_string_buffer(bytes(saved_a), len(saved_a))
+    ta, tb = ctypes.c_void_p(), ctypes.c_void_p()
+    sp = _stream_ptr(stream)
+    _check(lib().ckpt_compare_saved(ctypes.cast(buf, ctypes.c_void_p), len(saved_a), pa, pb, pn,
+                                    len(lb), chunks.data_ptr(), chunks.numel(), idx.data_ptr(),
+                                    idx.numel(), counts.data_ptr(), sp, ctypes.byref(ta),
+                                    ctypes.byref(tb)), "ckpt_compare_saved")
+    TA = Tree(ta.value, la, F32, 0, 0.0, sp)
+    TA.dtype, TA.chunk_bytes, TA.eps, _ = TA.params()
+    TB = Tree(tb.value, lb, TA.dtype, TA.chunk_bytes, TA.eps, sp)
+    return TA, TB
 
 
 def tree_diff(ta: Tree, tb: Tree, cap: Optional[int] = None, stream=None) -> torch.Tensor:
@@ -449,7 +539,8 @@ def diff_verify_async(ta: Tree, tb: Tree, arrays_a, arrays_b, chunks: torch.Tens
 
 
 def compare_pair_async(arrays_a, arrays_b, chunk_bytes: int, eps: float, chunks: torch.Tensor,
-                       idx: torch.Tensor, counts: torch.Tensor, stream=None) -> Tuple[Tree, Tree]:
+                       idx: torch.Tensor, counts: torch.Tensor, stream=None,
+                       hash_block: int = 16) -> Tuple[Tree, Tree]:
     """Fused pair compare (ckpt_compare_pair_async): steps 1-4 for two checkpoints of identical
     shape with the leaf-digest comparison and the element marking inside the leaf kernel.
 
@@ -462,20 +553,11 @@ def compare_pair_async(arrays_a, arrays_b, chunk_bytes: int, eps: float, chunks:
     pa, _k1 = _ptr_array(la)
     pb, _k2 = _ptr_array(lb)
     pn, _k3 = _u64_array([t.numel() for t in la])
-    L = lib()
-    if not getattr(L, "_cp_typed", False):
-        vp, u64 = ctypes.c_void_p, ctypes.c_uint64
-        L.ckpt_compare_pair_async.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp),
-                                              ctypes.POINTER(u64), ctypes.c_uint32, ctypes.c_int,
-                                              ctypes.c_uint32, ctypes.c_double, vp, u64, vp, u64,
-                                              vp, vp, ctypes.POINTER(vp), ctypes.POINTER(vp)]
-        L.ckpt_compare_pair_async.restype = ctypes.c_int
-        L._cp_typed = True
     ta, tb = ctypes.c_void_p(), ctypes.c_void_p()
     sp = _stream_ptr(stream)
-    _check(L.ckpt_compare_pair_async(pa, pb, pn, len(la), code, chunk_bytes, float(eps),
-                                     chunks.data_ptr(), chunks.numel(), idx.data_ptr(), idx.numel(),
-                                     counts.data_ptr(), sp, ctypes.byref(ta), ctypes.byref(tb)),
-           "ckpt_compare_pair_async")
+    _check(lib().ckpt_compare_pair_ex(pa, pb, pn, len(la), code, chunk_bytes, float(eps), hash_block,
+                                      chunks.data_ptr(), chunks.numel(), idx.data_ptr(), idx.numel(),
+                                      counts.data_ptr(), sp, ctypes.byref(ta), ctypes.byref(tb)),
+           "ckpt_compare_pair_ex")
     return (Tree(ta.value, la, code, chunk_bytes, float(eps), sp),
             Tree(tb.value, lb, code, chunk_bytes, float(eps), sp))

@@ -226,6 +226,7 @@ struct ckpt_tree {
     ckpt_dtype dtype = CKPT_F32;
     uint32_t chunk_bytes = 0;
     double eps = 0.0;
+    uint32_t hash_block = 16;              // bytes per chained Murmur3F call, <= chunk_bytes (R23)
     bool from_digests = false;
     uint32_t n_arrays = 0;
     uint32_t n_levels = 0;                 // max height
@@ -343,10 +344,18 @@ static ckpt_status check_common(ckpt_dtype dtype, uint32_t chunk_bytes, double e
     return CKPT_OK;
 }
 
-template <int DT, bool RAW, int CB, bool PAIR>
+// Hash block size (R23): a positive multiple of 16, or 0 = the whole chunk;
+// sizes >= chunk_bytes are the whole chunk.  Returns the effective size.
+static ckpt_status norm_block(uint32_t hb, uint32_t C, uint32_t *out) {
+    if (hb % 16 != 0) return fail(CKPT_EINVAL, "hash_block must be a multiple of 16 (0 = whole chunk)");
+    *out = (hb == 0 || hb > C) ? C : hb;
+    return CKPT_OK;
+}
+
+template <int DT, bool RAW, int CB, bool PAIR, bool WIDE = false>
 static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
     const uint64_t tasks = P.n_tasks;
-    auto k = leaf_kernel<DT, RAW, CB, PAIR>;
+    auto k = leaf_kernel<DT, RAW, CB, PAIR, WIDE>;
     static std::atomic<int> cached_per_sm{0};
     int per_sm = cached_per_sm.load(std::memory_order_relaxed);
     if (per_sm == 0) {
@@ -368,6 +377,14 @@ static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
 template <int DT, bool RAW>
 static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms, bool pair) {
     const uint32_t C = P.chunk;
+    if (P.hb16 != 1) {   // wide hash blocks (R23): the bench chunk size specialised, others generic
+        if (pair) {
+            if (C == 4096) return launch_leaf_t<DT, RAW, 4096, true, true>(P, s, sms);
+            return launch_leaf_t<DT, RAW, 0, true, true>(P, s, sms);
+        }
+        if (C == 4096) return launch_leaf_t<DT, RAW, 4096, false, true>(P, s, sms);
+        return launch_leaf_t<DT, RAW, 0, false, true>(P, s, sms);
+    }
     if (pair) {   // fused pair mode: the bench chunk size specialised, others generic
         if constexpr (!RAW) {
             if (C == 4096) return launch_leaf_t<DT, RAW, 4096, true>(P, s, sms);
@@ -496,12 +513,13 @@ static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
 
 // One leaf-kernel launch over every array of every tree in `table`.
 static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t tasks,
-                                 ckpt_dtype dtype, double eps, uint32_t C, cudaStream_t s, int sms,
-                                 const PairParams *pair = nullptr,
+                                 ckpt_dtype dtype, double eps, uint32_t C, uint32_t hash_block,
+                                 cudaStream_t s, int sms, const PairParams *pair = nullptr,
                                  unsigned long long *ticket = nullptr) {
     LeafParams P;
     std::memset(&P, 0, sizeof(P));
     quant_params(eps, &P.q);
+    P.hb16 = hash_block / 16;
     if (pair) P.pr = *pair;
     P.ticket = ticket;
     P.n_arrays = (int)table.size();
@@ -587,11 +605,13 @@ static ckpt_status get_pair_ctr(int dev, cudaStream_t s, size_t n, unsigned int 
 static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
                                     const uint32_t *arrays_per_tree, uint32_t n_trees,
                                     ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
-                                    void *stream, ckpt_tree **out, const PairParams *pair) {
+                                    uint32_t hash_block, void *stream, ckpt_tree **out,
+                                    const PairParams *pair) {
     if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
     for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
     if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
+    CK_TRY(norm_block(hash_block, chunk_bytes, &hash_block));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
     uint64_t total_arrays = 0;
     for (uint32_t k = 0; k < n_trees; ++k) {
@@ -622,6 +642,7 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
         t->dtype = dtype;
         t->chunk_bytes = chunk_bytes;
         t->eps = eps;
+        t->hash_block = hash_block;
         t->n_elems.assign(n + a0, n + a0 + na);
         std::vector<uint64_t> leaves(na);
         for (uint32_t a = 0; a < na; ++a) leaves[a] = (n[a0 + a] * esz + chunk_bytes - 1) / chunk_bytes;
@@ -655,7 +676,8 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
         ticket += kLeafTicketSlot;
     }
     if (st == CKPT_OK)
-        st = launch_leaves(table, task, dtype, eps, chunk_bytes, s, di.sms, pair ? &pp : nullptr, ticket);
+        st = launch_leaves(table, task, dtype, eps, chunk_bytes, hash_block, s, di.sms,
+                           pair ? &pp : nullptr, ticket);
     if (st == CKPT_OK) {
         // K2 on the side stream, after the leaves; each tree records its own event
         cudaStream_t ss = nullptr;
@@ -684,8 +706,16 @@ extern "C" ckpt_status ckpt_tree_build_batch(const void *const *data, const uint
                                              const uint32_t *arrays_per_tree, uint32_t n_trees,
                                              ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
                                              void *stream, ckpt_tree **out) {
-    return build_batch_impl(data, n, arrays_per_tree, n_trees, dtype, chunk_bytes, eps, stream, out,
-                            nullptr);
+    return build_batch_impl(data, n, arrays_per_tree, n_trees, dtype, chunk_bytes, eps, 16, stream,
+                            out, nullptr);
+}
+
+extern "C" ckpt_status ckpt_tree_build_batch_ex(const void *const *data, const uint64_t *n,
+                                                const uint32_t *arrays_per_tree, uint32_t n_trees,
+                                                ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                                uint32_t hash_block, void *stream, ckpt_tree **out) {
+    return build_batch_impl(data, n, arrays_per_tree, n_trees, dtype, chunk_bytes, eps, hash_block,
+                            stream, out, nullptr);
 }
 
 extern "C" ckpt_status ckpt_tree_build_arrays(const void *const *data, const uint64_t *n,
@@ -761,8 +791,9 @@ static ckpt_status check_pair(const ckpt_tree *a, const ckpt_tree *b) {
         return fail(CKPT_EINVAL, "trees built from digests cannot be diffed");
     if (a->dtype != b->dtype || a->chunk_bytes != b->chunk_bytes ||
         std::memcmp(&a->eps, &b->eps, sizeof(double)) != 0 || a->n_arrays != b->n_arrays ||
-        a->n_elems != b->n_elems)
-        return fail(CKPT_EMISMATCH, "trees differ in dtype, chunk_bytes, eps or array shapes");
+        a->n_elems != b->n_elems || a->hash_block != b->hash_block)
+        return fail(CKPT_EMISMATCH,
+                    "trees differ in dtype, chunk_bytes, eps, hash_block or array shapes");
     if (a->device != b->device) return fail(CKPT_EMISMATCH, "trees live on different devices");
     return CKPT_OK;
 }
@@ -1081,12 +1112,12 @@ extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tr
 // fused pair compare: K1 in pair mode (digest compare and
 // element marking in-kernel), then the ordered chunk list and the element ids
 // ---------------------------------------------------------------------------
-extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void *const *b,
-                                               const uint64_t *n, uint32_t n_arrays,
-                                               ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
-                                               uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
-                                               uint64_t idx_cap, uint64_t *counts_dev, void *stream,
-                                               ckpt_tree **out_a, ckpt_tree **out_b) {
+extern "C" ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *const *b,
+                                            const uint64_t *n, uint32_t n_arrays, ckpt_dtype dtype,
+                                            uint32_t chunk_bytes, double eps, uint32_t hash_block,
+                                            uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                            uint64_t idx_cap, uint64_t *counts_dev, void *stream,
+                                            ckpt_tree **out_a, ckpt_tree **out_b) {
     if (out_a) *out_a = nullptr;
     if (out_b) *out_b = nullptr;
     if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
@@ -1116,7 +1147,8 @@ extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void 
     }
     const uint32_t apt[2] = {n_arrays, n_arrays};
     ckpt_tree *trees[2] = {nullptr, nullptr};
-    CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, stream, trees, &pp));
+    CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
+                            trees, &pp));
     ckpt_status st = launch_compact(1, nullptr, nullptr, pp.flags, L, chunks, chunks_cap, counts_dev, s,
                                     di.sms);
     if (st == CKPT_OK)
@@ -1130,6 +1162,16 @@ extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void 
     *out_a = trees[0];
     *out_b = trees[1];
     return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void *const *b,
+                                               const uint64_t *n, uint32_t n_arrays,
+                                               ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                               uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                               uint64_t idx_cap, uint64_t *counts_dev, void *stream,
+                                               ckpt_tree **out_a, ckpt_tree **out_b) {
+    return ckpt_compare_pair_ex(a, b, n, n_arrays, dtype, chunk_bytes, eps, 16, chunks, chunks_cap,
+                                idx, idx_cap, counts_dev, stream, out_a, out_b);
 }
 
 extern "C" ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b,
@@ -1303,6 +1345,156 @@ extern "C" ckpt_status ckpt_compare_host(const void *const *a, const void *const
 }
 
 // ---------------------------------------------------------------------------
+// tree persistence: the tree is created at capture time
+// and stored with the checkpoint; a later comparison loads it
+// instead of re-hashing that run
+// ---------------------------------------------------------------------------
+static const char kTreeMagic[8] = {'C', 'K', 'P', 'T', 'T', 'R', 'E', '1'};
+constexpr uint32_t kTreeFormat = 1;
+constexpr size_t kTreeHdr = 40;   // fixed part before n_elems[]
+
+static size_t ser_prefix(uint32_t na) { return kTreeHdr + (size_t)na * 8 + 8 + 16; }
+
+extern "C" ckpt_status ckpt_tree_serialized_size(const ckpt_tree *t, uint64_t *bytes) {
+    if (!t || !bytes) return fail(CKPT_EINVAL, "NULL argument");
+    if (t->from_digests) return fail(CKPT_EINVAL, "trees built from digests are not serialisable");
+    *bytes = ser_prefix(t->n_arrays) + (t->array_nodes + t->top_nodes) * 16;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_serialize(const ckpt_tree *t, void *dst, uint64_t cap,
+                                           uint64_t *written, void *stream) {
+    uint64_t need = 0;
+    CK_TRY(ckpt_tree_serialized_size(t, &need));
+    if (!dst || !written) return fail(CKPT_EINVAL, "NULL argument");
+    *written = need;
+    if (cap < need) return fail(CKPT_EINVAL, "destination smaller than ckpt_tree_serialized_size");
+    uint8_t *o = (uint8_t *)dst;
+    std::memset(o, 0, ser_prefix(t->n_arrays));
+    std::memcpy(o, kTreeMagic, 8);
+    const uint32_t hdr32[5] = {kTreeFormat, (uint32_t)t->dtype, t->chunk_bytes, t->hash_block, 0};
+    std::memcpy(o + 8, hdr32, 16);
+    std::memcpy(o + 24, &t->eps, 8);
+    std::memcpy(o + 32, &t->n_arrays, 4);
+    std::memcpy(o + kTreeHdr, t->n_elems.data(), (size_t)t->n_arrays * 8);
+    const uint64_t nodes = t->array_nodes + t->top_nodes;
+    std::memcpy(o + kTreeHdr + (size_t)t->n_arrays * 8, &nodes, 8);
+    cudaStream_t s = (cudaStream_t)stream;
+    CK_TRY(wait_levels(t, s));
+    uint8_t *body = o + ser_prefix(t->n_arrays);
+    CK_CUDA(cudaMemcpyAsync(body, t->nodes, nodes * 16, cudaMemcpyDeviceToHost, s));
+    CK_CUDA(cudaStreamSynchronize(s));
+    std::memcpy(o + ser_prefix(t->n_arrays) - 16, body + (nodes - 1) * 16, 16);   // the root
+    return CKPT_OK;
+}
+
+// Host-only parse of a serialised tree (no device work): header checks and
+// the layout the body must have.
+static ckpt_status parse_tree(const uint8_t *in, uint64_t bytes, ckpt_tree *t) {
+    if (bytes < kTreeHdr || std::memcmp(in, kTreeMagic, 8) != 0)
+        return fail(CKPT_EINVAL, "not a serialised ckpt tree (bad magic)");
+    uint32_t hdr32[5];
+    std::memcpy(hdr32, in + 8, 16);
+    if (hdr32[0] != kTreeFormat) return fail(CKPT_EINVAL, "unsupported tree format version");
+    if (hdr32[1] != CKPT_F32 && hdr32[1] != CKPT_F64) return fail(CKPT_EINVAL, "bad dtype in tree header");
+    t->dtype = (ckpt_dtype)hdr32[1];
+    t->chunk_bytes = hdr32[2];
+    t->hash_block = hdr32[3];
+    std::memcpy(&t->eps, in + 24, 8);
+    CK_TRY(check_common(t->dtype, t->chunk_bytes, t->eps));
+    if (t->hash_block == 0 || t->hash_block % 16 || t->hash_block > t->chunk_bytes)
+        return fail(CKPT_EINVAL, "bad hash_block in tree header");
+    uint32_t na = 0;
+    std::memcpy(&na, in + 32, 4);
+    if (na == 0 || na >= (1u << 20)) return fail(CKPT_EINVAL, "bad array count in tree header");
+    if (bytes < ser_prefix(na)) return fail(CKPT_EINVAL, "truncated tree header");
+    t->n_elems.resize(na);
+    std::memcpy(t->n_elems.data(), in + kTreeHdr, (size_t)na * 8);
+    const uint64_t esz = t->dtype == CKPT_F32 ? 4 : 8;
+    std::vector<uint64_t> leaves(na);
+    for (uint32_t a = 0; a < na; ++a) {
+        if (t->n_elems[a] == 0 || t->n_elems[a] > (1ull << 50)) return fail(CKPT_EINVAL, "bad array length");
+        leaves[a] = (t->n_elems[a] * esz + t->chunk_bytes - 1) / t->chunk_bytes;
+    }
+    layout(t, leaves);
+    uint64_t nodes = 0;
+    std::memcpy(&nodes, in + kTreeHdr + (size_t)na * 8, 8);
+    if (nodes != t->array_nodes + t->top_nodes) return fail(CKPT_EINVAL, "node count does not match the header");
+    if (bytes != ser_prefix(na) + nodes * 16) return fail(CKPT_EINVAL, "serialised tree has the wrong size");
+    if (std::memcmp(in + ser_prefix(na) - 16, in + ser_prefix(na) + (nodes - 1) * 16, 16) != 0)
+        return fail(CKPT_EINVAL, "stored root does not match the last node");
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_deserialize(const void *src, uint64_t bytes, void *stream,
+                                             ckpt_tree **out) {
+    if (!out) return fail(CKPT_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!src) return fail(CKPT_EINVAL, "src is NULL");
+    ckpt_tree tmp;
+    CK_TRY(parse_tree((const uint8_t *)src, bytes, &tmp));      // no device work before this
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    cudaStream_t s = (cudaStream_t)stream;
+    ckpt_tree *t = new ckpt_tree(tmp);
+    t->device = dev;
+    t->stream = s;
+    t->levels_done = nullptr;
+    ckpt_status st = prepare_tree(t, s);
+    const uint64_t nodes = t->array_nodes + t->top_nodes;
+    if (st == CKPT_OK)
+        st = g_ring.copy(t->meta, t->meta_host.data(), t->meta_host.size() * 8, s);
+    if (st == CKPT_OK &&
+        cudaMemcpyAsync(t->nodes, (const uint8_t *)src + ser_prefix(t->n_arrays), nodes * 16,
+                        cudaMemcpyHostToDevice, s) != cudaSuccess)
+        st = fail(CKPT_ECUDA, "tree upload");
+    // the caller's buffer may be pageable and reused at once: finish the upload
+    if (st == CKPT_OK && cudaStreamSynchronize(s) != cudaSuccess) st = fail(CKPT_ECUDA, "sync");
+    if (st != CKPT_OK) { ckpt_tree_free_on(t, stream); return st; }
+    *out = t;
+    return CKPT_OK;
+}
+
+// Compare a live checkpoint (run B, device) with a stored run A: A's tree is
+// loaded from its serialised form instead of re-hashing A, B's tree is built
+// with A's parameters, the trees are diffed and only the flagged chunks of A
+// are read (a_data may be host memory the device can address: pinned /
+// registered host memory through UVA, so the verify kernel reads just those
+// chunks over the host link, the two-stage I/O of P:568-578).
+extern "C" ckpt_status ckpt_compare_saved(const void *saved_a, uint64_t saved_bytes,
+                                          const void *const *a_data, const void *const *b,
+                                          const uint64_t *n, uint32_t n_arrays, uint64_t *chunks,
+                                          uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                                          uint64_t *counts_dev, void *stream, ckpt_tree **out_a,
+                                          ckpt_tree **out_b) {
+    if (out_a) *out_a = nullptr;
+    if (out_b) *out_b = nullptr;
+    if (!out_a || !out_b || !a_data || !b || !n || !counts_dev || (!chunks && chunks_cap) ||
+        (!idx && idx_cap))
+        return fail(CKPT_EINVAL, "NULL argument");
+    ckpt_tree hdr;
+    CK_TRY(parse_tree((const uint8_t *)saved_a, saved_bytes, &hdr));
+    if (hdr.n_arrays != n_arrays || !std::equal(hdr.n_elems.begin(), hdr.n_elems.end(), n))
+        return fail(CKPT_EMISMATCH, "live checkpoint shape differs from the stored tree");
+    ckpt_tree *ta = nullptr, *tb = nullptr;
+    CK_TRY(ckpt_tree_deserialize(saved_a, saved_bytes, stream, &ta));
+    ckpt_status st = build_batch_impl(b, n, &n_arrays, 1, ta->dtype, ta->chunk_bytes, ta->eps,
+                                      ta->hash_block, stream, &tb, nullptr);
+    if (st == CKPT_OK)
+        st = ckpt_diff_verify_async(ta, tb, a_data, b, chunks, chunks_cap, idx, idx_cap, counts_dev,
+                                    stream);
+    if (st != CKPT_OK) {
+        ckpt_tree_free_on(ta, stream);
+        ckpt_tree_free_on(tb, stream);
+        return st;
+    }
+    *out_a = ta;
+    *out_b = tb;
+    return CKPT_OK;
+}
+
+// ---------------------------------------------------------------------------
 // accessors
 // ---------------------------------------------------------------------------
 extern "C" ckpt_status ckpt_tree_wait(const ckpt_tree *t, void *stream) {
@@ -1317,6 +1509,17 @@ extern "C" ckpt_status ckpt_tree_info(const ckpt_tree *t, uint32_t *n_arrays, ui
     if (n_leaves) *n_leaves = t->total_leaves;
     if (n_levels) *n_levels = t->n_levels;
     if (n_nodes) *n_nodes = t->array_nodes;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_tree_params(const ckpt_tree *t, ckpt_dtype *dtype, uint32_t *chunk_bytes,
+                                        double *eps, uint32_t *hash_block) {
+    if (!t) return fail(CKPT_EINVAL, "NULL tree");
+    if (t->from_digests) return fail(CKPT_EINVAL, "tree built from digests has no hashing parameters");
+    if (dtype) *dtype = t->dtype;
+    if (chunk_bytes) *chunk_bytes = t->chunk_bytes;
+    if (eps) *eps = t->eps;
+    if (hash_block) *hash_block = t->hash_block;
     return CKPT_OK;
 }
 

@@ -75,10 +75,10 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
     return v;
 }
 
-// Hash one 16-byte block (raw bits in v), exact words for every input:
-// per-element fast/slow selection (generic path: ragged tasks and retries).
+// Exact hashed words of one 16-byte piece (raw bits in v): per-element
+// fast/slow selection (generic path: ragged tasks and retries).
 template <int DT, bool RAW>
-__device__ __forceinline__ void chain_block_exact(U64p &h1, U64p &h2, uint4 v, const QuantParams &q) {
+__device__ __forceinline__ uint4 words_exact(uint4 v, const QuantParams &q) {
     uint4 w;
     if (RAW) {
         w = v;
@@ -90,6 +90,13 @@ __device__ __forceinline__ void chain_block_exact(U64p &h1, U64p &h2, uint4 v, c
         const uint64_t k1 = word_f64(__hiloint2double((int)v.w, (int)v.z), q);
         w = make_uint4((uint32_t)k0, (uint32_t)(k0 >> 32), (uint32_t)k1, (uint32_t)(k1 >> 32));
     }
+    return w;
+}
+
+// Hash one 16-byte block with exact words (canonical 16-byte hash blocks).
+template <int DT, bool RAW>
+__device__ __forceinline__ void chain_block_exact(U64p &h1, U64p &h2, uint4 v, const QuantParams &q) {
+    const uint4 w = words_exact<DT, RAW>(v, q);
     mm3p_block16(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
 }
 
@@ -97,8 +104,7 @@ __device__ __forceinline__ void chain_block_exact(U64p &h1, U64p &h2, uint4 v, c
 // "every element so far was inside the fast range" (FSETP ... AND chains, no
 // branch); a task whose warp saw any out-of-range element is redone exactly.
 template <int DT, bool RAW>
-__device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, const QuantParams &q,
-                                                 bool &ok, float &mx) {
+__device__ __forceinline__ uint4 words_fast(uint4 v, const QuantParams &q, bool &ok, float &mx) {
     uint4 w;
     if (RAW) {
         w = v;
@@ -135,9 +141,28 @@ __device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, co
         w.z = (uint32_t)__double2loint(t1);
         w.w = (uint32_t)__double2hiint(t1) - 0x43380000u;
     }
+    return w;
+}
+
+template <int DT, bool RAW>
+__device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, const QuantParams &q,
+                                                 bool &ok, float &mx) {
+    const uint4 w = words_fast<DT, RAW>(v, q, ok, mx);
     mm3p_block16(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
 }
 
+// Wide hash blocks (reading R23): a block of B = 16*hb16 bytes is
+// one Murmur3F call, i.e. a body step per 16-byte piece and one finalisation
+// (len = B) when the block is complete.  `left` counts the pieces still
+// missing from the current block (uniform across the warp: no divergence).
+__device__ __forceinline__ void wide_piece(U64p &h1, U64p &h2, uint4 w, const QuantParams &q,
+                                           uint32_t &left, uint32_t hb16) {
+    mm3p_body(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
+    if (--left == 0u) {
+        mm3p_final(h1, h2, hb16 * 16u);
+        left = hb16;
+    }
+}
 // Short final block of `len` bytes (len in {4,8,12} for F32, 8 for F64),
 // read straight from global memory (only the array's last chunk has one).
 template <int DT, bool RAW>
@@ -157,6 +182,41 @@ __device__ __noinline__ void chain_tail(uint64_t &h1, uint64_t &h2, const uint8_
     }
     mm3_block_tail(h1, h2, (uint64_t)w[0] | ((uint64_t)w[1] << 32),
                    (uint64_t)w[2] | ((uint64_t)w[3] << 32), len);
+}
+
+// Wide-block variant of the chunk end: the <16-byte tail (if any) is mixed
+// into the open block, then the open block (blen bytes, pieces + tail) is
+// finalised with its own length, as Murmur3F does for a short key.
+template <int DT, bool RAW>
+__device__ __noinline__ void wide_end(uint64_t &h1, uint64_t &h2, const uint8_t *p, uint32_t tail,
+                                      uint32_t blen, const QuantParams &q) {
+    if (tail) {
+        uint32_t w[4] = {0u, 0u, 0u, 0u};
+        if (DT == 0) {
+            for (uint32_t e = 0; e < tail / 4; ++e) {
+                const uint32_t bits = reinterpret_cast<const uint32_t *>(p)[e];
+                w[e] = RAW ? bits : word_f32(__uint_as_float(bits), q);
+            }
+        } else {
+            const uint64_t bits = reinterpret_cast<const uint64_t *>(p)[0];
+            const uint64_t k = RAW ? bits : word_f64(__longlong_as_double((long long)bits), q);
+            w[0] = (uint32_t)k;
+            w[1] = (uint32_t)(k >> 32);
+        }
+        uint64_t k1 = (uint64_t)w[0] | ((uint64_t)w[1] << 32);
+        uint64_t k2 = (uint64_t)w[2] | ((uint64_t)w[3] << 32);
+        if (tail > 8) {
+            k2 *= kC2;
+            k2 = rotl64(k2, 33);
+            k2 *= kC1;
+            h2 ^= k2;
+        }
+        k1 *= kC1;
+        k1 = rotl64(k1, 31);
+        k1 *= kC2;
+        h1 ^= k1;
+    }
+    if (blen) mm3_final(h1, h2, blen);
 }
 
 constexpr int kLeafInline = 16;
@@ -188,6 +248,9 @@ struct LeafParams {
     // non-null: warps draw tasks in order from this counter (0 at launch; the
     // final draw resets it), so a warp held up by marking takes fewer tasks
     unsigned long long *ticket;
+    // hash block in 16-byte pieces (WIDE kernels only): B = 16*hb16 <= C bytes;
+    // B = C is one Murmur3F call per chunk
+    uint32_t hb16;
 };
 
 __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, uint64_t task) {
@@ -203,7 +266,9 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
 // A task is kRows = 32*kCh consecutive chunks of one array; lane l owns the
 // chains of rows l, l+32, ... (kCh independent chains per lane give the
 // scheduler two interleavable instruction streams).
-template <int DT, bool RAW, int CB, bool PAIR>
+// WIDE: hash blocks of P.hb16 pieces (reading R23) instead of the paper's
+// default 16-byte blocks.
+template <int DT, bool RAW, int CB, bool PAIR, bool WIDE = false>
 __global__ void __launch_bounds__(kLeafWarps * 32, CKPT_LEAF_MINB)
 leaf_kernel(const __grid_constant__ LeafParams P) {
     pdl_enter();
@@ -249,7 +314,9 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
         const int a = find_array(arrays, n_arrays, task);
         const LeafArray A = arrays[a];
         const uint64_t c0 = (task - A.task_begin) * kRows;   // first local chunk of the task
-        const bool full_task = (C % kSeg == 0) && (c0 + kRows) <= A.n_full;
+        // wide blocks take the fast path only when they tile the chunk exactly
+        const bool full_task = (C % kSeg == 0) && (c0 + kRows) <= A.n_full &&
+                               (!WIDE || (C / 16) % P.hb16 == 0);
         U64p h1[kCh], h2[kCh];
 #pragma unroll
         for (int j = 0; j < kCh; ++j) { h1[j] = U64p{0u, 0u}; h2[j] = U64p{0u, 0u}; }
@@ -267,6 +334,8 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             };
             bool ok = true;
             float mx = 0.0f;
+            const uint32_t hb16 = WIDE ? P.hb16 : 1u;
+            uint32_t left = hb16;
 #pragma unroll
             for (int s = 0; s < kStages - 1; ++s) {
                 if ((uint32_t)s < n_stages) issue(src + s * kSeg, s * kSlotBytes);
@@ -285,10 +354,16 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
                 const uint32_t row = my_row + slot;
 #pragma unroll
                 for (int b = 0; b < kPiecesPerChunk; ++b) {
+                    if constexpr (WIDE) {
+                        static_assert(!WIDE || kCh == 1, "wide blocks assume one chain per lane");
+                        const uint4 w = words_fast<DT, RAW>(lds128(row + b * 16), q, ok, mx);
+                        wide_piece(h1[0], h2[0], w, q, left, hb16);
+                    } else {
 #pragma unroll
-                    for (int j = 0; j < kCh; ++j)
-                        chain_block_fast<DT, RAW>(h1[j], h2[j], lds128(row + j * 32 * kPitch + b * 16),
-                                                  q, ok, mx);
+                        for (int j = 0; j < kCh; ++j)
+                            chain_block_fast<DT, RAW>(h1[j], h2[j], lds128(row + j * 32 * kPitch + b * 16),
+                                                      q, ok, mx);
+                    }
                 }
                 __syncwarp();
                 slot = (slot == (kStages - 1) * kSlotBytes) ? 0u : slot + kSlotBytes;
@@ -334,6 +409,9 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
                     cp_async_commit();
                 }
                 const uint64_t full_blocks = my_len / 16;
+                // wide blocks: bytes in the open block of B = bbytes
+                const uint32_t bbytes = WIDE ? P.hb16 * 16u : 16u;
+                uint32_t blen = 0;
                 for (uint32_t s = 0; s < n_stages; ++s) {
                     if (s + kStages - 1 < n_stages) issue(s + kStages - 1);
                     cp_async_commit();
@@ -343,17 +421,29 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
 #pragma unroll
                     for (int b = 0; b < kPiecesPerChunk; ++b) {
                         const uint64_t blk = (uint64_t)s * kPiecesPerChunk + b;
-                        if (blk < full_blocks)
-                            chain_block_exact<DT, RAW>(e1, e2, lds128(row + b * 16), q);
+                        if (blk < full_blocks) {
+                            if constexpr (WIDE) {
+                                const uint4 w = words_exact<DT, RAW>(lds128(row + b * 16), q);
+                                mm3p_body(e1, e2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
+                                blen += 16u;
+                                if (blen == bbytes) { mm3p_final(e1, e2, bbytes); blen = 0u; }
+                            } else {
+                                chain_block_exact<DT, RAW>(e1, e2, lds128(row + b * 16), q);
+                            }
+                        }
                     }
                     __syncwarp();
                 }
                 cp_async_wait<0>();
                 __syncwarp();
                 const uint32_t tail = (uint32_t)(my_len & 15);
-                if (tail) {
+                if (WIDE ? (tail | blen) != 0u : tail != 0u) {
                     uint64_t t1 = ((uint64_t)e1.hi << 32) | e1.lo, t2 = ((uint64_t)e2.hi << 32) | e2.lo;
-                    chain_tail<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail, q);
+                    if constexpr (WIDE)
+                        wide_end<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail,
+                                          blen + tail, q);
+                    else
+                        chain_tail<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail, q);
                     e1 = U64p{(uint32_t)t1, (uint32_t)(t1 >> 32)};
                     e2 = U64p{(uint32_t)t2, (uint32_t)(t2 >> 32)};
                 }

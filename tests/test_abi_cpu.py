@@ -57,3 +57,59 @@ def test_product_package_does_not_import_oracle():
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "ckpt_oracle" not in src and "liboracle" not in src, f
+
+
+# ------------------------------------------------ tree persistence (host) --
+# ckpt_tree_deserialize validates the header on the host before any device
+# work, so malformed buffers are rejected here without a GPU.
+
+def _deser(libckpt, buf: bytes) -> int:
+    libckpt.ckpt_tree_deserialize.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p,
+                                              ctypes.POINTER(ctypes.c_void_p)]
+    libckpt.ckpt_tree_deserialize.restype = ctypes.c_int
+    b = ctypes.create_string_buffer(buf, len(buf))
+    out = ctypes.c_void_p(1)
+    st = libckpt.ckpt_tree_deserialize(ctypes.cast(b, ctypes.c_void_p), len(buf), None,
+                                       ctypes.byref(out))
+    assert not out.value
+    return st
+
+
+def _oracle_buf():
+    import numpy as np
+    import oracle
+    from tests.treefmt import oracle_tree_bytes
+    rng = np.random.default_rng(3)
+    arrays = [rng.uniform(-1, 1, n).astype(np.float32) for n in (1000, 3000, 17)]
+    ck = oracle.build_checkpoint(arrays, 256, 1e-4)
+    return oracle_tree_bytes(ck, [a.size for a in arrays], 0, 256, 1e-4)
+
+
+def test_deserialize_rejects_malformed_buffers_on_host(libckpt):
+    import struct
+    good = _oracle_buf()
+    EINVAL = -1
+    assert _deser(libckpt, b"") == EINVAL
+    assert _deser(libckpt, b"NOTATREE" + good[8:]) == EINVAL            # magic
+    assert _deser(libckpt, good[:8] + struct.pack("<I", 2) + good[12:]) == EINVAL   # version
+    assert _deser(libckpt, good[:-16]) == EINVAL                           # truncated body
+    assert _deser(libckpt, good + b"\0" * 16) == EINVAL                    # trailing bytes
+    bad_root = bytearray(good)
+    hdr_end = 40 + 3 * 8 + 8
+    bad_root[hdr_end] ^= 1                                                 # stored root != last node
+    assert _deser(libckpt, bytes(bad_root)) == EINVAL
+    bad_hb = bytearray(good)
+    bad_hb[20:24] = struct.pack("<I", 24)                                  # hash_block % 16
+    assert _deser(libckpt, bytes(bad_hb)) == EINVAL
+    bad_n = bytearray(good)
+    bad_n[40:48] = struct.pack("<Q", 2000)                                 # layout != node count
+    assert _deser(libckpt, bytes(bad_n)) == EINVAL
+
+
+def test_oracle_written_tree_passes_host_validation(libckpt):
+    # a well-formed buffer gets past the header checks: without a GPU the first
+    # device call fails (CKPT_ECUDA), never CKPT_EINVAL
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present: covered by the GPU persistence tests")
+    assert _deser(libckpt, _oracle_buf()) == -4

@@ -498,3 +498,159 @@ def test_compare_pair_identical_and_truncated():
     assert np.array_equal(np_of(idx), ref[:64])
     with pytest.raises(ValueError):
         ck.compare_pair_async(a, [b[0]], 4096, 1e-6, chunks, idx, counts)
+
+
+# ------------------------------------------- hash block size variant (R23) --
+# "the block size is variable and can be adjusted": every leaf,
+# tree node, chunk list and element list equals the oracle at that block size.
+
+HB_CASES = [
+    # (n, dtype, chunk, eps, hash_block)
+    (100_003, torch.float32, 4096, 1e-6, 0),      # whole chunk, ragged last chunk + tail
+    ((1 << 18) + 3, torch.float32, 4096, 1e-5, 64),
+    (70_001, torch.float32, 4096, 1e-5, 1024),
+    (50_001, torch.float32, 4096, 1e-5, 48),      # does not divide C: exact path, short last block
+    (4097, torch.float32, 512, 1e-5, 0),          # runtime chunk size, whole chunk
+    (9_999, torch.float32, 48, 1e-4, 32),
+    (123_457, torch.float64, 1024, 1e-8, 0),
+    (123_457, torch.float64, 4096, 1e-8, 256),
+    (10_001, torch.float32, 4096, 0.0, 0),        # raw-bit mode, whole chunk
+    (10_001, torch.float64, 160, 0.0, 32),
+]
+
+
+@pytest.mark.parametrize("n,dtype,chunk,eps,hb", HB_CASES)
+def test_hash_block_tree_bit_exact(n, dtype, chunk, eps, hb):
+    a = _data(n, dtype, n + chunk + hb)
+    t = ck.tree_build(a, chunk, eps, hash_block=hb)
+    got = gpu_tree_nodes(t)
+    lv = oracle.leaves(np_of(a), chunk, eps, threads=8, hash_block=hb)
+    ref = oracle.levels(lv)
+    bad = np.nonzero(np.any(got != ref, axis=1))[0]
+    assert bad.size == 0, f"{bad.size} nodes differ, first {bad[:5]}"
+    assert t.params()[3] == (chunk if hb == 0 or hb > chunk else hb)
+
+
+def test_hash_block_special_values_take_the_exact_retry():
+    a = synth.uniform(77, 1 << 16, "cuda") * 2.0 - 1.0
+    a[5000] = float("nan"); a[20000] = float("inf"); a[40000] = 1e30
+    for hb in (0, 64):
+        got = gpu_tree_nodes(ck.tree_build(a, 4096, 1e-6, hash_block=hb))
+        ref = oracle.levels(oracle.leaves(np_of(a), 4096, 1e-6, hash_block=hb))
+        assert np.array_equal(got, ref), hb
+
+
+@pytest.mark.parametrize("hb", [0, 64, 1024])
+@pytest.mark.parametrize("name,make", _pair_cases()[:4], ids=[c[0] for c in _pair_cases()[:4]])
+def test_compare_pair_hash_block_matches_oracle(name, make, hb):
+    pair = make()
+    eps, chunk = pair.eps, 4096
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    L = sum(-(-t.numel() * t.element_size() // chunk) for t in pair.a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(sum(t.numel() for t in pair.a), dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(pair.a, pair.b, chunk, eps, chunks, idx, counts, hash_block=hb)
+    TA.wait(); TB.wait()
+    torch.cuda.synchronize()
+    A = oracle.build_checkpoint(an, chunk, eps, threads=8, hash_block=hb)
+    B = oracle.build_checkpoint(bn, chunk, eps, threads=8, hash_block=hb)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, chunk, ref_chunks, eps, A)
+    nc, nd = counts.tolist()
+    assert np.array_equal(np_of(chunks[:nc]), ref_chunks)
+    assert np.array_equal(np_of(idx[:nd]), ref_idx)
+    for k in range(len(an)):
+        assert np.array_equal(gpu_tree_nodes(TA, k), A.trees[k]), k
+    assert TA.root() == A.root and TB.root() == B.root
+    # same flagged chunks as the paper's default 16-byte blocks (barring collisions)
+    A16 = oracle.build_checkpoint(an, chunk, eps, threads=8)
+    B16 = oracle.build_checkpoint(bn, chunk, eps, threads=8)
+    assert np.array_equal(ref_chunks, oracle.diff_checkpoint(A16, B16))
+
+
+def test_hash_block_mismatch_and_invalid():
+    a = synth.uniform(5, 10_000, "cuda")
+    t16 = ck.tree_build(a, 4096, 1e-5)
+    t0 = ck.tree_build(a, 4096, 1e-5, hash_block=0)
+    t4k = ck.tree_build(a, 4096, 1e-5, hash_block=8192)       # >= C: the whole chunk too
+    assert t0.root() == t4k.root() != t16.root()
+    assert ck.tree_diff(t0, t4k).numel() == 0
+    with pytest.raises(ck.CkptError) as e:
+        ck.tree_diff(t16, t0)
+    assert e.value.status == ck.EMISMATCH
+    with pytest.raises(ck.CkptError) as e:
+        ck.tree_build(a, 4096, 1e-5, hash_block=24)
+    assert e.value.status == ck.EINVAL
+
+
+# --------------------------------------------------- tree persistence ------
+
+def test_serialize_matches_documented_format_and_roundtrips():
+    from tests.treefmt import oracle_tree_bytes
+    pair = synth.c2_pair(n_particles=(1 << 15) + 9, seed=61, device="cuda")
+    an = [np_of(t) for t in pair.a]
+    for hb in (16, 0):
+        t = ck.tree_build(pair.a, 4096, pair.eps, hash_block=hb)
+        blob = t.serialize()
+        A = oracle.build_checkpoint(an, 4096, pair.eps, hash_block=hb)
+        ref = oracle_tree_bytes(A, [x.size for x in an], 0, 4096, pair.eps, 4096 if hb == 0 else hb)
+        assert blob == ref                                  # byte-exact against the oracle's tree
+        t2 = ck.tree_deserialize(blob)
+        assert t2.root() == t.root() == A.root
+        assert t2.params() == t.params()
+        for k in range(len(an)):
+            assert np.array_equal(gpu_tree_nodes(t2, k), A.trees[k])
+        assert t2.serialize() == blob
+        assert ck.tree_diff(t, t2).numel() == 0
+
+
+def test_oracle_written_tree_diffs_against_live_tree():
+    # a tree written by the oracle (documented format) loads and diffs like a GPU-built one
+    from tests.treefmt import oracle_tree_bytes
+    pair = synth.c5_pair(n_ranks=1, n_particles=1 << 16, seed=62, device="cuda")
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    A = oracle.build_checkpoint(an, 4096, pair.eps)
+    B = oracle.build_checkpoint(bn, 4096, pair.eps)
+    ta = ck.tree_deserialize(oracle_tree_bytes(A, [x.size for x in an], 0, 4096, pair.eps))
+    tb = ck.tree_build(pair.b, 4096, pair.eps)
+    ref = oracle.diff_checkpoint(A, B)
+    assert np.array_equal(np_of(ck.tree_diff(ta, tb)), ref)
+    for T in (1, 100):                                      # mid-level BFS over a loaded tree
+        chunks = torch.empty(ta.n_leaves, dtype=torch.int64, device="cuda")
+        cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+        ck.tree_diff_async(ta, tb, chunks, cnt, T=T)
+        assert np.array_equal(np_of(chunks[: int(cnt.item())]), ref), T
+
+
+@pytest.mark.parametrize("host_a", [False, True])
+def test_compare_saved_matches_oracle(host_a, tmp_path):
+    pair = synth.c2_pair(n_particles=(1 << 17) + 5, seed=63, device="cuda")
+    eps, C = pair.eps, 4096
+    path = str(tmp_path / "runA.ckpttree")
+    ck.tree_build(pair.a, C, eps).save(path)
+    saved = open(path, "rb").read()
+    a_data = [t.cpu().pin_memory() for t in pair.a] if host_a else pair.a
+    L = sum(-(-t.numel() * 4 // C) for t in pair.a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(sum(t.numel() for t in pair.a), dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_saved(saved, a_data, pair.b, chunks, idx, counts)
+    torch.cuda.synchronize()
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    A = oracle.build_checkpoint(an, C, eps, threads=8)
+    B = oracle.build_checkpoint(bn, C, eps, threads=8)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, C, ref_chunks, eps, A)
+    nc, nd = counts.tolist()
+    assert nc > 0 and nd > 0
+    assert np.array_equal(np_of(chunks[:nc]), ref_chunks)
+    assert np.array_equal(np_of(idx[:nd]), ref_idx)
+    assert TA.root() == A.root and TB.root() == B.root
+    # shape mismatch with the stored tree
+    with pytest.raises(ck.CkptError) as e:
+        ck.compare_saved(saved, [t[:-4] for t in pair.a], [t[:-4] for t in pair.b], chunks, idx, counts)
+    assert e.value.status == ck.EMISMATCH

@@ -53,6 +53,70 @@ def test_two_block_chain_seeds_with_full_digest():
     assert leaf == h1.to_bytes(8, "little") + h2.to_bytes(8, "little")
 
 
+# ------------------------------------------- hash block size (R23) ----
+# "the block size is variable and can be adjusted": the chain runs
+# over blocks of `hash_block` bytes; 16 is the paper's default, 0 the
+# whole chunk in one call.
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+@pytest.mark.parametrize("eps", [1e-5, 0.0])
+@pytest.mark.parametrize("n,chunk,blk", [(7, 32, 32), (100, 48, 32), (257, 128, 64),
+                                         (1000, 512, 128), (1000, 512, 0), (33, 64, 48),
+                                         (300, 256, 1024)])
+def test_hash_block_leaves_match_py_ref(dt, eps, n, chunk, blk):
+    rng = np.random.default_rng(n * 7 + blk)
+    a = rand_arr(rng, n, dt)
+    got = oracle.leaves(a, chunk, eps, hash_block=blk)
+    ref = py_ref.leaves([float(v) for v in a], dt == np.float32, chunk, eps, blk)
+    assert [bytes(r) for r in got] == ref
+
+
+def test_hash_block_16_is_the_default_chain():
+    rng = np.random.default_rng(5)
+    a = rng.uniform(-1, 1, 999).astype(np.float32)
+    assert np.array_equal(oracle.leaves(a, 256, 1e-5), oracle.leaves(a, 256, 1e-5, hash_block=16))
+
+
+@pytest.mark.parametrize("chunk", [16, 64, 4096])
+def test_whole_chunk_block_is_one_standard_murmur3f_call(chunk):
+    # block = chunk: the leaf is SMHasher MurmurHash3_x64_128(words of the chunk, seed 0),
+    # computed here by the independent pure-Python implementation pinned to 0x6384BA69
+    rng = np.random.default_rng(chunk)
+    a = rng.uniform(-1, 1, 3 * chunk // 4 + 1).astype(np.float32)   # ragged last chunk
+    got = oracle.leaves(a, chunk, 1e-4, hash_block=0)
+    assert np.array_equal(got, oracle.leaves(a, chunk, 1e-4, hash_block=chunk))
+    per = chunk // 4
+    for c in range(got.shape[0]):
+        w = py_ref.words([float(v) for v in a[c * per:(c + 1) * per]], True, 1e-4)
+        assert got[c].tobytes() == py_ref.murmur3f(w, 0)
+
+
+def test_hash_block_larger_than_chunk_is_whole_chunk():
+    rng = np.random.default_rng(6)
+    a = rng.normal(size=77)
+    assert np.array_equal(oracle.leaves(a, 64, 1e-3, hash_block=1024),
+                          oracle.leaves(a, 64, 1e-3, hash_block=0))
+
+
+def test_hash_block_changes_digest_but_not_the_diff():
+    # different block sizes give different leaves, yet flag exactly the same chunks
+    rng = np.random.default_rng(8)
+    a = rng.uniform(-1, 1, 4096).astype(np.float32)
+    b = a.copy()
+    b[[5, 700, 701, 3000]] += np.float32(1e-2)
+    out = {}
+    for blk in (16, 64, 0):
+        la, lb = oracle.leaves(a, 512, 1e-5, hash_block=blk), oracle.leaves(b, 512, 1e-5, hash_block=blk)
+        out[blk] = np.nonzero((la != lb).any(axis=1))[0].tolist()
+    assert out[16] == out[64] == out[0] == [0, 5, 23]
+    assert not np.array_equal(oracle.leaves(a, 512, 1e-5), oracle.leaves(a, 512, 1e-5, hash_block=0))
+
+
+def test_hash_block_must_be_multiple_of_16():
+    with pytest.raises(ValueError):
+        oracle.leaves(np.zeros(8, np.float32), 32, 1e-3, hash_block=24)
+
+
 def test_raw_mode_hashes_input_bytes():
     # R10: eps == 0 hashes the raw element bytes
     rng = np.random.default_rng(3)
