@@ -45,7 +45,12 @@ CONFIGS = {
                "below-eps changes, 1% chunks below-eps only"),
     "c3": dict(n=1 << 29, workload="configs[2] (C=4 KiB, eps=1e-6 point): 2^29 float64 ~ N(0,1), "
                "1024 geometric clusters (mean 4096) with |d|=10^U(-9,-2)"),
+    "c4": dict(n=1 << 24, workload="configs[3]: one intermediate snapshot (default s=9) of a 64-rank "
+               "HACC run, 2^30 particles x 6 float32 per run (2^24 per rank), ranks sharded over the "
+               "GPUs (strong scaling), 4 KiB chunks, eps=1e-6, clustered divergence 1e-6*4^(s-3)"),
 }
+SNAPSHOT = 9
+C4_RANKS = 64
 CFG = "c2"
 HASH_BLOCK = 16
 N_PARTICLES = CONFIGS[CFG]["n"]
@@ -61,6 +66,16 @@ def make_pair(cfg: str, n: int, seed: int, device: str):
                              seed=seed, device=device)
     if cfg == "c3":
         return synth.c3_pair(n=n, seed=seed, device=device)
+    if cfg == "c4":
+        # full run: this rank's share of the 64 HACC ranks; oracle samples: one rank of n particles
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        rank = int(os.environ.get("RANK", "0"))
+        if n == CONFIGS["c4"]["n"] and device != "cpu":
+            per = C4_RANKS // world
+            ranks = range(rank * per, (rank + 1) * per)
+        else:
+            ranks = [0]
+        return synth.c4_snapshot(SNAPSHOT, ranks, n_particles=n, device=device)
     raise ValueError(cfg)
 
 def peaks():
@@ -242,13 +257,18 @@ def run_ours(args):
     import synth
 
     ck.lib()
+    if CFG == "c4" and C4_RANKS % world:
+        raise SystemExit("c4 shards 64 HACC ranks: the GPU count must divide 64")
     pair = make_pair(CFG, N_PARTICLES, SEED + 1000 * rank, "cuda")
     A, B = pair.a, pair.b
     bytes_pair = 2 * pair.nbytes
     n_elems = sum(t.numel() for t in A)
     L = sum(-(-t.numel() * t.element_size() // CHUNK) for t in A)
     chunks = torch.empty(L, dtype=torch.int64, device="cuda")
-    idx = torch.empty(n_elems, dtype=torch.int64, device="cuda")
+    # element-id output: every element for the per-GPU configs; c4 (6.4e9 elements at N=1) is
+    # capped at 2^28 ids (the full count is still returned; ~2.6e7 expected at s=9)
+    idx = torch.empty(min(n_elems, 1 << 28) if CFG == "c4" else n_elems, dtype=torch.int64,
+                      device="cuda")
     counts = torch.zeros(2, dtype=torch.int64, device="cuda")
     n_arrays = len(A)
     gathered = torch.empty((world * n_arrays, 16), dtype=torch.uint8, device="cuda")
@@ -338,7 +358,9 @@ def run_ours(args):
 
     # end-to-end through the public API with host buffers (pinned), H2D+D2H inside
     e2e = None
-    if not args.no_e2e:
+    if CFG == "c4" and not args.no_e2e:
+        e2e = {"skipped": "c4 holds 48 GiB per GPU at N=1: pinned host copies are not staged"}
+    elif not args.no_e2e:
         ha = [x.cpu().pin_memory() for x in A]
         hb = [x.cpu().pin_memory() for x in B]
         k_e2e = max(3, min(args.steps, 8))
@@ -368,10 +390,13 @@ def run_ours(args):
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": round(ms_max, 4),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "higher_is_better": True, "scaling": "strong" if CFG == "c4" else "weak",
+            "vs_baseline": None,
             "dtype": f"{'f64' if A[0].dtype == torch.float64 else 'f32'} in, f64 quantize/compare, u64 hash",
             "data": f"synthetic (seeded, synth {CFG} recipe)",
             "config": {"workload": WORKLOAD, "name": CFG, "elements_per_array": N_PARTICLES,
+                       **({"snapshot": SNAPSHOT, "hacc_ranks_per_gpu": C4_RANKS // world}
+                          if CFG == "c4" else {}),
                        "arrays_per_run": n_arrays,
                        "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair,
                        "l2": f"inputs larger than L2 ({bytes_pair / 1e9:.1f} GB per GPU per step >> 126 MB)",
@@ -406,13 +431,15 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--path", default="fused", choices=["fused", "unfused"],
                     help="fused: ckpt_compare_pair_async; unfused: build_batch + diff_verify_async")
+    ap.add_argument("--snapshot", type=int, default=9, help="c4: snapshot index 0..9")
     ap.add_argument("--hash-block", type=int, default=16,
                     help="bytes per chained Murmur3F call: 16 = the paper's 128-bit blocks "
                          "(P:610, default); 0 = whole chunk (P:615-618 variant, R23)")
     args = ap.parse_args()
-    global CFG, N_PARTICLES, WORKLOAD, HASH_BLOCK
+    global CFG, N_PARTICLES, WORKLOAD, HASH_BLOCK, SNAPSHOT
     CFG = args.config
     HASH_BLOCK = args.hash_block
+    SNAPSHOT = args.snapshot
     N_PARTICLES = CONFIGS[CFG]["n"]
     WORKLOAD = CONFIGS[CFG]["workload"]
     if args.impl == "reference":

@@ -265,11 +265,13 @@ ckpt_status ckpt_compare(const void *const *a, const void *const *b, const uint6
                          uint8_t *root_b16, void *stream);
 
 /* Same with HOST inputs and outputs: a, b are (host) arrays of host
- * pointers (pinned memory is fastest; pageable works).  The library stages
- * each array to the device (double-buffered over two streams so the copy
- * of one array overlaps the hashing of the previous), runs steps 1-4 and
- * copies the element ids back into idx (host, capacity idx_cap).
- * Synchronous. */
+ * pointers (pinned memory is fastest; pageable works).  The library copies
+ * both runs into one device staging allocation, runs steps 1-4 on the fused
+ * pair path (ckpt_compare_pair_async), sizes the device element-id buffer to
+ * the verified count (read back after the verify scan) and copies the ids
+ * into idx (host, capacity idx_cap).  Synchronous.  Device memory used:
+ * both runs + 8 bytes per chunk + 8 bytes per reported id; it stays cached in
+ * the library's stream-ordered pool (see ckpt_trim_device_memory). */
 ckpt_status ckpt_compare_host(const void *const *a, const void *const *b, const uint64_t *n,
                               uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
                               double eps, uint64_t *idx, uint64_t idx_cap, uint64_t *n_chunks,
@@ -362,6 +364,12 @@ ckpt_status ckpt_tree_nodes(const ckpt_tree *t, uint32_t array, void *dst, uint6
 /* Node count of array `array` (host). */
 ckpt_status ckpt_tree_array_info(const ckpt_tree *t, uint32_t array, uint64_t *n_leaves,
                                  uint64_t *n_nodes);
+
+/* The library allocates device memory from the device's default stream-ordered
+ * pool and keeps freed blocks cached there (no re-mapping between calls).
+ * This returns every unused cached block of the current device to the
+ * driver (synchronises the device). */
+ckpt_status ckpt_trim_device_memory(void);
 
 /* Default BFS threshold T for the current device (SMs * max threads/SM). */
 uint64_t ckpt_default_bfs_threshold(void);

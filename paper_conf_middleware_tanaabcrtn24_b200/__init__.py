@@ -103,6 +103,7 @@ def lib():
     L.ckpt_profile_timeline.restype = i32
     L.ckpt_default_bfs_threshold.restype = u64
     L.ckpt_launch_count.restype = u64
+    L.ckpt_trim_device_memory.restype = i32
     L.ckpt_strerror.argtypes = [i32]
     L.ckpt_strerror.restype = ctypes.c_char_p
     L.ckpt_last_error.restype = ctypes.c_char_p
@@ -467,6 +468,11 @@ def compare_host(arrays_a, arrays_b, chunk_bytes: int, eps: float, idx_cap: Opti
                                    ctypes.cast(rb, ctypes.c_void_p)),
            "ckpt_compare_host", allow_trunc=True)
     return idx[: min(nd.value, idx_cap)], nc.value, nd.value, bytes(ra), bytes(rb)
+
+
+def trim_device_memory() -> None:
+    """Return the library's cached device memory to the driver (ckpt_trim_device_memory)."""
+    _check(lib().ckpt_trim_device_memory(), "ckpt_trim_device_memory")
 
 
 def launch_count() -> int:

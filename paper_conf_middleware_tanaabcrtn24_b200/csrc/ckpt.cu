@@ -15,6 +15,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <deque>
+#include <functional>
 #include <map>
 #include <mutex>
 #include <string>
@@ -162,7 +163,9 @@ static ckpt_status dev_info(int *dev_out, DevInfo *info) {
     if (!d.pool_set) {
         cudaMemPool_t pool;
         CK_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
-        uint64_t thr = 8ull << 30;   // keep up to 8 GiB cached between frees
+        // keep freed blocks mapped in the pool (re-mapping tens of GB per call costs more
+        // than the copies); ckpt_trim_device_memory() returns them to the driver
+        uint64_t thr = UINT64_MAX;
         CK_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
         d.pool_set = true;
     }
@@ -988,13 +991,19 @@ extern "C" ckpt_status ckpt_tree_diff(const ckpt_tree *a, const ckpt_tree *b, ui
 // ---------------------------------------------------------------------------
 // stage 2: verify (K4)
 // ---------------------------------------------------------------------------
+// before_emit (optional): called after the scan kernel (the full count is in
+// *n_diff_dev once the stream reaches that point) and before the emit kernel;
+// it may replace the output buffer and its capacity (exact-size outputs).
+using EmitHook = std::function<ckpt_status(uint64_t **idx, uint64_t *cap)>;
+
 static ckpt_status verify_impl(const void *const *a, const void *const *b, const uint64_t *n,
                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
-                               uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s) {
+                               uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
+                               const EmitHook &before_emit = nullptr) {
     if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
-    if (!n_diff_dev || (!idx && cap)) return fail(CKPT_EINVAL, "NULL output");
+    if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
     std::vector<VerifyArray> va(na);
@@ -1084,6 +1093,7 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
         CK_LAUNCH();
         CK_CUDA(launch_k(verify_scan_kernel, dim3(g_scan), dim3(kVerifyThreads), 0, s, p));
         CK_LAUNCH();
+        if (before_emit) CK_TRY(before_emit(&p.out, &p.cap));
         CK_CUDA(launch_k(d == 0 ? verify_emit_kernel<0> : verify_emit_kernel<1>, dim3(g_emit),
                          dim3(kVerifyThreads), 0, s, p));
     }
@@ -1112,12 +1122,12 @@ extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tr
 // fused pair compare: K1 in pair mode (digest compare and
 // element marking in-kernel), then the ordered chunk list and the element ids
 // ---------------------------------------------------------------------------
-extern "C" ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *const *b,
-                                            const uint64_t *n, uint32_t n_arrays, ckpt_dtype dtype,
-                                            uint32_t chunk_bytes, double eps, uint32_t hash_block,
-                                            uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
-                                            uint64_t idx_cap, uint64_t *counts_dev, void *stream,
-                                            ckpt_tree **out_a, ckpt_tree **out_b) {
+static ckpt_status compare_pair_impl(const void *const *a, const void *const *b, const uint64_t *n,
+                                     uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                     double eps, uint32_t hash_block, uint64_t *chunks,
+                                     uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                                     uint64_t *counts_dev, void *stream, ckpt_tree **out_a,
+                                     ckpt_tree **out_b, const EmitHook &before_emit) {
     if (out_a) *out_a = nullptr;
     if (out_b) *out_b = nullptr;
     if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
@@ -1153,7 +1163,7 @@ extern "C" ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *co
                                     di.sms);
     if (st == CKPT_OK)
         st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
-                         idx, idx_cap, counts_dev + 1, s);
+                         idx, idx_cap, counts_dev + 1, s, before_emit);
     if (st != CKPT_OK) {
         ckpt_tree_free_on(trees[0], stream);
         ckpt_tree_free_on(trees[1], stream);
@@ -1162,6 +1172,16 @@ extern "C" ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *co
     *out_a = trees[0];
     *out_b = trees[1];
     return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *const *b,
+                                            const uint64_t *n, uint32_t n_arrays, ckpt_dtype dtype,
+                                            uint32_t chunk_bytes, double eps, uint32_t hash_block,
+                                            uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                            uint64_t idx_cap, uint64_t *counts_dev, void *stream,
+                                            ckpt_tree **out_a, ckpt_tree **out_b) {
+    return compare_pair_impl(a, b, n, n_arrays, dtype, chunk_bytes, eps, hash_block, chunks,
+                             chunks_cap, idx, idx_cap, counts_dev, stream, out_a, out_b, nullptr);
 }
 
 extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void *const *b,
@@ -1272,70 +1292,64 @@ extern "C" ckpt_status ckpt_compare_host(const void *const *a, const void *const
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
-    uint64_t L = 0;
+    uint64_t L = 0, bytes = 0;
     for (uint32_t k = 0; k < n_arrays; ++k) {
         if (!a[k] || !b[k] || n[k] == 0) return fail(CKPT_EINVAL, "NULL or empty array");
         L += (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
+        bytes += align256(n[k] * esz);
     }
-    cudaStream_t sc = nullptr, sk = nullptr;
-    cudaEvent_t ev_a = nullptr, ev_b = nullptr;
-    CK_CUDA(cudaStreamCreateWithFlags(&sc, cudaStreamNonBlocking));
+    cudaStream_t sk = nullptr;
     CK_CUDA(cudaStreamCreateWithFlags(&sk, cudaStreamNonBlocking));
-    CK_CUDA(cudaEventCreateWithFlags(&ev_a, cudaEventDisableTiming));
-    CK_CUDA(cudaEventCreateWithFlags(&ev_b, cudaEventDisableTiming));
-    std::vector<void *> da(n_arrays, nullptr), db(n_arrays, nullptr);
-    ckpt_tree *ta = nullptr, *tb = nullptr;
+    // one staging allocation for both runs (the pool keeps it mapped between calls)
+    uint8_t *stage = nullptr;
     uint64_t *dchunks = nullptr, *didx = nullptr, *dc = nullptr;
+    std::vector<const void *> da(n_arrays), db(n_arrays);
+    ckpt_tree *ta = nullptr, *tb = nullptr;
+    uint64_t hc[2] = {0, 0};
     ckpt_status st = CKPT_OK;
     auto cu = [&](cudaError_t e, const char *what) {
         if (st == CKPT_OK && e != cudaSuccess)
             st = fail(e == cudaErrorMemoryAllocation ? CKPT_ENOMEM : CKPT_ECUDA,
                       std::string(what) + ": " + cudaGetErrorString(e));
     };
+    cu(cudaMallocAsync((void **)&stage, 2 * bytes, sk), "alloc staging");
+    cu(cudaMallocAsync((void **)&dchunks, L * 8, sk), "alloc chunks");
+    cu(cudaMallocAsync((void **)&dc, 16, sk), "alloc counts");
+    uint64_t off = 0;
     for (uint32_t k = 0; k < n_arrays && st == CKPT_OK; ++k) {
-        cu(cudaMallocAsync(&da[k], n[k] * esz, sc), "alloc A");
-        cu(cudaMallocAsync(&db[k], n[k] * esz, sc), "alloc B");
+        da[k] = stage + off;
+        db[k] = stage + bytes + off;
+        off += align256(n[k] * esz);
     }
     for (uint32_t k = 0; k < n_arrays && st == CKPT_OK; ++k)
-        cu(cudaMemcpyAsync(da[k], a[k], n[k] * esz, cudaMemcpyHostToDevice, sc), "H2D A");
-    cu(cudaEventRecord(ev_a, sc), "event");
+        cu(cudaMemcpyAsync((void *)da[k], a[k], n[k] * esz, cudaMemcpyHostToDevice, sk), "H2D A");
     for (uint32_t k = 0; k < n_arrays && st == CKPT_OK; ++k)
-        cu(cudaMemcpyAsync(db[k], b[k], n[k] * esz, cudaMemcpyHostToDevice, sc), "H2D B");
-    cu(cudaEventRecord(ev_b, sc), "event");
-    cu(cudaMallocAsync((void **)&dchunks, L * 8, sk), "alloc chunks");
-    cu(cudaMallocAsync((void **)&didx, std::max<uint64_t>(idx_cap, 1) * 8, sk), "alloc idx");
-    cu(cudaMallocAsync((void **)&dc, 16, sk), "alloc counts");
-    cu(cudaStreamWaitEvent(sk, ev_a, 0), "wait A");
+        cu(cudaMemcpyAsync((void *)db[k], b[k], n[k] * esz, cudaMemcpyHostToDevice, sk), "H2D B");
+    // the element-id buffer is sized to the count (read back after the verify scan)
+    const EmitHook hook = [&](uint64_t **out, uint64_t *cap) -> ckpt_status {
+        CK_CUDA(cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, sk));
+        CK_CUDA(cudaStreamSynchronize(sk));
+        const uint64_t want = std::min(hc[1], idx_cap);
+        CK_CUDA(cudaMallocAsync((void **)&didx, std::max<uint64_t>(want, 1) * 8, sk));
+        *out = didx;
+        *cap = want;
+        return CKPT_OK;
+    };
     if (st == CKPT_OK)
-        st = ckpt_tree_build_arrays(da.data(), n, n_arrays, dtype, chunk_bytes, eps, sk, &ta);
-    cu(cudaStreamWaitEvent(sk, ev_b, 0), "wait B");
-    if (st == CKPT_OK)
-        st = ckpt_tree_build_arrays(db.data(), n, n_arrays, dtype, chunk_bytes, eps, sk, &tb);
-    if (st == CKPT_OK) st = ckpt_tree_diff_async(ta, tb, 0, dchunks, L, dc, sk);
-    if (st == CKPT_OK)
-        st = verify_impl(da.data(), db.data(), n, n_arrays, dtype, chunk_bytes, dchunks, dc, 0, L,
-                         eps, didx, idx_cap, dc + 1, sk);
-    uint64_t hc[2] = {0, 0};
-    cu(cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, sk), "D2H counts");
-    cu(cudaStreamSynchronize(sk), "sync");
+        st = compare_pair_impl(da.data(), db.data(), n, n_arrays, dtype, chunk_bytes, eps, 16, dchunks,
+                               L, nullptr, 0, dc, sk, &ta, &tb, hook);
     if (st == CKPT_OK && idx_cap && hc[1])
         cu(cudaMemcpyAsync(idx, didx, std::min(hc[1], idx_cap) * 8, cudaMemcpyDeviceToHost, sk), "D2H idx");
     if (st == CKPT_OK && root_a16) st = ckpt_tree_root(ta, root_a16, sk);
     if (st == CKPT_OK && root_b16) st = ckpt_tree_root(tb, root_b16, sk);
+    cu(cudaStreamSynchronize(sk), "sync");
     ckpt_tree_free_on(ta, sk);
     ckpt_tree_free_on(tb, sk);
-    for (uint32_t k = 0; k < n_arrays; ++k) {
-        if (da[k]) cudaFreeAsync(da[k], sk);
-        if (db[k]) cudaFreeAsync(db[k], sk);
-    }
+    if (stage) cudaFreeAsync(stage, sk);
     if (dchunks) cudaFreeAsync(dchunks, sk);
     if (didx) cudaFreeAsync(didx, sk);
     if (dc) cudaFreeAsync(dc, sk);
     cudaStreamSynchronize(sk);
-    cudaStreamSynchronize(sc);
-    cudaEventDestroy(ev_a);
-    cudaEventDestroy(ev_b);
-    cudaStreamDestroy(sc);
     cudaStreamDestroy(sk);
     if (st != CKPT_OK) return st;
     *n_chunks = hc[0];
@@ -1565,6 +1579,16 @@ extern "C" uint64_t ckpt_default_bfs_threshold(void) {
 }
 
 extern "C" uint64_t ckpt_launch_count(void) { return g_launches.load(); }
+
+extern "C" ckpt_status ckpt_trim_device_memory(void) {
+    int dev = 0;
+    CK_CUDA(cudaGetDevice(&dev));
+    CK_CUDA(cudaDeviceSynchronize());
+    cudaMemPool_t pool;
+    CK_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
+    CK_CUDA(cudaMemPoolTrimTo(pool, 0));
+    return CKPT_OK;
+}
 
 extern "C" const char *ckpt_strerror(ckpt_status s) {
     switch (s) {

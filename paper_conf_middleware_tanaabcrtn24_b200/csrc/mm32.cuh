@@ -79,6 +79,13 @@ __device__ __forceinline__ U64p add64(U64p a, U64p b) {
 }
 #endif
 
+#ifdef CKPT_MUL5_C
+// h*5 + c in plain 64-bit C: ptxas folds c into the IMAD.WIDE.U32 addend
+__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
+    const uint64_t x = (((uint64_t)h.hi << 32) | h.lo) * 5ull + c;
+    return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
+}
+#else
 // h*5 + c, c a 64-bit value held in a register pair (kept opaque to ptxas so it
 // emits one IMAD.WIDE.U32 with a 64-bit addend instead of IMAD.WIDE + IADD3 + IMAD.X)
 __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
@@ -93,6 +100,7 @@ __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
         : "r"(h.lo), "r"(h.hi), "l"(c));
     return r;
 }
+#endif
 
 #ifdef CKPT_XS_IMAD
 // hi >> 1 as IMAD.HI.U32(hi, 2^31): moves the shift from the ALU to the FMA pipe
@@ -149,8 +157,15 @@ __device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
 // One chained 16-byte block: (h1,h2) <- Murmur3F(k1||k2, len 16, state (h1,h2)).
 __device__ __forceinline__ void mm3p_block16(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,
                                              uint64_t m2) {
+#ifdef CKPT_PLAIN64
+    uint64_t a = ((uint64_t)h1.hi << 32) | h1.lo, b = ((uint64_t)h2.hi << 32) | h2.lo;
+    mm3_block16(a, b, ((uint64_t)k1.hi << 32) | k1.lo, ((uint64_t)k2.hi << 32) | k2.lo);
+    h1 = U64p{(uint32_t)a, (uint32_t)(a >> 32)};
+    h2 = U64p{(uint32_t)b, (uint32_t)(b >> 32)};
+#else
     mm3p_body(h1, h2, k1, k2, m1, m2);
     mm3p_final(h1, h2, 16u);
+#endif
 }
 
 // Interior node: Murmur3F(left || right, 32 bytes, seed 0)  (Alg. 1, R14).

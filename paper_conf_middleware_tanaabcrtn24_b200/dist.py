@@ -110,3 +110,63 @@ def compare_runs(arrays_a: Sequence[torch.Tensor], arrays_b: Sequence[torch.Tens
     res = RunComparison(ra, rb, chunks[: nl[0]], idx[: nl[1]], chunk_off, elem_off, counts,
                         (TA, TB, top_a, top_b) if keep_trees else ())
     return res
+
+
+# ---------------------------------------------------------------------------
+# one array larger than a GPU's share (optional row)
+# ---------------------------------------------------------------------------
+
+def array_shard(n_elems: int, elem_bytes: int, chunk_bytes: int, world: int,
+                rank: int) -> Tuple[int, int, int, int]:
+    """Split ONE array over `world` GPUs so that every shard is an exact subtree of the
+    single-GPU tree (level-ordered layout with odd-node promotion, reading R13).
+
+    Shards are blocks of 2^k chunks, 2^k = the smallest power of two >= ceil(L / world): GPU g
+    owns chunks [g*2^k, min(L, (g+1)*2^k)).  Node j of level l covers leaves
+    [j*2^l, (j+1)*2^l), and a block starts at an even index on every level below k, so the
+    pairing and the promotion of the last odd node are the same in the shard's own tree as in the
+    global one; the shard root is global node (k, g).  The tree over the gathered shard roots
+    (ckpt_tree_from_digests) is therefore levels k.. of the global tree and its root the
+    single-GPU root.  Returns (elem_lo, elem_hi, chunk_lo, k); an empty shard has lo == hi."""
+    L = -(-n_elems * elem_bytes // chunk_bytes)
+    per = -(-L // world)
+    k = max(0, (per - 1).bit_length())
+    c_lo = min(L, rank << k)
+    c_hi = min(L, (rank + 1) << k)
+    per_elems = chunk_bytes // elem_bytes
+    return min(n_elems, c_lo * per_elems), min(n_elems, c_hi * per_elems), c_lo, k
+
+
+def compare_sharded_array(a_local: torch.Tensor, b_local: torch.Tensor, n_total: int,
+                          chunk_bytes: int, eps: float, group=None) -> RunComparison:
+    """Compare this GPU's shard (array_shard) of ONE large array of run A and run B.
+
+    Every rank builds its subtree, C1 all-gathers the shard roots (empty shards send none) and
+    every rank builds the same top levels -> the single-GPU root; C2 all-reduces the counts.
+    Local ids are shifted to global ones with chunk_offset / elem_offset."""
+    from . import compare_pair_async, tree_from_digests
+    world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+    rank = dist.get_rank(group) if world > 1 else 0
+    lo, hi, c_lo, _ = array_shard(n_total, a_local.element_size(), chunk_bytes, world, rank)
+    if a_local.numel() != hi - lo or b_local.numel() != hi - lo:
+        raise ValueError(f"rank {rank} must hold elements [{lo}, {hi}) of the array")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    chunks = torch.empty(max(1, -(-(hi - lo) * a_local.element_size() // chunk_bytes)),
+                         dtype=torch.int64, device="cuda")
+    idx = torch.empty(max(1, hi - lo), dtype=torch.int64, device="cuda")
+    if hi > lo:
+        TA, TB = compare_pair_async([a_local], [b_local], chunk_bytes, eps, chunks, idx, counts)
+        ra, rb = TA.array_roots(), TB.array_roots()
+    else:
+        TA = TB = None
+        ra = rb = torch.zeros((0, 16), dtype=torch.uint8, device="cuda")
+    local = counts.clone()
+    if world > 1:
+        roots_a, roots_b = gather_roots(ra, group), gather_roots(rb, group)
+        allreduce_counts(counts, group)
+    else:
+        roots_a, roots_b = ra, rb
+    top_a, top_b = tree_from_digests(roots_a), tree_from_digests(roots_b)
+    nl = local.cpu().tolist()
+    return RunComparison(top_a.root(), top_b.root(), chunks[: nl[0]], idx[: nl[1]], c_lo, lo,
+                         counts, (TA, TB, top_a, top_b))

@@ -203,6 +203,31 @@ def rank_pair(rank: int, n_particles: int, seed_base: int, device="cpu", eps: fl
     return Pair(f"rank{rank}", a, b, chunk_bytes, eps, {"clusters": clusters})
 
 
+def c4_frac(snapshot: int) -> float:
+    """Config 4 divergence: none for s <= 2, then 1e-6 * 4^(s-3) of the particles."""
+    return 0.0 if snapshot <= 2 else 1e-6 * 4.0 ** (snapshot - 3)
+
+
+def c4_snapshot(snapshot: int, ranks, n_particles: int = 1 << 24, device="cpu",
+                eps: float = 1e-6, chunk_bytes: int = 4096, n_clusters: int = 8) -> Pair:
+    """Config 4 (BASELINE configs[3]): one intermediate snapshot of a 64-rank HACC run, the
+    given ranks only (a GPU's shard): 6 f32 arrays per rank per run, 2^24 particles per rank
+    (2^30 in total), clustered divergence growing with the snapshot index (c4_frac)."""
+    frac = c4_frac(snapshot)
+    a_list, b_list, meta = [], [], {}
+    for r in ranks:
+        a = hacc_arrays(n_particles, (40 + snapshot) * 1000 + r, device)
+        if frac > 0:
+            b, cl = cluster_mask_perturb(a, frac, n_clusters, (40 + snapshot) * 1000 + 500 + r)
+        else:
+            b, cl = [t.clone() for t in a], []
+        a_list += a
+        b_list += b
+        meta[r] = cl
+    return Pair(f"c4_s{snapshot}", a_list, b_list, chunk_bytes, eps,
+                {"snapshot": snapshot, "ranks": list(ranks), "frac": frac, "clusters": meta})
+
+
 def c5_pair(n_ranks: int = 8, n_particles: int = 50 << 20, seed: int = 50, device="cpu",
             eps: float = 1e-6, chunk_bytes: int = 4096, frac_true: float = 0.10,
             frac_fp: float = 0.01, per_chunk: int = 8) -> Pair:

@@ -88,3 +88,62 @@ def test_root_is_independent_of_rank_count_gloo(world):
         tot_chunks = sum(s[0] for s in sizes)
         assert tot_chunks == sum(ref.n_leaves)
         assert sum(s[1] for s in sizes) == sum(a.size for a in arrays)
+
+
+# ------------------------------------------- one array sharded over GPUs ----
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 5, 8])
+@pytest.mark.parametrize("n", [1, 100, 4096, 100_003, 262_144])
+def test_array_shard_subtree_roots_give_the_single_gpu_root(world, n):
+    # pins the subtree property array_shard relies on, with the oracle standing in for the GPU
+    import oracle
+    rng = np.random.default_rng(n + world)
+    a = rng.uniform(-1, 1, n).astype(np.float32)
+    C = 512
+    ref = oracle.levels(oracle.leaves(a, C, 1e-5))[-1]
+    roots, spans = [], []
+    for r in range(world):
+        lo, hi, c_lo, k = ckd.array_shard(n, 4, C, world, r)
+        spans.append((lo, hi))
+        if hi > lo:
+            assert c_lo == r << k and lo == c_lo * (C // 4)
+            roots.append(oracle.levels(oracle.leaves(a[lo:hi], C, 1e-5))[-1])
+    assert spans[0][0] == 0 and max(h for _, h in spans) == n
+    for (a0, b0), (a1, b1) in zip(spans, spans[1:]):
+        assert b0 == a1 or (a1 == b1 == n)
+    top = oracle.levels(np.stack(roots))[-1]
+    assert top.tobytes() == ref.tobytes()
+
+
+def _shard_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        rng = np.random.default_rng(7)
+        a = rng.uniform(-1, 1, 70_001).astype(np.float32)
+        lo, hi, _, _ = ckd.array_shard(a.size, 4, 1024, world, rank)
+        root = oracle.levels(oracle.leaves(a[lo:hi], 1024, 1e-5))[-1:]
+        gathered = ckd.gather_roots(torch.from_numpy(root.copy()))
+        q.put((rank, oracle.levels(gathered.numpy())[-1].tobytes()))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_array_shard_root_over_gloo_world2():
+    import oracle
+    rng = np.random.default_rng(7)
+    a = rng.uniform(-1, 1, 70_001).astype(np.float32)
+    ref = oracle.levels(oracle.leaves(a, 1024, 1e-5))[-1].tobytes()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_shard_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=120) for _ in range(2)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(top == ref for _, top in out)

@@ -654,3 +654,59 @@ def test_compare_saved_matches_oracle(host_a, tmp_path):
     with pytest.raises(ck.CkptError) as e:
         ck.compare_saved(saved, [t[:-4] for t in pair.a], [t[:-4] for t in pair.b], chunks, idx, counts)
     assert e.value.status == ck.EMISMATCH
+
+
+# ------------------------------------------- config 4 snapshot shard shape --
+
+@pytest.mark.parametrize("snapshot", [2, 6, 9])
+def test_c4_snapshot_shard_matches_oracle(snapshot):
+    # BASELINE configs[3]: a GPU's shard of HACC ranks of one snapshot (reduced particle count)
+    pair = synth.c4_snapshot(snapshot, range(3, 6), n_particles=(1 << 16) + 5, device="cuda")
+    eps, C = pair.eps, 4096
+    an = [np_of(t) for t in pair.a]
+    bn = [np_of(t) for t in pair.b]
+    L = sum(-(-t.numel() * 4 // C) for t in pair.a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(sum(t.numel() for t in pair.a), dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(pair.a, pair.b, C, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    A = oracle.build_checkpoint(an, C, eps, threads=8)
+    B = oracle.build_checkpoint(bn, C, eps, threads=8)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, C, ref_chunks, eps, A)
+    assert np.array_equal(ref_idx, oracle.brute_checkpoint(an, bn, eps))
+    nc, nd = counts.tolist()
+    assert np.array_equal(np_of(chunks[:nc]), ref_chunks)
+    assert np.array_equal(np_of(idx[:nd]), ref_idx)
+    assert TA.root() == A.root and TB.root() == B.root
+    assert (nc == 0) == (snapshot <= 2)
+
+
+# --------------------------------- one array sharded over GPUs (8e, opt) ----
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_array_shards_reassemble_single_gpu_results(world):
+    # every rank's work done in turn on one GPU: shard subtrees + top tree over the shard roots
+    from paper_conf_middleware_tanaabcrtn24_b200 import dist as ckd
+    pair = synth.c3_pair(n=(1 << 20) + 77, seed=71, device="cuda", n_clusters=24, mean_len=300)
+    a, b = pair.a[0], pair.b[0]
+    C, eps = 2048, pair.eps
+    whole = ck.compare(a, b, C, eps)
+    roots_a, roots_b, chunks, idx = [], [], [], []
+    for r in range(world):
+        lo, hi, c_lo, _ = ckd.array_shard(a.numel(), 8, C, world, r)
+        if hi == lo:
+            continue
+        L = -(-(hi - lo) * 8 // C)
+        ch = torch.empty(L, dtype=torch.int64, device="cuda")
+        ix = torch.empty(hi - lo, dtype=torch.int64, device="cuda")
+        cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+        TA, TB = ck.compare_pair_async([a[lo:hi]], [b[lo:hi]], C, eps, ch, ix, cnt)
+        roots_a.append(TA.array_roots()); roots_b.append(TB.array_roots())
+        nc, nd = cnt.tolist()
+        chunks.append(ch[:nc] + c_lo); idx.append(ix[:nd] + lo)
+    assert ck.tree_from_digests(torch.cat(roots_a)).root() == whole[4]
+    assert ck.tree_from_digests(torch.cat(roots_b)).root() == whole[5]
+    assert torch.equal(torch.cat(chunks), whole[0])
+    assert torch.equal(torch.cat(idx), whole[1])
