@@ -277,6 +277,31 @@ ckpt_status ckpt_compare_host(const void *const *a, const void *const *b, const 
                               double eps, uint64_t *idx, uint64_t idx_cap, uint64_t *n_chunks,
                               uint64_t *n_diff, uint8_t *root_a16, uint8_t *root_b16);
 
+/* Out-of-core form: runs larger than HBM, or simply
+ * host-resident, are streamed through a two-slot device ring of segments of
+ * segment_bytes (rounded down to a multiple of chunk_bytes; a segment never
+ * spans two arrays).  The H2D copy of segment k+1 (own stream) overlaps the
+ * hashing (fused pair leaf kernel), compaction and verify of segment k, the
+ * paper's I/O/compute overlap (Fig. 3) with PCIe in place
+ * of Lustre.  Leaves land at their global position in full-size device trees,
+ * so the roots equal the in-HBM build's; interior levels are built at the end.
+ *   a, b        (host) arrays of n_arrays HOST pointers (pinned for full
+ *               overlap; pageable works, with synchronous copies)
+ *   hash_block  as ckpt_tree_build_batch_ex (16 = default)
+ *   chunks, idx (host) outputs, capacities chunks_cap / idx_cap, ascending
+ *               global ids; either may be NULL with capacity 0
+ *   n_chunks, n_diff (host) full counts; root_a16 / root_b16 (host, may be
+ *               NULL) the checkpoint roots
+ * Device memory: 4 x segment_bytes + both trees (32 B per chunk each) + one
+ * byte per chunk + the largest segment's ids.  Synchronous.  Errors as
+ * ckpt_compare_host. */
+ckpt_status ckpt_compare_stream(const void *const *a, const void *const *b, const uint64_t *n,
+                                uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                double eps, uint32_t hash_block, uint64_t segment_bytes,
+                                uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx,
+                                uint64_t idx_cap, uint64_t *n_chunks, uint64_t *n_diff,
+                                uint8_t *root_a16, uint8_t *root_b16);
+
 /* ------------------------------------------------------------------------
  * Tree persistence.  The tree is built at capture time
  * and stored next to the checkpoint (metadata ~0.8% of the data

@@ -30,6 +30,7 @@ __all__ = [
     "CkptError", "Tree", "lib", "tree_build", "tree_from_digests", "tree_diff", "tree_diff_async",
     "verify", "verify_async", "compare", "compare_host", "launch_count", "default_bfs_threshold",
     "tree_deserialize", "tree_load", "compare_saved", "compare_pair_async", "tree_build_batch",
+    "compare_stream", "trim_device_memory",
     "F32", "F64",
 ]
 
@@ -73,6 +74,8 @@ def lib():
     L.ckpt_tree_serialize.argtypes = [vp, vp, u64, pu64, vp]
     L.ckpt_tree_deserialize.argtypes = [vp, u64, vp, pp]
     L.ckpt_compare_saved.argtypes = [vp, u64, pp, pp, pu64, u32, vp, u64, vp, u64, vp, vp, pp, pp]
+    L.ckpt_compare_stream.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, u32, u64, vp, u64, vp, u64,
+                                      pu64, pu64, vp, vp]
     L.ckpt_tree_params.argtypes = [vp, ctypes.POINTER(i32), ctypes.POINTER(u32),
                                    ctypes.POINTER(dbl), ctypes.POINTER(u32)]
     L.ckpt_tree_from_digests.argtypes = [vp, u64, vp, pp]
@@ -111,7 +114,7 @@ def lib():
     for name in ("ckpt_tree_build", "ckpt_tree_build_arrays", "ckpt_tree_build_batch",
                  "ckpt_tree_build_batch_ex", "ckpt_compare_pair_ex", "ckpt_tree_params",
                  "ckpt_tree_serialized_size", "ckpt_tree_serialize", "ckpt_tree_deserialize",
-                 "ckpt_compare_saved",
+                 "ckpt_compare_saved", "ckpt_compare_stream",
                  "ckpt_tree_from_digests",
                  "ckpt_tree_diff", "ckpt_tree_diff_async", "ckpt_verify",
                  "ckpt_verify_arrays_async", "ckpt_compare", "ckpt_compare_host",
@@ -473,6 +476,40 @@ def compare_host(arrays_a, arrays_b, chunk_bytes: int, eps: float, idx_cap: Opti
 def trim_device_memory() -> None:
     """Return the library's cached device memory to the driver (ckpt_trim_device_memory)."""
     _check(lib().ckpt_trim_device_memory(), "ckpt_trim_device_memory")
+
+
+def compare_stream(arrays_a, arrays_b, chunk_bytes: int, eps: float,
+                   segment_bytes: int = 256 << 20, hash_block: int = 16,
+                   chunks_cap: Optional[int] = None, idx_cap: Optional[int] = None):
+    """Steps 1-4 on HOST checkpoints streamed through a device ring (ckpt_compare_stream).
+
+    Returns (chunks, idx (host int64 tensors), n_chunks, n_diff, root_a, root_b)."""
+    ta, tb = _as_list(arrays_a), _as_list(arrays_b)
+    if len(ta) != len(tb) or any(x.numel() != y.numel() for x, y in zip(ta, tb)):
+        raise ValueError("A and B must have the same arrays and lengths")
+    for t in ta + tb:
+        if t.is_cuda or not t.is_contiguous():
+            raise ValueError("compare_stream takes contiguous host tensors")
+    code = _dtype_code(ta[0])
+    esz = 4 if code == F32 else 8
+    L = sum(-(-t.numel() * esz // chunk_bytes) for t in ta)
+    chunks_cap = L if chunks_cap is None else chunks_cap
+    idx_cap = sum(t.numel() for t in ta) if idx_cap is None else idx_cap
+    chunks = torch.empty(max(chunks_cap, 1), dtype=torch.int64)
+    idx = torch.empty(max(idx_cap, 1), dtype=torch.int64)
+    pa, _k1 = _ptr_array(ta)
+    pb, _k2 = _ptr_array(tb)
+    pn, _k3 = _u64_array([t.numel() for t in ta])
+    nc, nd = ctypes.c_uint64(), ctypes.c_uint64()
+    ra, rb = (ctypes.c_uint8 * 16)(), (ctypes.c_uint8 * 16)()
+    _check(lib().ckpt_compare_stream(pa, pb, pn, len(ta), code, chunk_bytes, float(eps), hash_block,
+                                     segment_bytes, chunks.data_ptr(), chunks_cap, idx.data_ptr(),
+                                     idx_cap, ctypes.byref(nc), ctypes.byref(nd),
+                                     ctypes.cast(ra, ctypes.c_void_p),
+                                     ctypes.cast(rb, ctypes.c_void_p)),
+           "ckpt_compare_stream", allow_trunc=True)
+    return (chunks[: min(nc.value, chunks_cap)], idx[: min(nd.value, idx_cap)], nc.value, nd.value,
+            bytes(ra), bytes(rb))
 
 
 def launch_count() -> int:

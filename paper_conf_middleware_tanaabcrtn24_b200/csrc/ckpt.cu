@@ -849,7 +849,7 @@ static ckpt_status get_work(int dev, cudaStream_t s, size_t bytes, uint8_t **wor
 
 static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, const uint8_t *flags,
                                   uint64_t n, uint64_t *out, uint64_t cap, uint64_t *count,
-                                  cudaStream_t s, int sms) {
+                                  cudaStream_t s, int sms, uint64_t base = 0) {
     const uint64_t n_tiles = (n + kCompactTile - 1) / kCompactTile;
     int dev = 0;
     CK_CUDA(cudaGetDevice(&dev));
@@ -862,6 +862,7 @@ static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, co
     p.out = out;
     p.cap = cap;
     p.count = count;
+    p.base = base;
     // co-resident grid (the look-back relies on it); static tile striding
     static std::atomic<int> occ0{0}, occ1{0};
     std::atomic<int> &occ = mode == 0 ? occ0 : occ1;
@@ -1001,14 +1002,15 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
-                               const EmitHook &before_emit = nullptr) {
+                               const EmitHook &before_emit = nullptr, uint64_t chunk_base0 = 0,
+                               uint64_t elem_base0 = 0) {
     if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
     if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
     std::vector<VerifyArray> va(na);
     std::vector<uint64_t> cb(na);
-    uint64_t c = 0, e = 0;
+    uint64_t c = chunk_base0, e = elem_base0;   // global ids of the first array's chunk / element 0
     for (uint32_t k = 0; k < na; ++k) {
         if (!a[k] || !b[k]) return fail(CKPT_EINVAL, "NULL data pointer");
         if ((uintptr_t)a[k] % 16 || (uintptr_t)b[k] % 16)
@@ -1027,7 +1029,7 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     int dev;
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
-    const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c);
+    const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c - chunk_base0);
     VerifyParams p;
     std::memset(&p, 0, sizeof(p));
     uint8_t *tab = nullptr;
@@ -1355,6 +1357,211 @@ extern "C" ckpt_status ckpt_compare_host(const void *const *a, const void *const
     *n_chunks = hc[0];
     *n_diff = hc[1];
     if (hc[1] > idx_cap) return fail(CKPT_ETRUNC, "difference list longer than cap");
+    return CKPT_OK;
+}
+
+// ---------------------------------------------------------------------------
+// out-of-core streaming compare: host-resident runs are
+// streamed through a two-slot device ring of chunk-aligned segments; the H2D
+// copy of segment k+1 (copy stream) overlaps the leaf hashing, the in-kernel
+// digest compare, the compaction and the verify of segment k (compute
+// stream).  Leaves land at their global position in full-size trees, so the
+// trees (and roots) equal the in-HBM build; device memory is bounded by the
+// ring, the trees, one flag byte per chunk and the per-segment outputs.
+// The paper's pipeline overlaps I/O and hashing the same way (Fig. 3
+// P:476-495), there from Lustre through io_uring.
+// ---------------------------------------------------------------------------
+static ckpt_status alloc_tree(const uint64_t *n, uint32_t na, ckpt_dtype dtype, uint32_t C, double eps,
+                              uint32_t hb, int dev, cudaStream_t s, ckpt_tree **out) {
+    const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
+    ckpt_tree *t = new ckpt_tree();
+    t->device = dev;
+    t->stream = s;
+    t->dtype = dtype;
+    t->chunk_bytes = C;
+    t->eps = eps;
+    t->hash_block = hb;
+    t->n_elems.assign(n, n + na);
+    std::vector<uint64_t> leaves(na);
+    for (uint32_t a = 0; a < na; ++a) leaves[a] = (n[a] * esz + C - 1) / C;
+    layout(t, leaves);
+    ckpt_status st = prepare_tree(t, s);
+    if (st != CKPT_OK) { ckpt_tree_free_on(t, s); return st; }
+    *out = t;
+    return CKPT_OK;
+}
+
+extern "C" ckpt_status ckpt_compare_stream(const void *const *a, const void *const *b,
+                                           const uint64_t *n, uint32_t n_arrays, ckpt_dtype dtype,
+                                           uint32_t chunk_bytes, double eps, uint32_t hash_block,
+                                           uint64_t segment_bytes, uint64_t *chunks,
+                                           uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                                           uint64_t *n_chunks, uint64_t *n_diff, uint8_t *root_a16,
+                                           uint8_t *root_b16) {
+    if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
+    if (!n_chunks || !n_diff || (!idx && idx_cap) || (!chunks && chunks_cap))
+        return fail(CKPT_EINVAL, "NULL output");
+    CK_TRY(check_common(dtype, chunk_bytes, eps));
+    CK_TRY(norm_block(hash_block, chunk_bytes, &hash_block));
+    const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
+    for (uint32_t k = 0; k < n_arrays; ++k)
+        if (!a[k] || !b[k] || n[k] == 0) return fail(CKPT_EINVAL, "NULL or empty array");
+    const uint64_t seg = std::max<uint64_t>(1, segment_bytes / chunk_bytes) * chunk_bytes;
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    // segments: (array, byte offset, bytes, global chunk id, global element id)
+    struct Seg { uint32_t a; uint64_t off, bytes, chunk0, elem0; };
+    std::vector<Seg> segs;
+    uint64_t L = 0, E = 0;
+    for (uint32_t k = 0; k < n_arrays; ++k) {
+        const uint64_t nb = n[k] * esz;
+        for (uint64_t o = 0; o < nb; o += seg)
+            segs.push_back({k, o, std::min(seg, nb - o), L + o / chunk_bytes, E + o / esz});
+        L += (nb + chunk_bytes - 1) / chunk_bytes;
+        E += n[k];
+    }
+    cudaStream_t sc = nullptr, sk = nullptr;
+    CK_CUDA(cudaStreamCreateWithFlags(&sc, cudaStreamNonBlocking));
+    CK_CUDA(cudaStreamCreateWithFlags(&sk, cudaStreamNonBlocking));
+    cudaEvent_t copied[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr};
+    uint8_t *ring = nullptr, *flags = nullptr;
+    uint64_t *dchunks = nullptr, *didx = nullptr, *dc = nullptr;
+    uint64_t didx_cap = 0;
+    ckpt_tree *ta = nullptr, *tb = nullptr;
+    uint64_t tot_c = 0, tot_e = 0;
+    ckpt_status st = CKPT_OK;
+    auto cu = [&](cudaError_t e, const char *what) {
+        if (st == CKPT_OK && e != cudaSuccess)
+            st = fail(e == cudaErrorMemoryAllocation ? CKPT_ENOMEM : CKPT_ECUDA,
+                      std::string(what) + ": " + cudaGetErrorString(e));
+    };
+    for (int i = 0; i < 2; ++i) {
+        cu(cudaEventCreateWithFlags(&copied[i], cudaEventDisableTiming), "event");
+        cu(cudaEventCreateWithFlags(&freed[i], cudaEventDisableTiming), "event");
+    }
+    cu(cudaMallocAsync((void **)&ring, 4 * seg, sk), "alloc ring");          // 2 slots x (A, B)
+    cu(cudaMallocAsync((void **)&flags, std::max<uint64_t>(L, 1), sk), "alloc flags");
+    cu(cudaMallocAsync((void **)&dchunks, std::max<uint64_t>(seg / chunk_bytes, 1) * 8, sk), "alloc chunks");
+    cu(cudaMallocAsync((void **)&dc, 16, sk), "alloc counts");
+    if (st == CKPT_OK) st = alloc_tree(n, n_arrays, dtype, chunk_bytes, eps, hash_block, dev, sk, &ta);
+    if (st == CKPT_OK) st = alloc_tree(n, n_arrays, dtype, chunk_bytes, eps, hash_block, dev, sk, &tb);
+    // the ring exists before the copy stream uses it
+    cu(cudaEventRecord(freed[0], sk), "event");
+    cu(cudaEventRecord(freed[1], sk), "event");
+    uint64_t hc[2] = {0, 0};
+    unsigned int *ctr = nullptr;
+    unsigned long long *ticket = nullptr;
+    auto enqueue_copy = [&](size_t k) {
+        const Seg &g = segs[k];
+        const int sl = (int)(k & 1);
+        uint8_t *da = ring + (size_t)sl * 2 * seg, *db = da + seg;
+        cu(cudaStreamWaitEvent(sc, freed[sl], 0), "wait slot");
+        cu(cudaMemcpyAsync(da, (const uint8_t *)a[g.a] + g.off, g.bytes, cudaMemcpyHostToDevice, sc), "H2D A");
+        cu(cudaMemcpyAsync(db, (const uint8_t *)b[g.a] + g.off, g.bytes, cudaMemcpyHostToDevice, sc), "H2D B");
+        cu(cudaEventRecord(copied[sl], sc), "event");
+    };
+    if (st == CKPT_OK && !segs.empty()) enqueue_copy(0);
+    for (size_t k = 0; k < segs.size() && st == CKPT_OK; ++k) {
+        const Seg &g = segs[k];
+        const int sl = (int)(k & 1);
+        uint8_t *da = ring + (size_t)sl * 2 * seg, *db = da + seg;
+        if (k + 1 < segs.size()) enqueue_copy(k + 1);        // overlaps everything below
+        cu(cudaStreamWaitEvent(sk, copied[sl], 0), "wait copy");
+        // leaves of both runs' segment in one pair-mode launch, written at their global slots
+        const uint64_t nl = (g.bytes + chunk_bytes - 1) / chunk_bytes;
+        const uint64_t local0 = g.off / chunk_bytes;                  // chunk index inside the array
+        const uint64_t tasks_per = (nl + kRows - 1) / kRows;
+        std::vector<LeafArray> table(2);
+        ckpt_tree *tt[2] = {ta, tb};
+        uint8_t *src[2] = {da, db};
+        for (int r = 0; r < 2; ++r) {
+            LeafArray &e = table[r];
+            e.data = src[r];
+            e.nbytes = g.bytes;
+            e.n_leaves = nl;
+            e.n_full = g.bytes / chunk_bytes;
+            e.task_begin = (uint64_t)r * tasks_per;
+            e.out = tt[r]->nodes + tt[r]->off[g.a] + local0;
+            e.chunk_base = g.chunk0;
+        }
+        PairParams pp;
+        std::memset(&pp, 0, sizeof(pp));
+        pp.flags = flags;
+        pp.n_pair = tasks_per;
+        pp.m = 1;
+        if (st == CKPT_OK) st = get_pair_ctr(dev, sk, tasks_per, &ctr);
+        pp.ctr = ctr;
+        if (st == CKPT_OK && !ticket) {
+            uint64_t *unused_states;
+            uint32_t unused_epoch;
+            st = get_scratch(dev, sk, 0, &unused_states, &ticket, &unused_epoch);
+            ticket += kLeafTicketSlot;
+        }
+        if (st == CKPT_OK)
+            st = launch_leaves(table, 2 * tasks_per, dtype, eps, chunk_bytes, hash_block, sk, di.sms, &pp,
+                               ticket);
+        // this segment's flagged chunks (global ids), then its verify
+        if (st == CKPT_OK)
+            st = launch_compact(1, nullptr, nullptr, flags + g.chunk0, nl, dchunks, nl, dc, sk, di.sms,
+                                g.chunk0);
+        uint64_t seg_c = 0, seg_e = 0;
+        const EmitHook hook = [&](uint64_t **out, uint64_t *cap) -> ckpt_status {
+            CK_CUDA(cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, sk));
+            CK_CUDA(cudaStreamSynchronize(sk));
+            seg_c = hc[0];
+            seg_e = hc[1];
+            if (seg_e > didx_cap) {
+                if (didx) CK_CUDA(cudaFreeAsync(didx, sk));
+                didx_cap = std::max<uint64_t>(seg_e, 2 * didx_cap);
+                CK_CUDA(cudaMallocAsync((void **)&didx, didx_cap * 8, sk));
+            }
+            *out = didx;
+            *cap = didx_cap;
+            return CKPT_OK;
+        };
+        const void *va[1] = {da}, *vb[1] = {db};
+        const uint64_t vn[1] = {g.bytes / esz};
+        if (st == CKPT_OK)
+            st = verify_impl(va, vb, vn, 1, dtype, chunk_bytes, dchunks, dc, 0, nl, eps, nullptr, 0, dc + 1,
+                             sk, hook, g.chunk0, g.elem0);
+        cu(cudaEventRecord(freed[sl], sk), "event");          // slot reusable after the verify
+        // append this segment's ids to the caller's host buffers (ascending across segments)
+        if (st == CKPT_OK && seg_c && tot_c < chunks_cap)
+            cu(cudaMemcpyAsync(chunks + tot_c, dchunks, std::min(seg_c, chunks_cap - tot_c) * 8,
+                               cudaMemcpyDeviceToHost, sk), "D2H chunks");
+        if (st == CKPT_OK && seg_e && tot_e < idx_cap)
+            cu(cudaMemcpyAsync(idx + tot_e, didx, std::min(seg_e, idx_cap - tot_e) * 8,
+                               cudaMemcpyDeviceToHost, sk), "D2H idx");
+        tot_c += seg_c;
+        tot_e += seg_e;
+    }
+    if (st == CKPT_OK) {
+        ckpt_tree *both[2] = {ta, tb};
+        st = launch_levels(both, 2, sk);
+    }
+    if (st == CKPT_OK && root_a16) st = ckpt_tree_root(ta, root_a16, sk);
+    if (st == CKPT_OK && root_b16) st = ckpt_tree_root(tb, root_b16, sk);
+    cu(cudaStreamSynchronize(sk), "sync");
+    cudaStreamSynchronize(sc);
+    ckpt_tree_free_on(ta, sk);
+    ckpt_tree_free_on(tb, sk);
+    if (ring) cudaFreeAsync(ring, sk);
+    if (flags) cudaFreeAsync(flags, sk);
+    if (dchunks) cudaFreeAsync(dchunks, sk);
+    if (didx) cudaFreeAsync(didx, sk);
+    if (dc) cudaFreeAsync(dc, sk);
+    cudaStreamSynchronize(sk);
+    for (int i = 0; i < 2; ++i) {
+        if (copied[i]) cudaEventDestroy(copied[i]);
+        if (freed[i]) cudaEventDestroy(freed[i]);
+    }
+    cudaStreamDestroy(sc);
+    cudaStreamDestroy(sk);
+    if (st != CKPT_OK) return st;
+    *n_chunks = tot_c;
+    *n_diff = tot_e;
+    if (tot_c > chunks_cap || tot_e > idx_cap) return fail(CKPT_ETRUNC, "output longer than cap");
     return CKPT_OK;
 }
 

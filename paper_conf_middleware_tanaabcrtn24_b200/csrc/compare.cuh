@@ -129,6 +129,7 @@ struct CompactParams {
     uint64_t *states;         // >= n_tiles entries (epoch-tagged, never cleared)
     unsigned long long *ticket;  // 0 on entry, 0 again on exit
     uint32_t epoch;
+    uint64_t base;            // added to every output index (a segment's global chunk id)
 };
 
 template <int MODE>
@@ -189,7 +190,7 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_c
         for (int k = 0; k < kCompactRows; ++k) {
             if (bits[k] & (1u << lane)) {
                 const uint64_t pos = excl + row_off[k * 8 + warp] + __popc(bits[k] & lt);
-                if (pos < p.cap) p.out[pos] = t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
+                if (pos < p.cap) p.out[pos] = p.base + t0 + (uint64_t)k * kCompactThreads + warp * 32 + lane;
             }
         }
         __syncthreads();

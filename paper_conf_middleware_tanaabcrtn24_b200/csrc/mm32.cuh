@@ -7,7 +7,7 @@
 //   * 64-bit x constant -> IMAD.WIDE.U32 + 2 x IMAD (fma pipe, 3 instr),
 //   * k ^= k >> 33      -> lo ^= hi >> 1 (SHF + LOP3),
 //   * rotl64 by r       -> two funnel shifts (SHF.L.W) on swapped halves,
-//   * h*5 + c           -> IMAD.WIDE.U32 with a 64-bit addend + IMAD.
+//   * h*5 + c           -> IMAD.WIDE.U32 with a 64-bit addend + IMAD + IADD3.
 // The leaf kernel is issue-bound, so every instruction
 // of this step is throughput.
 #pragma once
@@ -79,28 +79,14 @@ __device__ __forceinline__ U64p add64(U64p a, U64p b) {
 }
 #endif
 
-#ifdef CKPT_MUL5_C
-// h*5 + c in plain 64-bit C: ptxas folds c into the IMAD.WIDE.U32 addend
+// h*5 + c in plain 64-bit C: ptxas folds the 64-bit addend c into IMAD.WIDE.U32
+// (lo*5 + c) and adds hi*5 with one IMAD + IADD3.  (An inline-asm mad.wide with
+// an immediate multiplier was split by ptxas into IMAD.WIDE + IADD3 + IMAD.X:
+// 2 more instructions per block, measured 1.8% slower in the leaf kernel.)
 __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
     const uint64_t x = (((uint64_t)h.hi << 32) | h.lo) * 5ull + c;
     return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
 }
-#else
-// h*5 + c, c a 64-bit value held in a register pair (kept opaque to ptxas so it
-// emits one IMAD.WIDE.U32 with a 64-bit addend instead of IMAD.WIDE + IADD3 + IMAD.X)
-__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
-    U64p r;
-    asm("{\n\t"
-        ".reg .u64 p;\n\t"
-        "mad.wide.u32 p, %2, 5, %4;\n\t"
-        "mov.b64 {%0, %1}, p;\n\t"
-        "mad.lo.u32 %1, %3, 5, %1;\n\t"
-        "}"
-        : "=r"(r.lo), "=r"(r.hi)
-        : "r"(h.lo), "r"(h.hi), "l"(c));
-    return r;
-}
-#endif
 
 #ifdef CKPT_XS_IMAD
 // hi >> 1 as IMAD.HI.U32(hi, 2^31): moves the shift from the ALU to the FMA pipe
@@ -157,15 +143,8 @@ __device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
 // One chained 16-byte block: (h1,h2) <- Murmur3F(k1||k2, len 16, state (h1,h2)).
 __device__ __forceinline__ void mm3p_block16(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,
                                              uint64_t m2) {
-#ifdef CKPT_PLAIN64
-    uint64_t a = ((uint64_t)h1.hi << 32) | h1.lo, b = ((uint64_t)h2.hi << 32) | h2.lo;
-    mm3_block16(a, b, ((uint64_t)k1.hi << 32) | k1.lo, ((uint64_t)k2.hi << 32) | k2.lo);
-    h1 = U64p{(uint32_t)a, (uint32_t)(a >> 32)};
-    h2 = U64p{(uint32_t)b, (uint32_t)(b >> 32)};
-#else
     mm3p_body(h1, h2, k1, k2, m1, m2);
     mm3p_final(h1, h2, 16u);
-#endif
 }
 
 // Interior node: Murmur3F(left || right, 32 bytes, seed 0)  (Alg. 1, R14).

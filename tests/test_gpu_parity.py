@@ -710,3 +710,44 @@ def test_array_shards_reassemble_single_gpu_results(world):
     assert ck.tree_from_digests(torch.cat(roots_b)).root() == whole[5]
     assert torch.equal(torch.cat(chunks), whole[0])
     assert torch.equal(torch.cat(idx), whole[1])
+
+
+# -------------------------------------------- out-of-core streaming (f3) ----
+
+@pytest.mark.parametrize("seg", [4096, 1 << 16, 3 * 4096 + 100, 1 << 30])
+@pytest.mark.parametrize("pinned", [True, False])
+def test_compare_stream_matches_oracle(seg, pinned):
+    pair = synth.c5_pair(n_ranks=1, n_particles=(1 << 15) + 300, seed=81, device="cpu")
+    C, eps = 4096, pair.eps
+    ha = [t.pin_memory() if pinned else t for t in pair.a]
+    hb = [t.pin_memory() if pinned else t for t in pair.b]
+    chunks, idx, nc, nd, ra, rb = ck.compare_stream(ha, hb, C, eps, segment_bytes=seg)
+    an = [t.numpy() for t in pair.a]
+    bn = [t.numpy() for t in pair.b]
+    A = oracle.build_checkpoint(an, C, eps, threads=8)
+    B = oracle.build_checkpoint(bn, C, eps, threads=8)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, C, ref_chunks, eps, A)
+    assert nc == ref_chunks.size and nd == ref_idx.size and nd > 0
+    assert np.array_equal(chunks.numpy(), ref_chunks)
+    assert np.array_equal(idx.numpy(), ref_idx)
+    assert ra == A.root and rb == B.root
+
+
+def test_compare_stream_f64_hash_block_and_truncation():
+    pair = synth.c3_pair(n=(1 << 18) + 3, seed=82, device="cpu", n_clusters=12, mean_len=200)
+    C, eps = 1024, pair.eps
+    an, bn = [pair.a[0].numpy()], [pair.b[0].numpy()]
+    A = oracle.build_checkpoint(an, C, eps, hash_block=0)
+    B = oracle.build_checkpoint(bn, C, eps, hash_block=0)
+    ref_chunks = oracle.diff_checkpoint(A, B)
+    ref_idx = oracle.verify_checkpoint(an, bn, C, ref_chunks, eps, A)
+    chunks, idx, nc, nd, ra, rb = ck.compare_stream(pair.a, pair.b, C, eps, segment_bytes=50_000,
+                                                    hash_block=0)
+    assert np.array_equal(chunks.numpy(), ref_chunks) and np.array_equal(idx.numpy(), ref_idx)
+    assert ra == A.root and rb == B.root
+    # truncated outputs keep the ascending prefix and the full counts
+    chunks, idx, nc, nd, _, _ = ck.compare_stream(pair.a, pair.b, C, eps, segment_bytes=50_000,
+                                                  hash_block=0, chunks_cap=5, idx_cap=7)
+    assert nc == ref_chunks.size and nd == ref_idx.size
+    assert np.array_equal(chunks.numpy(), ref_chunks[:5]) and np.array_equal(idx.numpy(), ref_idx[:7])
