@@ -751,3 +751,98 @@ def test_compare_stream_f64_hash_block_and_truncation():
                                                   hash_block=0, chunks_cap=5, idx_cap=7)
     assert nc == ref_chunks.size and nd == ref_idx.size
     assert np.array_equal(chunks.numpy(), ref_chunks[:5]) and np.array_equal(idx.numpy(), ref_idx[:7])
+
+
+# ------------------------------------------- maximum sizes (64-bit ids) ----
+
+@pytest.mark.slow
+def test_array_beyond_2pow32_elements_fused_path():
+    """One f32 array of 2^32 + 4099 elements (17.2 GB per run; element ids and byte offsets
+    beyond 32 bits, ragged last chunk) on the fused pair path: chunk list and element ids equal
+    the oracle's on every perturbed chunk, leaves of sampled chunks (incl. both sides of the
+    2^32-element boundary and the last chunk) equal the oracle's, every interior level equals
+    the oracle's levels over the GPU leaves, and b == a outside the perturbed elements."""
+    n = (1 << 32) + 4099
+    C, eps = 4096, 1e-6
+    per = C // 4
+    a = torch.empty(n, dtype=torch.float32, device="cuda")
+    step = 1 << 28
+    for o in range(0, n, step):
+        m = min(step, n - o)
+        a[o:o + m] = synth.uniform(91, m, "cuda", offset=o) * 2.0 - 1.0
+    b = a.clone()
+    rng = np.random.default_rng(91)
+    pos = np.unique(np.concatenate([rng.integers(0, n, 40), rng.integers(1 << 32, n, 16),
+                                    [n - 1, (1 << 32) - 1, 1 << 32, 0]]))
+    mag = rng.uniform(0.05, 20.0, pos.size) * eps * np.where(rng.random(pos.size) < 0.5, -1, 1)
+    ip = torch.as_tensor(pos, dtype=torch.int64, device="cuda")
+    b[ip] = (a[ip].double() + torch.as_tensor(mag, device="cuda")).float()
+    changed = np_of(torch.nonzero(a != b).view(-1))
+    assert np.isin(changed, pos).all() and changed.size > 40
+    L = -(-n * 4 // C)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(1 << 16, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async([a], [b], C, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    nc, nd = counts.tolist()
+    # expected: only perturbed chunks can differ; the oracle decides each of them
+    cand = np.unique(pos // per)
+    ref_chunks, ref_idx = [], []
+    for c in cand:
+        lo, hi = c * per, min(n, (c + 1) * per)
+        ca, cb = np_of(a[lo:hi]), np_of(b[lo:hi])
+        if not np.array_equal(oracle.leaves(ca, C, eps), oracle.leaves(cb, C, eps)):
+            ref_chunks.append(c)
+            ref_idx.extend((oracle.brute(ca, cb, eps) + lo).tolist())
+    assert nc == len(ref_chunks) and np.array_equal(np_of(chunks[:nc]), np.array(ref_chunks))
+    assert nd == len(ref_idx) and np.array_equal(np_of(idx[:nd]), np.array(ref_idx))
+    assert max(ref_idx) >= (1 << 32)
+    # leaves of sampled chunks + every interior level of tree A
+    na = gpu_tree_nodes(TA, 0)
+    sample = np.unique(np.concatenate([rng.integers(0, L, 64), [0, L - 1, (1 << 32) // per - 1,
+                                                                (1 << 32) // per]]))
+    for c in sample:
+        lo, hi = c * per, min(n, (c + 1) * per)
+        assert np.array_equal(oracle.leaves(np_of(a[lo:hi]), C, eps)[0], na[c]), c
+    assert np.array_equal(oracle.levels(na[:L]), na)
+    del a, b
+
+
+@pytest.mark.slow
+def test_config5_full_size_sampled_parity():
+    """BASELINE configs[4] per-GPU shard at full size (8 ranks x 50*2^20 particles x 6 f32,
+    20 GB per run) on the fused path: every flagged chunk and every element id of a sampled
+    set of arrays equals the oracle's over those arrays, and the global counts equal a
+    brute-force device count of |a-b| > eps (property at full size)."""
+    pair = synth.c5_pair(device="cuda")
+    C, eps = pair.chunk_bytes, pair.eps
+    L = sum(-(-t.numel() * 4 // C) for t in pair.a)
+    n_el = sum(t.numel() for t in pair.a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(n_el, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(pair.a, pair.b, C, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    nc, nd = counts.tolist()
+    got_c, got_i = np_of(chunks[:nc]), np_of(idx[:nd])
+    # brute-force property over all 2.5e9 elements (binary64 |a-b| > eps on the device)
+    brute = 0
+    for x, y in zip(pair.a, pair.b):
+        brute += int((x.double() - y.double()).abs().gt(eps).sum().item())
+    assert nd == brute
+    # oracle over sampled arrays (global numbering)
+    per = C // 4
+    chunk_base = np.cumsum([0] + [-(-t.numel() * 4 // C) for t in pair.a])
+    elem_base = np.cumsum([0] + [t.numel() for t in pair.a])
+    for k in (0, 7, 23, len(pair.a) - 1):
+        an, bn = np_of(pair.a[k]), np_of(pair.b[k])
+        la = oracle.leaves(an, C, eps, threads=os.cpu_count() or 8)
+        lb = oracle.leaves(bn, C, eps, threads=os.cpu_count() or 8)
+        ref_c = np.nonzero(np.any(la != lb, axis=1))[0]
+        ref_i = oracle.verify(an, bn, C, ref_c, eps)
+        sel_c = got_c[(got_c >= chunk_base[k]) & (got_c < chunk_base[k + 1])] - chunk_base[k]
+        sel_i = got_i[(got_i >= elem_base[k]) & (got_i < elem_base[k + 1])] - elem_base[k]
+        assert np.array_equal(sel_c, ref_c), k
+        assert np.array_equal(sel_i, ref_i), k
+        assert np.array_equal(gpu_tree_nodes(TA, k)[: la.shape[0]], la), k
