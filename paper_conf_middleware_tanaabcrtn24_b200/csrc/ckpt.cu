@@ -369,10 +369,17 @@ static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
     } else {
         CK_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kLeafSmem));
     }
-    uint64_t want = (tasks + kLeafWarps - 1) / kLeafWarps;
-    uint64_t grid = std::min<uint64_t>(want, (uint64_t)sms * per_sm);
+    // Few tasks (fewer 32-chunk tasks than resident warps, e.g. large chunks): one-warp CTAs, one
+    // per task, so the block scheduler spreads the chains evenly over the SMs (8-warp CTAs
+    // would put 16 warps on some SMs and 8 on others, and the loaded SMs set the time).
+    const uint64_t resident = (uint64_t)sms * per_sm * kLeafWarps;
+    const bool few = tasks < resident;
+    const unsigned cta_warps = few ? 1u : (unsigned)kLeafWarps;
+    const size_t smem = (size_t)cta_warps * kWarpSmem + 16;
+    uint64_t want = (tasks + cta_warps - 1) / cta_warps;
+    uint64_t grid = few ? want : std::min<uint64_t>(want, (uint64_t)sms * per_sm);
     ProfScope prof(0, s);
-    CK_CUDA(launch_k(k, dim3((unsigned)grid), dim3(kLeafWarps * 32), kLeafSmem, s, P));
+    CK_CUDA(launch_k(k, dim3((unsigned)grid), dim3(cta_warps * 32), smem, s, P));
     CK_LAUNCH();
     return CKPT_OK;
 }
@@ -391,6 +398,8 @@ static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms, 
     if (pair) {   // fused pair mode: the bench chunk size specialised, others generic
         if constexpr (!RAW) {
             if (C == 4096) return launch_leaf_t<DT, RAW, 4096, true>(P, s, sms);
+            if (C == 32768) return launch_leaf_t<DT, RAW, 32768, true>(P, s, sms);
+            if (C == 65536) return launch_leaf_t<DT, RAW, 65536, true>(P, s, sms);
         }
         return launch_leaf_t<DT, RAW, 0, true>(P, s, sms);
     }

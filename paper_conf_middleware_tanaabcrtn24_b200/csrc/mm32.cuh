@@ -108,24 +108,36 @@ __device__ __forceinline__ U64p fmix64p(U64p k) {
     return k;
 }
 
-// Murmur3F body step for one full 16-byte block.
-__device__ __forceinline__ void mm3p_body(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,
-                                          uint64_t m2) {
+// Murmur3F body, key half: k1 = rotl(k1*c1, 31)*c2, k2 = rotl(k2*c2, 33)*c1.  It does
+// not depend on the state, so a chain can mix the keys of later blocks ahead.
+__device__ __forceinline__ void mm3p_kmix(U64p &k1, U64p &k2) {
     // c1 = 0x87c37b91114253d5, c2 = 0x4cf5ad432745937f
     k1 = mulc(k1, 0x114253d5u, 0x87c37b91u);
     k1 = rotl_lt32<31>(k1);
     k1 = mulc(k1, 0x2745937fu, 0x4cf5ad43u);
+    k2 = mulc(k2, 0x2745937fu, 0x4cf5ad43u);
+    k2 = rotl_gt32<33>(k2);
+    k2 = mulc(k2, 0x114253d5u, 0x87c37b91u);
+}
+
+// Murmur3F body, state half, with mixed keys.
+__device__ __forceinline__ void mm3p_hstep(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,
+                                           uint64_t m2) {
     h1 = xor64(h1, k1);
     h1 = rotl_lt32<27>(h1);
     h1 = add64(h1, h2);
     h1 = mul5_add(h1, m1);   // m1 = 0x52dce729
-    k2 = mulc(k2, 0x2745937fu, 0x4cf5ad43u);
-    k2 = rotl_gt32<33>(k2);
-    k2 = mulc(k2, 0x114253d5u, 0x87c37b91u);
     h2 = xor64(h2, k2);
     h2 = rotl_lt32<31>(h2);
     h2 = add64(h2, h1);
     h2 = mul5_add(h2, m2);   // m2 = 0x38495ab5
+}
+
+// Murmur3F body step for one full 16-byte block.
+__device__ __forceinline__ void mm3p_body(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,
+                                          uint64_t m2) {
+    mm3p_kmix(k1, k2);
+    mm3p_hstep(h1, h2, k1, k2, m1, m2);
 }
 
 // Murmur3F finalisation for a total length `len` < 2^32.

@@ -846,3 +846,30 @@ def test_config5_full_size_sampled_parity():
         assert np.array_equal(sel_c, ref_c), k
         assert np.array_equal(sel_i, ref_i), k
         assert np.array_equal(gpu_tree_nodes(TA, k)[: la.shape[0]], la), k
+
+
+# -------------------------- latency variant of the leaf kernel (few chains) --
+
+@pytest.mark.parametrize("dt,chunk,n,eps", [(torch.float32, 16384, (1 << 22) + 5, 1e-6),
+                                            (torch.float64, 65536, (1 << 21) + 3, 1e-8),
+                                            (torch.float32, 32768, 300_001, 0.0)])
+def test_large_chunk_latency_variant_matches_oracle(dt, chunk, n, eps):
+    # few long chains -> one-warp CTAs of the LAT instantiation (pair and single-tree paths)
+    a = _data(n, dt, 5 + chunk)
+    b = a.clone()
+    b[:: 40_000] += 1e-3
+    L = -(-n * a.element_size() // chunk)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(n, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async([a], [b], chunk, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    an, bn = np_of(a), np_of(b)
+    la, lb = oracle.leaves(an, chunk, eps, threads=8), oracle.leaves(bn, chunk, eps, threads=8)
+    na, nb = oracle.levels(la), oracle.levels(lb)
+    assert np.array_equal(gpu_tree_nodes(TA), na) and np.array_equal(gpu_tree_nodes(TB), nb)
+    ref_c = oracle.diff(na, nb, L)
+    ref_i = oracle.verify(an, bn, chunk, ref_c, eps)
+    nc, nd = counts.tolist()
+    assert np.array_equal(np_of(chunks[:nc]), ref_c) and np.array_equal(np_of(idx[:nd]), ref_i)
+    assert np.array_equal(gpu_tree_nodes(ck.tree_build(a, chunk, eps)), na)
