@@ -462,12 +462,16 @@ def main():
     ap.add_argument("--path", default="fused", choices=["fused", "unfused"],
                     help="fused: ckpt_compare_pair_async; unfused: build_batch + diff_verify_async")
     ap.add_argument("--snapshot", type=int, default=9, help="c4: snapshot index 0..9")
+    ap.add_argument("--chunk", type=int, default=4096, help="chunk bytes (configs[2] sweeps 512..65536)")
+    ap.add_argument("--eps", type=float, default=1e-6)
     ap.add_argument("--hash-block", type=int, default=16,
                     help="bytes per chained Murmur3F call: 16 = the paper's 128-bit blocks "
                          "(P:610, default); 0 = whole chunk (P:615-618 variant, R23)")
     args = ap.parse_args()
-    global CFG, N_PARTICLES, WORKLOAD, HASH_BLOCK, SNAPSHOT
+    global CFG, N_PARTICLES, WORKLOAD, HASH_BLOCK, SNAPSHOT, CHUNK, EPS
     CFG = args.config
+    CHUNK = args.chunk
+    EPS = args.eps
     HASH_BLOCK = args.hash_block
     SNAPSHOT = args.snapshot
     N_PARTICLES = CONFIGS[CFG]["n"]

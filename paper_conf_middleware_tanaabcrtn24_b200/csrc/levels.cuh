@@ -7,10 +7,12 @@
 // an exact subtree.
 //
 // Phase 1 (every CTA, no block barrier per level): a CTA of 8 warps takes an
-//   aligned group of 512 nodes of level ls of one array.  Each warp hashes its
-//   64 nodes up 6 levels with register shuffles (lane l holds node l after the
-//   first level; the right child of a level-k node comes from lane
-//   + 2^(k-2)), then warp 0 builds 3 more levels from the 8 warp roots.
+//   aligned group of 4096 nodes of level ls of one array.  Each thread hashes
+//   its own aligned 16 nodes up 4 levels in registers (15 hashes, every lane
+//   busy, 8-way independent at the first level); each warp then hashes its 32
+//   subtree roots up 5 more levels with register shuffles (the right child of
+//   a level-k node comes from lane + 2^(k-5)), and warp 0 builds the last 3
+//   levels from the 8 warp roots.
 // Phase 2 (last CTA of each tree, atomic ticket): loads the remaining level
 //   of every array into shared memory, builds all upper levels there, then
 //   the top tree over the array roots (R15).  Levels that do not fit in
@@ -24,8 +26,10 @@
 namespace ckpt {
 
 constexpr int kLevelThreads = 256;
-constexpr int kLog = 9;
-constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA
+constexpr int kLogT = 4;                     // levels each thread builds alone
+constexpr int kPerThread = 1 << kLogT;       // nodes of level ls per thread
+constexpr int kLog = 12;
+constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA (256 threads x 16)
 constexpr int kLevelSmemNodes = 1536;        // phase-2 shared memory in nodes (24 KiB)
 constexpr int kLevelSmem = kLevelSmemNodes * 16;
 constexpr int kMaxLevelTrees = 4;
@@ -170,25 +174,45 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         auto write = [&](int k, uint64_t jglob, uint4 v) {
             if (p.ls + k < h) p.nodes[p.off[(uint64_t)(p.ls + k) * na + a] + (start >> k) + jglob] = v;
         };
-        // warp w: nodes [64w, 64w+64) of the group
-        int mw = m0 - 64 * warp;
-        mw = mw < 0 ? 0 : (mw > 64 ? 64 : mw);
-        uint4 v = make_uint4(0u, 0u, 0u, 0u);
-        if (2 * lane < mw) {
-            v = src[64 * warp + 2 * lane];
-            if (2 * lane + 1 < mw) v = hash_children32(v, src[64 * warp + 2 * lane + 1]);
-            write(1, 32 * warp + lane, v);
+        // thread t: nodes [16t, 16t+16) of the group, 4 levels in registers
+        int mt = m0 - kPerThread * tid;
+        mt = mt < 0 ? 0 : (mt > kPerThread ? kPerThread : mt);
+        uint4 x[kPerThread / 2];
+#pragma unroll
+        for (int j = 0; j < kPerThread / 2; ++j) {
+            x[j] = make_uint4(0u, 0u, 0u, 0u);
+            if (2 * j < mt) {
+                x[j] = __ldg(src + kPerThread * tid + 2 * j);
+                if (2 * j + 1 < mt) x[j] = hash_children32(x[j], __ldg(src + kPerThread * tid + 2 * j + 1));
+                write(1, (kPerThread / 2) * tid + j, x[j]);
+            }
         }
-        int m1 = (mw + 1) >> 1;
-        v = warp_levels(v, m1, 2, 6, lane, [&](int k, int j, uint4 x) {
-            write(k, (uint64_t)(64 >> k) * warp + j, x);
+        int m = (mt + 1) >> 1;
+#pragma unroll
+        for (int k = 2; k <= kLogT; ++k) {
+#pragma unroll
+            for (int j = 0; j < (kPerThread >> k); ++j) {
+                if (j < ((m + 1) >> 1)) {
+                    if (2 * j + 1 < m) x[j] = hash_children32(x[2 * j], x[2 * j + 1]);
+                    else x[j] = x[2 * j];
+                    write(k, (uint64_t)(kPerThread >> k) * tid + j, x[j]);
+                }
+            }
+            m = (m + 1) >> 1;
+        }
+        // warp w: its 32 level-kLogT nodes, lane l holding node l, up 5 levels
+        int mw = ((m0 + kPerThread - 1) >> kLogT) - 32 * warp;
+        mw = mw < 0 ? 0 : (mw > 32 ? 32 : mw);
+        constexpr int kWarpSpan = 32 * kPerThread;          // group nodes per warp
+        const uint4 v = warp_levels(x[0], mw, kLogT + 1, kLogT + 5, lane, [&](int k, int j, uint4 y) {
+            write(k, (uint64_t)(kWarpSpan >> k) * warp + j, y);
         });
         if (lane == 0) s_root[warp] = v;
         __syncthreads();
         if (warp == 0) {
-            const int m6 = (m0 + 63) >> 6;       // valid warp roots
-            uint4 x = lane < m6 ? s_root[lane] : make_uint4(0u, 0u, 0u, 0u);
-            warp_levels(x, m6, 7, kLog, lane, [&](int k, int j, uint4 y) { write(k, j, y); });
+            const int m9 = (m0 + kWarpSpan - 1) / kWarpSpan;  // valid warp roots
+            uint4 y = lane < m9 ? s_root[lane] : make_uint4(0u, 0u, 0u, 0u);
+            warp_levels(y, m9, kLogT + 6, kLog, lane, [&](int k, int j, uint4 z) { write(k, j, z); });
         }
     }
     // ------------------------------ phase 2 ------------------------------
