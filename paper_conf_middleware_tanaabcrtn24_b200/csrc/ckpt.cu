@@ -859,7 +859,8 @@ static ckpt_status get_work(int dev, cudaStream_t s, size_t bytes, uint8_t **wor
 static ckpt_status launch_compact(int mode, const uint4 *la, const uint4 *lb, const uint8_t *flags,
                                   uint64_t n, uint64_t *out, uint64_t cap, uint64_t *count,
                                   cudaStream_t s, int sms, uint64_t base = 0) {
-    const uint64_t n_tiles = (n + kCompactTile - 1) / kCompactTile;
+    const uint64_t tile = mode == 0 ? compact_tile<0>() : compact_tile<1>();
+    const uint64_t n_tiles = (n + tile - 1) / tile;
     int dev = 0;
     CK_CUDA(cudaGetDevice(&dev));
     CompactParams p;

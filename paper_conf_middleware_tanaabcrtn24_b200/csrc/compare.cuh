@@ -114,9 +114,11 @@ __device__ __forceinline__ uint64_t draw_tile(unsigned long long *ticket, uint64
 // flag byte is set (MODE 1).  Output value = item index (a global chunk id).
 // ---------------------------------------------------------------------------
 constexpr int kCompactThreads = 256;
-constexpr int kCompactRows = 4;                           // rows of 32 items per warp
-constexpr int kCompactTile = kCompactThreads * kCompactRows;  // 1024 items
-constexpr int kRowsPerLane = kCompactRows * 8 / 32;       // scan: row counts per lane
+// rows of 32 items per warp: 4 for digest pairs (MODE 0, 32 B per item), 16 for
+// flag bytes (MODE 1: 4096-item tiles, so the look-back chain has 4x fewer
+// links; with 1 KB tiles it set the compaction time, e.g. 78 us for 8.4 M flags)
+template <int MODE> __host__ __device__ constexpr int compact_rows() { return MODE == 0 ? 4 : 16; }
+template <int MODE> __host__ __device__ constexpr int compact_tile() { return kCompactThreads * compact_rows<MODE>(); }
 
 struct CompactParams {
     const uint4 *leaf_a;
@@ -135,6 +137,9 @@ struct CompactParams {
 template <int MODE>
 __global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_constant__ CompactParams p) {
     pdl_enter();
+    constexpr int kCompactRows = compact_rows<MODE>();
+    constexpr int kCompactTile = compact_tile<MODE>();
+    constexpr int kRowsPerLane = kCompactRows * 8 / 32;       // scan: row counts per lane
     __shared__ uint32_t row_cnt[kCompactRows * 8];
     __shared__ uint32_t row_off[kCompactRows * 8];
     __shared__ uint64_t s_excl;

@@ -467,13 +467,28 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             static_assert(!PAIR || kCh == 1, "pair mode assumes one chain per lane");
             const int side = a >= P.pr.m ? 1 : 0;
             const uint64_t pt = task - (side ? P.pr.n_pair : 0);
-            // publish my leaves, then count in; the second of the pair does the compare
+            // publish my leaves, then count in; the second of the pair does the compare.
+#ifdef CKPT_PAIR_FENCES
             __threadfence();
             unsigned int order = 0;
             if (lane == 0) order = atomicInc(&P.pr.ctr[pt], 1u);
             order = __shfl_sync(0xffffffffu, order, 0);
             if (order == 1) {
                 __threadfence();
+#else
+            // The warp barrier orders every lane's leaf stores before lane 0's
+            // acq_rel atomic (release: cumulative over what the barrier made
+            // visible to it; acquire: the other run's leaves, published by its
+            // own release, are visible after the next barrier) -- no full fences.
+            __syncwarp();
+            unsigned int order = 0;
+            if (lane == 0)
+                asm volatile("atom.acq_rel.gpu.global.inc.u32 %0, [%1], 1;"
+                             : "=r"(order) : "l"(&P.pr.ctr[pt]) : "memory");
+            order = __shfl_sync(0xffffffffu, order, 0);
+            if (order == 1) {
+                __syncwarp();   // lane 0's acquire, then every lane's loads
+#endif
                 const LeafArray Pa = arrays[side ? a - P.pr.m : a + P.pr.m];   // the other run
                 const uint64_t c = c0 + lane;
                 if (c < A.n_leaves) {
