@@ -248,10 +248,17 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # CKPT_DIST_BACKEND=gloo + more ranks than GPUs: a functional test of the N>1 path on one
+    # GPU (ranks share it; timings are not meaningful).  Production: one rank per GPU, NCCL.
+    backend = os.environ.get("CKPT_DIST_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
     torch.cuda.set_device(local)
     group = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     import paper_conf_middleware_tanaabcrtn24_b200 as ck
     from paper_conf_middleware_tanaabcrtn24_b200 import dist as ckd
     import synth
