@@ -314,13 +314,25 @@ def tree_from_digests(digests: torch.Tensor, stream=None) -> Tree:
     return Tree(out.value, [d], F32, 16, 0.0, sp)
 
 
-def tree_deserialize(data: bytes, stream=None) -> Tree:
-    """Load a serialised tree onto the current device (ckpt_tree_deserialize)."""
-    buf = ctypes.create_string_buffer(bytes(data), len(data))
+def _host_blob(data):
+    """(pointer, size) of a serialised tree given as bytes or a contiguous CPU uint8 tensor (pin it
+    for a fast upload; bytes are copied into a ctypes buffer that lives as long as the call)."""
+    if isinstance(data, torch.Tensor):
+        if data.is_cuda or data.dtype != torch.uint8 or not data.is_contiguous():
+            raise ValueError("a serialised tree tensor must be a contiguous CPU uint8 tensor")
+        return ctypes.c_void_p(data.data_ptr()), data.numel()
+    b = bytes(data)
+    buf = ctypes.create_string_buffer(b, len(b))
+    _host_blob.keep = buf
+    return ctypes.cast(buf, ctypes.c_void_p), len(b)
+
+
+def tree_deserialize(data, stream=None) -> Tree:
+    """Load a serialised tree (bytes or CPU uint8 tensor) onto the current device."""
+    buf, nbytes = _host_blob(data)
     out = ctypes.c_void_p()
     sp = _stream_ptr(stream)
-    _check(lib().ckpt_tree_deserialize(ctypes.cast(buf, ctypes.c_void_p), len(data), sp,
-                                       ctypes.byref(out)), "ckpt_tree_deserialize")
+    _check(lib().ckpt_tree_deserialize(buf, nbytes, sp, ctypes.byref(out)), "ckpt_tree_deserialize")
     t = Tree(out.value, [], F32, 0, 0.0, sp)
     t.dtype, t.chunk_bytes, t.eps, _ = t.params()
     return t
@@ -346,15 +358,16 @@ def compare_saved(saved_a: bytes, arrays_a, arrays_b, chunks: torch.Tensor, idx:
         if not t.is_contiguous():
             raise ValueError("arrays must be contiguous")
     code = _check_arrays(lb)
-    if len(saved_a) >= 16 and int.from_bytes(bytes(saved_a[12:16]), "little") != code:
+    buf, nbytes = _host_blob(saved_a)
+    hdr = ctypes.string_at(buf, 16) if nbytes >= 16 else b""
+    if len(hdr) == 16 and int.from_bytes(hdr[12:16], "little") != code:
         raise ValueError("run B's dtype differs from the stored tree's")
     pa, _k1 = _ptr_array(la)
     pb, _k2 = _ptr_array(lb)
     pn, _k3 = _u64_array([t.numel() for t in lb])
-    buf = ctypes.create_string_buffer(bytes(saved_a), len(saved_a))
     ta, tb = ctypes.c_void_p(), ctypes.c_void_p()
     sp = _stream_ptr(stream)
-    _check(lib().ckpt_compare_saved(ctypes.cast(buf, ctypes.c_void_p), len(saved_a), pa, pb, pn,
+    _check(lib().ckpt_compare_saved(buf, nbytes, pa, pb, pn,
                                     len(lb), chunks.data_ptr(), chunks.numel(), idx.data_ptr(),
                                     idx.numel(), counts.data_ptr(), sp, ctypes.byref(ta),
                                     ctypes.byref(tb)), "ckpt_compare_saved")
