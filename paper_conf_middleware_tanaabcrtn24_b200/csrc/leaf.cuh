@@ -403,7 +403,9 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
                             uint64_t rem = A.nbytes - off;
                             const uint64_t crem = C - rel;
                             if (crem < rem) rem = crem;
-                            nb = rem >= 16 ? 16u : (uint32_t)rem;
+                            // a piece shorter than 16 bytes is the chunk's Murmur3F tail,
+                            // hashed from global memory (chain_tail / wide_end): not staged
+                            nb = rem >= 16 ? 16u : 0u;
                         }
                         const uint8_t *sp = nb ? (A.data + off) : A.data;
                         cp_async16(slot + qq * kPitch + my_sub * 16, sp, nb);

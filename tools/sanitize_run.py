@@ -1,0 +1,67 @@
+#!/usr/bin/env python
+"""Small workloads through every libckpt entry point, for compute-sanitizer
+(memcheck / racecheck / synccheck / initcheck).  Checks results against the oracle too."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import oracle  # noqa: E402
+import paper_conf_middleware_tanaabcrtn24_b200 as ck  # noqa: E402
+import synth  # noqa: E402
+
+torch.cuda.set_device(0)
+pair = synth.c1_pair(n=(1 << 16) + 77, seed=5, device="cuda")          # ragged tail
+a, b = pair.a[0], pair.b[0]
+C, eps = 4096, pair.eps
+an, bn = a.cpu().numpy(), b.cpu().numpy()
+ref_c = oracle.diff(oracle.levels(oracle.leaves(an, C, eps)), oracle.levels(oracle.leaves(bn, C, eps)),
+                    oracle.n_chunks(an.size, 0, C))
+ref_i = oracle.verify(an, bn, C, ref_c, eps)
+L = oracle.n_chunks(an.size, 0, C)
+# unfused: build, BFS diff from the leaves and from a mid level, verify
+ta, tb = ck.tree_build(a, C, eps), ck.tree_build(b, C, eps)
+assert np.array_equal(ck.tree_diff(ta, tb).cpu().numpy(), ref_c)
+for T in (1, 7):
+    ch = torch.empty(L, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    ck.tree_diff_async(ta, tb, ch, cnt, T=T)
+    assert np.array_equal(ch[: int(cnt.item())].cpu().numpy(), ref_c)
+idx, n = ck.verify(a, b, torch.as_tensor(ref_c, device="cuda"), C, eps)
+assert np.array_equal(idx.cpu().numpy(), ref_i)
+# fused pair path, 16-byte and whole-chunk hash blocks
+for hb in (16, 0):
+    ch = torch.empty(L, dtype=torch.int64, device="cuda")
+    ix = torch.empty(a.numel(), dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async([a], [b], C, eps, ch, ix, cnt, hash_block=hb)
+    TA.wait(); TB.wait()
+    nc, nd = cnt.tolist()
+    assert np.array_equal(ch[:nc].cpu().numpy(), ref_c) and np.array_equal(ix[:nd].cpu().numpy(), ref_i)
+# host paths, persistence, streaming
+out = ck.compare_host([a.cpu()], [b.cpu()], C, eps)
+assert np.array_equal(out[0].numpy(), ref_i)
+out = ck.compare_stream([a.cpu().pin_memory()], [b.cpu().pin_memory()], C, eps, segment_bytes=3 * C)
+assert np.array_equal(out[1].numpy(), ref_i)
+blob = ta.serialize()
+t2 = ck.tree_deserialize(blob)
+assert t2.root() == ta.root()
+ch = torch.empty(L, dtype=torch.int64, device="cuda")
+ix = torch.empty(a.numel(), dtype=torch.int64, device="cuda")
+cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+ck.compare_saved(blob, [a.cpu().pin_memory()], [b], ch, ix, cnt)
+torch.cuda.synchronize()
+nc, nd = cnt.tolist()
+assert np.array_equal(ix[:nd].cpu().numpy(), ref_i)
+# multi-array checkpoint (c5 shape, small) through the fused path
+p5 = synth.c5_pair(n_ranks=1, n_particles=1 << 13, seed=3, device="cuda")
+L5 = sum(-(-t.numel() * 4 // C) for t in p5.a)
+ch = torch.empty(L5, dtype=torch.int64, device="cuda")
+ix = torch.empty(sum(t.numel() for t in p5.a), dtype=torch.int64, device="cuda")
+cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+TA, TB = ck.compare_pair_async(p5.a, p5.b, C, p5.eps, ch, ix, cnt)
+TA.wait(); TB.wait()
+torch.cuda.synchronize()
+print("sanitize workload ok", ck.launch_count(), "launches")
