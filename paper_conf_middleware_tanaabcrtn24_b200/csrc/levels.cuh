@@ -25,16 +25,25 @@
 
 namespace ckpt {
 
+#ifdef CKPT_LV_OLD
 constexpr int kLevelThreads = 256;
 constexpr int kLogT = 4;                     // levels each thread builds alone
 constexpr int kPerThread = 1 << kLogT;       // nodes of level ls per thread
 constexpr int kLog = 12;
 constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA (256 threads x 16)
+#else
+constexpr int kLevelThreads = 512;
+constexpr int kLog = 11;
+constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA (512 threads x 4)
+#endif
 constexpr int kLevelSmemNodes = 1536;        // phase-2 shared memory in nodes (24 KiB)
 constexpr int kLevelSmem = kLevelSmemNodes * 16;
 constexpr int kMaxLevelTrees = 4;
 
-constexpr int kLevelInlineWords = 512;       // 4 KiB of tree metadata in the kernel params
+#ifndef CKPT_LEVEL_INLINE
+#define CKPT_LEVEL_INLINE 512
+#endif
+constexpr int kLevelInlineWords = CKPT_LEVEL_INLINE;   // 4 KiB of tree metadata in the kernel params
 
 // Per-tree launch record.  The metadata tables live in one blob (layout below)
 // that is either inline in the kernel parameters (small trees: no H2D copy;
@@ -134,9 +143,14 @@ __device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 
 __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_constant__ LevelBatch pb) {
     pdl_enter();
     extern __shared__ __align__(16) uint4 sm[];
+#ifdef CKPT_LV_OLD
     __shared__ uint4 s_root[kLevelThreads / 32];
+#endif
     __shared__ unsigned int s_ticket;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int tid = threadIdx.x;
+#ifdef CKPT_LV_OLD
+    const int lane = tid & 31, warp = tid >> 5;
+#endif
     int ti = 0;
     while (ti + 1 < pb.n && blockIdx.x >= pb.cta_begin[ti + 1]) ++ti;
     const LevelParams &lp = pb.t[ti];
@@ -162,6 +176,7 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         for (uint32_t w = tid; w < lp.meta_words; w += kLevelThreads) dst[w] = pb.blob[lp.inl + w];
     }
     // ------------------------------ phase 1 ------------------------------
+#ifdef CKPT_LV_OLD
     {
         const uint64_t gid = blockIdx.x - pb.cta_begin[ti];
         const int a = find_le(p.gbegin, na, gid);
@@ -215,15 +230,77 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
             warp_levels(y, m9, kLogT + 6, kLog, lane, [&](int k, int j, uint4 z) { write(k, j, z); });
         }
     }
+#else
+    {
+        // Passes of two levels through shared memory: in pass r/2 the first
+        // ceil(cnt/4) threads each take 4 consecutive level-r nodes of the
+        // group (cnt valid), hash them up to one level-(r+2) node (2 + 1
+        // hashes, the first two independent) and store it for the next pass.
+        // Every pass but the last few keeps whole warps busy, so the CTA's
+        // 2047 hashes cost ~2047/32 warp-hashes instead of a lane-halving
+        // shuffle tree, and 16 warps per CTA hide the hash latency.
+        const uint64_t gid = blockIdx.x - pb.cta_begin[ti];
+        const int a = find_le(p.gbegin, na, gid);
+        const uint64_t g = gid - p.gbegin[a];
+        const uint64_t n0 = p.cnt[(uint64_t)p.ls * na + a];
+        const uint64_t start = g * kGroup;
+        const int m0 = (int)((n0 - start) < (uint64_t)kGroup ? (n0 - start) : (uint64_t)kGroup);
+        const int h = (int)p.height[a];
+        const uint4 *src = p.nodes + p.off[(uint64_t)p.ls * na + a] + start;
+        auto write = [&](int k, uint64_t j, uint4 v) {
+            if (p.ls + k < h) p.nodes[p.off[(uint64_t)(p.ls + k) * na + a] + (start >> k) + j] = v;
+        };
+        uint4 *buf[2] = {sm, sm + kLevelThreads};       // ping-pong: 512 + 128 nodes
+        int cnt = m0;
+        for (int r = 0; r < kLog; r += 2) {
+            const bool two = r + 2 <= kLog;
+            const int need = two ? (cnt + 3) >> 2 : (cnt + 1) >> 1;
+            const uint4 *in = buf[(r >> 1) & 1];
+            uint4 *out = buf[((r >> 1) + 1) & 1];
+            if (tid < need) {
+                const int per = two ? 4 : 2;
+                int mt = cnt - per * tid;
+                mt = mt > per ? per : mt;
+                uint4 x[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    x[j] = make_uint4(0u, 0u, 0u, 0u);
+                    if (j < mt) x[j] = r == 0 ? __ldg(src + per * tid + j) : in[per * tid + j];
+                }
+                const uint4 y0 = mt >= 2 ? hash_children32(x[0], x[1]) : x[0];
+                write(r + 1, (uint64_t)(per / 2) * tid, y0);
+                if (two) {
+                    uint4 y1 = make_uint4(0u, 0u, 0u, 0u);
+                    if (mt >= 3) {
+                        y1 = mt == 4 ? hash_children32(x[2], x[3]) : x[2];
+                        write(r + 1, (uint64_t)2 * tid + 1, y1);
+                    }
+                    const uint4 z = mt >= 3 ? hash_children32(y0, y1) : y0;
+                    write(r + 2, (uint64_t)tid, z);
+                    out[tid] = z;
+                } else {
+                    out[tid] = y0;
+                }
+            }
+            cnt = need;
+            __syncthreads();
+        }
+    }
+#endif
     // ------------------------------ phase 2 ------------------------------
+    // Last-CTA hand-off without sequentially consistent fences (MEMBAR.SC.GPU
+    // costs microseconds): the barrier orders every thread's node stores before
+    // thread 0's acq_rel atomic, whose release is cumulative over them; in the
+    // last CTA the same atomic acquires every other CTA's release, and the
+    // next barrier extends that to all of its threads.
     __syncthreads();
     if (tid == 0) {
-        __threadfence();
-        s_ticket = atomicAdd(p.ticket, 1u);
+        unsigned int t;
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(t) : "l"(p.ticket) : "memory");
+        s_ticket = t;
     }
     __syncthreads();
     if (s_ticket != p.n_groups - 1) return;
-    __threadfence();
     int F = p.ls + kLog;                       // highest level phase 1 completed
     if (F > p.n_levels - 1) F = p.n_levels - 1;
     if (F + 1 <= p.n_levels - 1) {

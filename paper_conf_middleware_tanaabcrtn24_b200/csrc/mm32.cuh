@@ -83,10 +83,40 @@ __device__ __forceinline__ U64p add64(U64p a, U64p b) {
 // (lo*5 + c) and adds hi*5 with one IMAD + IADD3.  (An inline-asm mad.wide with
 // an immediate multiplier was split by ptxas into IMAD.WIDE + IADD3 + IMAD.X:
 // 2 more instructions per block, measured 1.8% slower in the leaf kernel.)
+#if defined(CKPT_M5ASM)
+__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
+    U64p r;
+    asm("{\n\t.reg .u64 p;\n\t"
+        "mad.wide.u32 p, %2, 5, %4;\n\t"
+        "mov.b64 {%0, %1}, p;\n\t"
+        "mad.lo.u32 %1, %3, 5, %1;\n\t}"
+        : "=r"(r.lo), "=r"(r.hi)
+        : "r"(h.lo), "r"(h.hi), "l"(c));
+    return r;
+}
+#endif
+// h*5 + c on the ALU pipe: (h << 2) + h + c
+__device__ __forceinline__ U64p mul5_add_alu(U64p h, uint64_t c) {
+    U64p r;
+    asm("{\n\t.reg .u32 s, t;\n\t"
+        "shf.l.wrap.b32 t, %2, %3, 2;\n\t"
+        "shl.b32 s, %2, 2;\n\t"
+        "add.cc.u32 s, s, %2;\n\t"
+        "addc.u32 t, t, %3;\n\t"
+        "add.cc.u32 %0, s, %4;\n\t"
+        "addc.u32 %1, t, 0;\n\t}"
+        : "=r"(r.lo), "=r"(r.hi)
+        : "r"(h.lo), "r"(h.hi), "r"((uint32_t)c));
+    return r;
+}
+#if defined(CKPT_M5LEA)
+__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) { return mul5_add_alu(h, c); }
+#elif !defined(CKPT_M5ASM)
 __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
     const uint64_t x = (((uint64_t)h.hi << 32) | h.lo) * 5ull + c;
     return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
 }
+#endif
 
 #ifdef CKPT_XS_IMAD
 // hi >> 1 as IMAD.HI.U32(hi, 2^31): moves the shift from the ALU to the FMA pipe
@@ -126,7 +156,11 @@ __device__ __forceinline__ void mm3p_hstep(U64p &h1, U64p &h2, U64p k1, U64p k2,
     h1 = xor64(h1, k1);
     h1 = rotl_lt32<27>(h1);
     h1 = add64(h1, h2);
+#ifdef CKPT_M5MIX
+    h1 = mul5_add_alu(h1, m1);   // ALU pipe: balances the FMA-heavy pipe (IMAD.WIDE = 2 slots)
+#else
     h1 = mul5_add(h1, m1);   // m1 = 0x52dce729
+#endif
     h2 = xor64(h2, k2);
     h2 = rotl_lt32<31>(h2);
     h2 = add64(h2, h1);
@@ -141,6 +175,28 @@ __device__ __forceinline__ void mm3p_body(U64p &h1, U64p &h2, U64p k1, U64p k2, 
 }
 
 // Murmur3F finalisation for a total length `len` < 2^32.
+#ifdef CKPT_ADD3
+// a + b + b (h2 += h1 right after h1 += h2, as one 3-input add off h1's critical path)
+__device__ __forceinline__ U64p add64_abb(U64p a, U64p b) {
+    const uint64_t x = (((uint64_t)a.hi << 32) | a.lo) + (((uint64_t)b.hi << 32) | b.lo) +
+                       (((uint64_t)b.hi << 32) | b.lo);
+    return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
+}
+__device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
+    h1.lo ^= len;
+    h2.lo ^= len;
+    {
+        const U64p a = add64(h1, h2), b = add64_abb(h1, h2);
+        h1 = a; h2 = b;
+    }
+    h1 = fmix64p(h1);
+    h2 = fmix64p(h2);
+    {
+        const U64p a = add64(h1, h2), b = add64_abb(h1, h2);
+        h1 = a; h2 = b;
+    }
+}
+#else
 __device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
     h1.lo ^= len;
     h2.lo ^= len;
@@ -151,6 +207,7 @@ __device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
     h1 = add64(h1, h2);
     h2 = add64(h2, h1);
 }
+#endif
 
 // One chained 16-byte block: (h1,h2) <- Murmur3F(k1||k2, len 16, state (h1,h2)).
 __device__ __forceinline__ void mm3p_block16(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,

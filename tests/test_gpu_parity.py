@@ -74,6 +74,32 @@ def test_tree_bit_exact(n, dtype, chunk, eps):
     assert t.n_leaves == L
 
 
+# Interior levels (K2) over leaf counts around its CTA group (2048 nodes) and pass
+# boundaries (4 nodes per thread, two levels per pass): every node vs the oracle's
+# level construction (Alg. 1, R13 promotion of an odd last node).
+@pytest.mark.parametrize("L", [1, 2, 3, 4, 5, 7, 8, 9, 31, 33, 511, 513, 2047, 2048, 2049, 2050,
+                               4095, 4097, 6143, 65537, 300_001])
+def test_levels_from_digests_bit_exact(L):
+    g = torch.Generator().manual_seed(L)
+    d = torch.randint(0, 256, (L, 16), dtype=torch.uint8, generator=g)
+    t = ck.tree_from_digests(d.cuda())
+    got = gpu_tree_nodes(t)
+    ref = oracle.levels(d.numpy())
+    assert got.shape == ref.shape
+    bad = np.nonzero(np.any(got != ref, axis=1))[0]
+    assert bad.size == 0, f"{bad.size} nodes differ, first {bad[:5]}"
+
+
+# Multi-array batch: arrays of different heights whose groups end mid-pass.
+def test_levels_multi_array_ragged_groups():
+    sizes = [4097 * 4096, 1 * 4096, 2049 * 4096 + 8, 3 * 4096]
+    arrs = [synth.uniform(77 + i, nb // 4, "cuda") for i, nb in enumerate(sizes)]
+    t = ck.tree_build(arrs, 4096, 1e-5)
+    for i, x in enumerate(arrs):
+        ref, _ = oracle_tree(np_of(x), 4096, 1e-5)
+        assert np.array_equal(gpu_tree_nodes(t, i), ref), f"array {i}"
+
+
 SPECIALS32 = np.array([0.0, -0.0, np.inf, -np.inf, np.nan, 1e-45, -1e-45, 1.17549435e-38,
                        -1.17549435e-38, 3.4028235e38, -3.4028235e38, 1.0, -1.0, 0.5, -0.5,
                        2.0 ** 24, -(2.0 ** 24), 2.0 ** 31, 2.0 ** 40, -(2.0 ** 60), 1e-5, -1e-5,

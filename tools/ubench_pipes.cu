@@ -84,6 +84,26 @@ __global__ void k(uint32_t *out, uint32_t seed) {
 #define S(x) asm volatile("prmt.b32 %0, %0, %1, 0x3210;" : "+r"(x) : "r"(b));
             CHAIN8(S)
 #undef S
+        } else if (OP == 17) {  // 2 IMAD imm + 1 LOP3
+#define S(x) asm volatile("mad.lo.u32 %0, %0, 0x2745937f, %1;\n\tmad.lo.u32 %0, %0, 0x114253d5, %2;\n\tlop3.b32 %0, %0, %1, %2, 0x96;" : "+r"(x) : "r"(b), "r"(c));
+            CHAIN8(S)
+#undef S
+        } else if (OP == 18) {  // SHF + IMAD imm
+#define S(x) asm volatile("shf.l.wrap.b32 %0, %0, %1, 13;\n\tmad.lo.u32 %0, %0, 0x2745937f, %1;" : "+r"(x) : "r"(b));
+            CHAIN8(S)
+#undef S
+        } else if (OP == 19) {  // IMAD.WIDE imm + LOP3
+#define S(x) asm volatile("{.reg .u64 p; mul.wide.u32 p, %0, 0x2745937f; cvt.u32.u64 %0, p;}\n\tlop3.b32 %0, %0, %1, %2, 0x96;" : "+r"(x) : "r"(b), "r"(c));
+            CHAIN8(S)
+#undef S
+        } else if (OP == 20) {  // 3 IMAD imm + 1 LOP3 + 1 SHF
+#define S(x) asm volatile("mad.lo.u32 %0, %0, 0x2745937f, %1;\n\tmad.lo.u32 %0, %0, 0x114253d5, %2;\n\tlop3.b32 %0, %0, %1, %2, 0x96;\n\tmad.lo.u32 %0, %0, 0x1a85ec53, %2;\n\tshf.l.wrap.b32 %0, %0, %1, 13;" : "+r"(x) : "r"(b), "r"(c));
+            CHAIN8(S)
+#undef S
+        } else if (OP == 21) {  // IMAD.MOV-free 2-reg IMAD imm x*imm (no addend)
+#define S(x) asm volatile("mul.lo.u32 %0, %0, 0x2745937f;" : "+r"(x));
+            CHAIN8(S)
+#undef S
         } else if (OP == 13) {  // FFMA (reference)
 #define S(x) asm volatile("fma.rn.f32 %0, %0, 1.0001, 0.5;" : "+f"(f##x));
             S(0) S(1) S(2) S(3) S(4) S(5) S(6) S(7)
@@ -138,5 +158,10 @@ int main() {
     run<14>("IMAD.WIDE x*1+pair (64b add)", sms, out, 1);
     run<15>("IMAD x*32+y", sms, out, 1);
     run<16>("PRMT", sms, out, 1);
+    run<17>("2 IMAD imm + LOP3 (3)", sms, out, 3);
+    run<18>("SHF + IMAD imm (2)", sms, out, 2);
+    run<19>("IMAD.WIDE imm + LOP3 (2)", sms, out, 2);
+    run<20>("3 IMADi+LOP3+SHF (5)", sms, out, 5);
+    run<21>("IMUL imm", sms, out, 1);
     return 0;
 }
