@@ -1,5 +1,7 @@
 #!/usr/bin/env python
-"""Per-kernel timeline of bench steps (events around every library launch)."""
+"""Per-kernel timeline of bench steps (events around every library launch).
+
+usage: step_timeline.py [N_STEPS] [--unfused]   (default: the fused pair path bench.py times)"""
 import os
 import sys
 
@@ -17,9 +19,15 @@ idx = torch.empty(sum(t.numel() for t in A), dtype=torch.int64, device="cuda")
 counts = torch.zeros(2, dtype=torch.int64, device="cuda")
 
 
+FUSED = "--unfused" not in sys.argv     # the bench path: ckpt_compare_pair_async
+
+
 def step():
-    TA, TB = ck.tree_build_batch([A, B], 4096, 1e-6)
-    ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)
+    if FUSED:
+        TA, TB = ck.compare_pair_async(A, B, 4096, 1e-6, chunks, idx, counts)
+    else:
+        TA, TB = ck.tree_build_batch([A, B], 4096, 1e-6)
+        ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)
     TA.wait()
     TB.wait()
     return TA, TB
@@ -31,7 +39,8 @@ torch.cuda.synchronize()
 ck.profile_reset()
 ck.profile_enable(True)
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-n_steps = int(sys.argv[1]) if len(sys.argv) > 1 else 3
+args = [a for a in sys.argv[1:] if not a.startswith("--")]
+n_steps = int(args[0]) if args else 3
 e0.record()
 for _ in range(n_steps):
     keep = step()
