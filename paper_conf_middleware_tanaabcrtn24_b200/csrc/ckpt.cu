@@ -569,6 +569,8 @@ struct Scratch {
     size_t pair_cap = 0;
     uint8_t *pair_flags = nullptr;      // fused pair mode: one flag byte per chunk
     size_t flags_cap = 0;
+    uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
+    size_t tile_pairs = 0;              // pair-tasks the buffers hold
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -595,6 +597,39 @@ static bool leaf_static_tasks() {
         return e && e[0] == '1';
     }();
     return on;
+}
+
+// K1 tile-compaction buffers for n_pair pair-tasks (leaf.cuh PairParams):
+// [tctr: n_tiles u32, zeroed once; self-resetting] [tagg: n_tiles u32]
+// [tmask: n_pair u32] [tbase: n_pair u64] [tids: n_tiles * kTileTasks * 32 u64]
+static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, PairParams *pp) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    Scratch &sc = g_scr[std::make_pair(dev, s)];
+    n_pair = std::max<uint64_t>(n_pair, 1);
+    auto layout_of = [](uint64_t np, size_t o[5]) {
+        const uint64_t nt = (np + kTileTasks - 1) / kTileTasks;
+        o[0] = 0;
+        o[1] = align256(nt * 4);
+        o[2] = o[1] + align256(nt * 4);
+        o[3] = o[2] + align256(np * 4);
+        o[4] = o[3] + align256(np * 8);
+        return o[4] + nt * kTileTasks * 32 * 8;
+    };
+    size_t o[5];
+    if (sc.tile_pairs < n_pair) {
+        if (sc.tile) CK_CUDA(cudaFreeAsync(sc.tile, s));
+        sc.tile_pairs = std::max<uint64_t>(n_pair, 2 * sc.tile_pairs);
+        const size_t bytes = layout_of(sc.tile_pairs, o);
+        CK_CUDA(cudaMallocAsync((void **)&sc.tile, bytes, s));
+        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters
+    }
+    layout_of(sc.tile_pairs, o);
+    pp->tctr = (unsigned int *)(sc.tile + o[0]);
+    pp->tagg = (uint32_t *)(sc.tile + o[1]);
+    pp->tmask = (uint32_t *)(sc.tile + o[2]);
+    pp->tbase = (uint64_t *)(sc.tile + o[3]);
+    pp->tids = (uint64_t *)(sc.tile + o[4]);
+    return CKPT_OK;
 }
 
 // Zero-initialised pair-task counters (they return to 0 after every launch).
@@ -1160,6 +1195,9 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     pp.m = (int)n_arrays;
     // flag bytes live in their own per-stream buffer (verify's work buffer may regrow)
     CK_TRY(get_pair_flags(dev, s, L, &pp.flags));
+    uint64_t n_pair = 0;                          // pair-tasks: kRows chunks of one array each
+    for (uint32_t k = 0; k < n_arrays; ++k) n_pair += ((n[k] * esz + chunk_bytes - 1) / chunk_bytes + kRows - 1) / kRows;
+    CK_TRY(get_tile_scratch(dev, s, n_pair, &pp));
     std::vector<const void *> data(2 * (size_t)n_arrays);
     std::vector<uint64_t> nn(2 * (size_t)n_arrays);
     for (uint32_t k = 0; k < n_arrays; ++k) {
@@ -1171,8 +1209,22 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     ckpt_tree *trees[2] = {nullptr, nullptr};
     CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
                             trees, &pp));
-    ckpt_status st = launch_compact(1, nullptr, nullptr, pp.flags, L, chunks, chunks_cap, counts_dev, s,
-                                    di.sms);
+    // the ordered chunk list from K1's per-tile compaction (one gather pass)
+    ckpt_status st = CKPT_OK;
+    {
+        TileGatherParams g;
+        g.tagg = pp.tagg;
+        g.tids = pp.tids;
+        g.n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
+        g.tile_ids = (uint64_t)kTileTasks * 32;
+        g.out = chunks;
+        g.cap = chunks_cap;
+        g.count = counts_dev;
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(g.n_tiles, (uint64_t)di.sms * 8));
+        ProfScope prof(2, s);
+        if (launch_k(tile_gather_kernel, dim3(grid), dim3(kGatherThreads), 0, s, g) != cudaSuccess)
+            st = fail(CKPT_ECUDA, "tile gather launch");
+    }
     if (st == CKPT_OK)
         st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
                          idx, idx_cap, counts_dev + 1, s, before_emit);

@@ -203,6 +203,52 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_c
 }
 
 // ---------------------------------------------------------------------------
+// Ordered chunk list of the fused pair path from K1's tile compaction
+// (leaf.cuh, tile_compact): tile t's ids go to out[sum of tagg[0..t) ..].
+// One pass, no look-back; CTA 0 also writes the total count.
+// ---------------------------------------------------------------------------
+struct TileGatherParams {
+    const uint32_t *tagg;         // [n_tiles] flagged chunks per tile
+    const uint64_t *tids;         // [n_tiles * tile_ids] tile-compacted chunk ids
+    uint64_t n_tiles;
+    uint64_t tile_ids;            // id slots per tile
+    uint64_t *out;
+    uint64_t cap;
+    uint64_t *count;              // device: total flagged chunks
+};
+
+constexpr int kGatherThreads = 256;
+
+__global__ void __launch_bounds__(kGatherThreads) tile_gather_kernel(const __grid_constant__ TileGatherParams p) {
+    pdl_enter();
+    __shared__ uint64_t s_red[kGatherThreads / 32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    auto block_sum = [&](uint64_t upto) -> uint64_t {   // sum of tagg[0..upto)
+        uint64_t x = 0;
+        for (uint64_t i = threadIdx.x; i < upto; i += kGatherThreads) x += p.tagg[i];
+        x = warp_sum_u64(x);
+        if (lane == 0) s_red[warp] = x;
+        __syncthreads();
+        uint64_t t = 0;
+#pragma unroll
+        for (int w = 0; w < kGatherThreads / 32; ++w) t += s_red[w];
+        __syncthreads();
+        return t;
+    };
+    if (blockIdx.x == 0) {
+        const uint64_t total = block_sum(p.n_tiles);
+        if (threadIdx.x == 0) *p.count = total;
+    }
+    for (uint64_t t = blockIdx.x; t < p.n_tiles; t += gridDim.x) {
+        const uint64_t base = block_sum(t);
+        const uint32_t n = p.tagg[t];
+        const uint64_t *src = p.tids + t * p.tile_ids;
+        for (uint32_t k = threadIdx.x; k < n; k += kGatherThreads)
+            if (base + k < p.cap) p.out[base + k] = src[k];
+    }
+}
+
+// ---------------------------------------------------------------------------
 // BFS steps for a start level above the leaves.
 // Frontier entry: array (20 bits) | level (6 bits) | node (38 bits).
 // ---------------------------------------------------------------------------

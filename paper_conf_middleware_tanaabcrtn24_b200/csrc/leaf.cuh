@@ -230,12 +230,53 @@ constexpr int kLeafInline = 16;
 // the diff at start level 0 happens inside K1.  (Marking the flagged chunks'
 // elements here as well was measured slower than K4a: flagged chunks cluster,
 // so the marking serialises in the few warps that own them.)
+// Tile compaction (optional, tmask != null): pair-tasks are grouped in tiles
+// of kTileTasks; the warp that completes a tile's last pair-task (a
+// self-resetting acq_rel counter per tile) writes the tile's flagged chunk ids,
+// ascending, to tids[tile * kTileTasks * 32 ..] and their number to tagg[tile].
+// The ordered chunk list is then one gather pass (tile_gather_kernel) with no
+// look-back: the digest compare, the flags AND their compaction happen in K1.
+constexpr int kTileTasks = 128;                // pair-tasks per tile (4096 chunks)
 struct PairParams {
     uint8_t *flags;               // [L] 1 if the chunk's leaf digests differ
     unsigned int *ctr;            // [n_pair] 0 between launches (atomicInc wraps 1 -> 0)
     uint64_t n_pair;              // pair-tasks (A's warp tasks)
     int m;                        // arrays per checkpoint
+    uint32_t *tmask;              // [n_pair] differing-chunk mask per pair-task, or null
+    uint64_t *tbase;              // [n_pair] global chunk id of the pair-task's chunk 0
+    unsigned int *tctr;           // [n_tiles] 0 between launches
+    uint32_t *tagg;               // [n_tiles] flagged chunks per tile
+    uint64_t *tids;               // [n_tiles * kTileTasks * 32] tile-compacted chunk ids
 };
+
+// The tile's ordered chunk ids, by the warp that completed its last pair-task
+// (after an acquire of every pair-task's release).
+__device__ __noinline__ void tile_compact(const PairParams &pr, uint64_t tile, int lane) {
+    const uint64_t t0 = tile * kTileTasks;
+    const uint64_t t1 = (t0 + kTileTasks) < pr.n_pair ? t0 + kTileTasks : pr.n_pair;
+    uint64_t *dst = pr.tids + t0 * 32;
+    uint32_t run = 0;
+    for (uint64_t k = t0; k < t1; k += 32) {
+        const uint64_t pt = k + lane;
+        uint32_t m = 0;
+        uint64_t b = 0;
+        if (pt < t1) {
+            m = __ldcg(pr.tmask + pt);
+            b = __ldcg(reinterpret_cast<const unsigned long long *>(pr.tbase) + pt);
+        }
+        uint32_t x = __popc(m);
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        const uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
+        uint32_t pos = run + x - __popc(m);
+        for (uint32_t mm = m; mm; mm &= mm - 1) dst[pos++] = b + (uint64_t)(__ffs(mm) - 1);
+        run += tot;
+    }
+    if (lane == 0) pr.tagg[tile] = run;
+}
 
 struct LeafParams {
     const LeafArray *arrays;      // device table when n_arrays > kLeafInline
@@ -493,11 +534,30 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
 #endif
                 const LeafArray Pa = arrays[side ? a - P.pr.m : a + P.pr.m];   // the other run
                 const uint64_t c = c0 + lane;
+                bool differ = false;
                 if (c < A.n_leaves) {
                     const uint4 o = __ldcg(Pa.out + c);
-                    const bool differ = (o.x != h1[0].lo) | (o.y != h1[0].hi) | (o.z != h2[0].lo) |
-                                        (o.w != h2[0].hi);
+                    differ = (o.x != h1[0].lo) | (o.y != h1[0].hi) | (o.z != h2[0].lo) | (o.w != h2[0].hi);
                     P.pr.flags[A.chunk_base + c] = differ ? 1 : 0;
+                }
+                if (P.pr.tmask) {
+                    // publish this pair-task's mask, then count it into its tile
+                    const uint32_t m = __ballot_sync(0xffffffffu, differ);
+                    const uint64_t tile = pt / kTileTasks;
+                    const uint64_t rest = P.pr.n_pair - tile * kTileTasks;
+                    const unsigned int in_tile = (unsigned int)(rest < kTileTasks ? rest : kTileTasks);
+                    unsigned int done = 0;
+                    if (lane == 0) {
+                        P.pr.tmask[pt] = m;
+                        P.pr.tbase[pt] = A.chunk_base + c0;
+                        asm volatile("atom.acq_rel.gpu.global.inc.u32 %0, [%1], %2;"
+                                     : "=r"(done) : "l"(P.pr.tctr + tile), "r"(in_tile - 1u) : "memory");
+                    }
+                    done = __shfl_sync(0xffffffffu, done, 0);
+                    if (done == in_tile - 1u) {
+                        __syncwarp();
+                        tile_compact(P.pr, tile, lane);
+                    }
                 }
             }
         }
