@@ -526,6 +526,58 @@ def test_compare_pair_identical_and_truncated():
         ck.compare_pair_async(a, [b[0]], 4096, 1e-6, chunks, idx, counts)
 
 
+# K1 tile compaction (128 pair-tasks = 4096 chunks per tile) + tile_gather_kernel:
+# ragged arrays (pair-tasks of < 32 chunks), several tiles with a ragged last
+# one, every chunk flagged, no chunk flagged, and a chunk-list cap that cuts
+# through a tile -- all against the plain leaf comparison and brute force.
+@pytest.mark.parametrize("mode", ["all", "none", "sparse", "cap"])
+def test_compare_pair_tile_compaction(mode):
+    sizes = [300 * 1024 + 5, 7 * 1024, 4096 * 1024 + 3, 1]       # f32 elements; C = 4 KiB
+    a = [synth.uniform(90 + i, n, "cuda") for i, n in enumerate(sizes)]
+    b = [t.clone() for t in a]
+    if mode in ("all", "cap"):
+        for t in b:
+            t += 1.0                                              # every element differs
+    elif mode == "sparse":
+        for i, t in enumerate(b):
+            t[(7 + 13 * i)::(5000 + 97 * i)] -= 0.5
+    L = sum(-(-n * 4 // 4096) for n in sizes)
+    n_el = sum(sizes)
+    cap = 1500 if mode == "cap" else L
+    chunks = torch.empty(cap, dtype=torch.int64, device="cuda")
+    idx = torch.empty(n_el, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(a, b, 4096, 1e-6, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    nc, nd = counts.tolist()
+    an = np.concatenate([np_of(t).astype(np.float64) for t in a])
+    bn = np.concatenate([np_of(t).astype(np.float64) for t in b])
+    hit = np.abs(an - bn) > 1e-6
+    # chunk ids are global over the arrays in order (each array starts a new chunk)
+    ids = []
+    base_c = 0
+    off = 0
+    for n in sizes:
+        h = np.nonzero(hit[off:off + n])[0]
+        ids.append(base_c + np.unique(h // 1024))
+        base_c += -(-n // 1024)
+        off += n
+    ref_chunks = np.concatenate(ids).astype(np.int64)
+    assert nc == ref_chunks.size
+    assert np.array_equal(np_of(chunks[:min(nc, cap)]), ref_chunks[:cap])
+    if mode == "cap":
+        # verify covers the first `cap` listed chunks only
+        ref_idx = np.nonzero(hit)[0]
+        lim = np.isin(np.concatenate([base + (np.arange(n) // 1024) for base, n in
+                                      zip(np.cumsum([0] + [-(-n // 1024) for n in sizes])[:-1], sizes)]),
+                      ref_chunks[:cap])
+        ref_idx = np.nonzero(hit & lim)[0]
+    else:
+        ref_idx = np.nonzero(hit)[0]
+    assert nd == ref_idx.size
+    assert np.array_equal(np_of(idx[:nd]), ref_idx)
+
+
 # ------------------------------------------- hash block size variant (R23) --
 # "the block size is variable and can be adjusted": every leaf,
 # tree node, chunk list and element list equals the oracle at that block size.
