@@ -599,6 +599,16 @@ static bool leaf_static_tasks() {
     return on;
 }
 
+// CKPT_TILE_GATHER=1: always place the fused path's chunk list with tile_gather_kernel
+// (A/B and tests of that path; by default K4a reads the tiles itself).
+static bool tile_gather_forced() {
+    static const bool on = [] {
+        const char *e = std::getenv("CKPT_TILE_GATHER");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
 // K1 tile-compaction buffers for n_pair pair-tasks (leaf.cuh PairParams):
 // [tctr: n_tiles u32, zeroed once; self-resetting] [tagg: n_tiles u32]
 // [tmask: n_pair u32] [tbase: n_pair u64] [tids: n_tiles * kTileTasks * 32 u64]
@@ -1048,7 +1058,7 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
                                const EmitHook &before_emit = nullptr, uint64_t chunk_base0 = 0,
-                               uint64_t elem_base0 = 0) {
+                               uint64_t elem_base0 = 0, const PairParams *tiles = nullptr) {
     if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
     if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
@@ -1102,6 +1112,15 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     p.out = idx;
     p.cap = cap;
     p.count = n_diff_dev;
+    if (tiles) {
+        // fused pair path: K4a reads K1's tile compaction and writes the chunk list + its count
+        p.tagg = tiles->tagg;
+        p.tids = tiles->tids;
+        p.n_tiles = (uint32_t)((tiles->n_pair + kTileTasks - 1) / kTileTasks);
+        p.tile_ids = (uint32_t)kTileTasks * 32;
+        p.list_out = const_cast<uint64_t *>(chunks);
+        p.n_chunks_out = const_cast<uint64_t *>(n_chunks_dev);
+    }
     static std::atomic<int> occ[5] = {{0}, {0}, {0}, {0}, {0}};
     const int d = dtype == CKPT_F32 ? 0 : 1;
     if (occ[d].load() == 0) {
@@ -1209,9 +1228,13 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     ckpt_tree *trees[2] = {nullptr, nullptr};
     CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
                             trees, &pp));
-    // the ordered chunk list from K1's per-tile compaction (one gather pass)
+    // the ordered chunk list from K1's per-tile compaction: read by K4a directly (up to
+    // kVerifyMaxTiles tiles), else placed by one gather pass
     ckpt_status st = CKPT_OK;
-    {
+    const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
+    const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
+    pp.n_pair = n_pair;
+    if (!tiles_in_mark) {
         TileGatherParams g;
         g.tagg = pp.tagg;
         g.tids = pp.tids;
@@ -1227,7 +1250,7 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     }
     if (st == CKPT_OK)
         st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
-                         idx, idx_cap, counts_dev + 1, s, before_emit);
+                         idx, idx_cap, counts_dev + 1, s, before_emit, 0, 0, tiles_in_mark ? &pp : nullptr);
     if (st != CKPT_OK) {
         ckpt_tree_free_on(trees[0], stream);
         ckpt_tree_free_on(trees[1], stream);

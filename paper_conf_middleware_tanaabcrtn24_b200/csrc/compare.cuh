@@ -389,7 +389,18 @@ struct VerifyParams {
     uint64_t *count;
     uint64_t *states;             // look-back state words (K4b)
     uint32_t epoch;
+    // fused pair path: the chunk list is K1's tile compaction (leaf.cuh
+    // tile_compact) read directly by K4a, which also writes it out (list_out,
+    // n_chunks_out = the device count every later kernel reads as n_chunks_dev)
+    const uint32_t *tagg;         // [n_tiles] flagged chunks per tile, or null
+    const uint64_t *tids;         // [n_tiles * tile_ids]
+    uint32_t n_tiles;
+    uint32_t tile_ids;
+    uint64_t *list_out;
+    uint64_t *n_chunks_out;
 };
+
+constexpr int kVerifyMaxTiles = 4096;   // tile prefix table of K4a in shared memory
 
 __device__ __forceinline__ uint64_t verify_n_chunks(const VerifyParams &p) {
     const uint64_t n = p.n_chunks_dev ? *p.n_chunks_dev : p.n_chunks_host;
@@ -398,10 +409,9 @@ __device__ __forceinline__ uint64_t verify_n_chunks(const VerifyParams &p) {
 
 // Locate listed chunk q: data pointers at its first element, its length and
 // the global id of its first element.
-__device__ __forceinline__ void verify_locate(const VerifyParams &p, uint64_t q, int esz,
-                                              const uint8_t *&pa, const uint8_t *&pb,
-                                              uint64_t &len, uint64_t &gbase) {
-    const uint64_t g = p.chunks[q];
+__device__ __forceinline__ void verify_locate_g(const VerifyParams &p, uint64_t g, int esz,
+                                                const uint8_t *&pa, const uint8_t *&pb,
+                                                uint64_t &len, uint64_t &gbase) {
     const bool inl = p.n_arrays <= kVerifyInline;
     const int a = find_u64(inl ? p.inl_base : p.chunk_base, p.n_arrays, g);
     const VerifyArray A = inl ? p.inl[a] : p.arrays[a];
@@ -411,6 +421,52 @@ __device__ __forceinline__ void verify_locate(const VerifyParams &p, uint64_t q,
     pa = A.a + e_begin * esz;
     pb = A.b + e_begin * esz;
     gbase = A.elem_base + e_begin;
+}
+
+__device__ __forceinline__ void verify_locate(const VerifyParams &p, uint64_t q, int esz,
+                                              const uint8_t *&pa, const uint8_t *&pb,
+                                              uint64_t &len, uint64_t &gbase) {
+    verify_locate_g(p, p.chunks[q], esz, pa, pb, len, gbase);
+}
+
+// Tile mode: exclusive prefix of the tile counts into s_tpre[0..n_tiles]
+// (s_tpre[n_tiles] = total).  Called by all threads of the CTA.
+__device__ __forceinline__ void tile_prefix(const VerifyParams &p, uint32_t *s_tpre) {
+    __shared__ uint32_t s_w[kVerifyWarps];
+    constexpr int kPer = kVerifyMaxTiles / kVerifyThreads;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t nt = p.n_tiles;
+    const uint32_t t0 = threadIdx.x * kPer;
+    uint32_t v[kPer], sum = 0;
+#pragma unroll
+    for (int k = 0; k < kPer; ++k) {
+        v[k] = t0 + k < nt ? __ldcg(p.tagg + t0 + k) : 0u;
+        sum += v[k];
+    }
+    uint32_t wt;
+    uint32_t ex = warp_excl_scan_u32(sum, lane, wt);
+    if (lane == 0) s_w[warp] = wt;
+    __syncthreads();
+#pragma unroll
+    for (int w = 0; w < kVerifyWarps; ++w) ex += w < warp ? s_w[w] : 0u;
+#pragma unroll
+    for (int k = 0; k < kPer; ++k) {
+        if (t0 + k <= nt) s_tpre[t0 + k] = ex;
+        ex += v[k];
+    }
+    if (threadIdx.x == kVerifyThreads - 1 && nt == kVerifyMaxTiles) s_tpre[nt] = ex;
+    __syncthreads();
+}
+
+// Tile mode: chunk id of list position q (q < total).
+__device__ __forceinline__ uint64_t tile_chunk(const VerifyParams &p, const uint32_t *s_tpre, uint64_t q) {
+    uint32_t lo = 0, hi = p.n_tiles - 1;               // last tile with s_tpre[t] <= q
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (s_tpre[mid] <= q) lo = mid; else hi = mid - 1;
+    }
+    return __ldcg(reinterpret_cast<const unsigned long long *>(p.tids) + (uint64_t)lo * p.tile_ids +
+                  (q - s_tpre[lo]));
 }
 
 // Chunks per warp group: the largest power of two <= 32 that still gives
@@ -441,15 +497,31 @@ template <int DT>
 __global__ void __launch_bounds__(kVerifyThreads) verify_mark_kernel(const __grid_constant__ VerifyParams p) {
     pdl_enter();
     constexpr int ESZ = DT == 0 ? 4 : 8;
+    __shared__ uint32_t s_tpre[kVerifyMaxTiles + 1];
     const int lane = threadIdx.x & 31;
-    const uint64_t n_chunks = verify_n_chunks(p);
+    uint64_t n_chunks;
+    if (p.tagg) {
+        tile_prefix(p, s_tpre);
+        const uint64_t total = s_tpre[p.n_tiles];
+        if (blockIdx.x == 0 && threadIdx.x == 0) *p.n_chunks_out = total;
+        n_chunks = total < p.chunks_cap ? total : p.chunks_cap;
+    } else {
+        n_chunks = verify_n_chunks(p);
+    }
     const uint64_t n_warps = (uint64_t)gridDim.x * kVerifyWarps;
     const uint32_t G = verify_group(n_chunks, n_warps);
     for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + (threadIdx.x >> 5)) * G; q0 < n_chunks;
          q0 += n_warps * G) {
       ChunkLoc mine{nullptr, nullptr, 0, 0};
-      if (lane < (int)G && q0 + lane < n_chunks)
-          verify_locate(p, q0 + lane, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+      if (lane < (int)G && q0 + lane < n_chunks) {
+          if (p.tagg) {
+              const uint64_t g = tile_chunk(p, s_tpre, q0 + lane);
+              p.list_out[q0 + lane] = g;
+              verify_locate_g(p, g, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+          } else {
+              verify_locate(p, q0 + lane, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+          }
+      }
       const uint32_t nq = (n_chunks - q0) < G ? (uint32_t)(n_chunks - q0) : G;
       for (uint32_t j = 0; j < nq; ++j) {
         const uint64_t q = q0 + j;
