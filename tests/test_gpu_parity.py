@@ -578,6 +578,20 @@ def test_compare_pair_tile_compaction(mode):
     assert np.array_equal(np_of(idx[:nd]), ref_idx)
 
 
+def test_compare_pair_tile_gather_path():
+    """The gather kernel (used past 4096 tiles) in a fresh process with CKPT_TILE_GATHER=1."""
+    import subprocess
+    import sys
+    code = (
+        "import sys; sys.path.insert(0, %r); import test_gpu_parity as t; "
+        "[t.test_compare_pair_tile_compaction(m) for m in ('all', 'none', 'sparse', 'cap')]; print('ok')"
+        % os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, CKPT_TILE_GATHER="1")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stdout[-2000:] + r.stderr[-2000:]
+
+
 # ------------------------------------------- hash block size variant (R23) --
 # "the block size is variable and can be adjusted" (P:615-618): every leaf,
 # tree node, chunk list and element list equals the oracle at that block size.
