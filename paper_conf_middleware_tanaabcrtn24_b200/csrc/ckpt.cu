@@ -1941,3 +1941,12 @@ extern "C" ckpt_status ckpt_profile_timeline(double *out, uint64_t cap, uint64_t
     }
     return CKPT_OK;
 }
+
+#ifdef CKPT_LEAF_TRACE
+// debug builds only (tools/leaf_trace.py): the last leaf launch's per-warp trace
+extern "C" int ckpt_debug_leaf_trace(uint64_t *host_out, int max_warps) {
+    const int n = max_warps < kTraceWarps ? max_warps : kTraceWarps;
+    if (cudaMemcpyFromSymbol(host_out, g_leaf_trace, (size_t)n * 3 * 8) != cudaSuccess) return -1;
+    return n;
+}
+#endif

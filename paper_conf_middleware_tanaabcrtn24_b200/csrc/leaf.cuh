@@ -221,6 +221,16 @@ __device__ __noinline__ void wide_end(uint64_t &h1, uint64_t &h2, const uint8_t 
 
 constexpr int kLeafInline = 16;
 
+#ifdef CKPT_LEAF_TRACE
+constexpr int kTraceWarps = 8192;
+__device__ uint64_t g_leaf_trace[3 * kTraceWarps];
+__device__ __forceinline__ uint32_t smid() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+    return r;
+}
+#endif
+
 // Fused pair mode: the table holds checkpoint A's m
 // arrays then B's m arrays (identical shapes); warp task t < n_pair is A's
 // task t, t >= n_pair is B's task t - n_pair (the usual batch order, so the
@@ -316,6 +326,12 @@ template <int DT, bool RAW, int CB, bool PAIR, bool WIDE = false>
 __global__ void __launch_bounds__(kLeafWarps * 32, CB >= 32768 ? 1 : CKPT_LEAF_MINB)
 leaf_kernel(const __grid_constant__ LeafParams P) {
     pdl_enter();
+#ifdef CKPT_LEAF_TRACE
+    // debug build only: per-warp start / end globaltimer and tasks done (tools/leaf_trace.py)
+    uint64_t t_start;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
+    uint32_t n_done = 0;
+#endif
     // small array tables travel in the kernel parameters (no H2D copy per build)
     const LeafArray *arrays = P.n_arrays <= kLeafInline ? P.inl : P.arrays;
     const int n_arrays = P.n_arrays;
@@ -562,7 +578,22 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             }
         }
         __syncwarp();
+#ifdef CKPT_LEAF_TRACE
+        ++n_done;
+#endif
     }
+#ifdef CKPT_LEAF_TRACE
+    if ((threadIdx.x & 31) == 0) {
+        uint64_t t_end;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+        const uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+        if (w < kTraceWarps) {
+            g_leaf_trace[3 * w] = t_start;
+            g_leaf_trace[3 * w + 1] = t_end;
+            g_leaf_trace[3 * w + 2] = ((uint64_t)smid() << 32) | n_done;
+        }
+    }
+#endif
 }
 
 }  // namespace ckpt
