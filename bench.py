@@ -278,7 +278,8 @@ def run_ours(args):
                       device="cuda")
     counts = torch.zeros(2, dtype=torch.int64, device="cuda")
     n_arrays = len(A)
-    gathered = torch.empty((world * n_arrays, 16), dtype=torch.uint8, device="cuda")
+    send = torch.empty((2 * n_arrays + 1, 16), dtype=torch.uint8, device="cuda")
+    recv = torch.empty((world, 2 * n_arrays + 1, 16), dtype=torch.uint8, device="cuda")
     keep = []
 
     saved_a, host_a = None, None
@@ -301,12 +302,17 @@ def run_ours(args):
             TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS, hash_block=args.hash_block)
             ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # BFS diff, then verify
         if world > 1:
-            tops = []
-            for T in (TA, TB):
-                dist.all_gather_into_tensor(gathered.view(-1), T.array_roots().view(-1))
-                tops.append(ck.tree_from_digests(gathered))
-            tot = counts.clone()
-            dist.all_reduce(tot)
+            # C1 + C2 in ONE collective: every rank contributes [A roots | B roots | counts]
+            # (2*n_arrays*16 + 16 bytes); the counts are summed locally and both top trees
+            # are built by one levels launch
+            TA.array_roots(out=send[:n_arrays])
+            TB.array_roots(out=send[n_arrays:2 * n_arrays])
+            send[2 * n_arrays].view(torch.int64).copy_(counts)
+            dist.all_gather_into_tensor(recv.view(-1), send.view(-1))
+            roots = recv[:, :2 * n_arrays].reshape(world, 2, n_arrays, 16).transpose(0, 1)
+            tops = ck.tree_from_digests_batch(roots.reshape(2 * world * n_arrays, 16),
+                                              [world * n_arrays, world * n_arrays])
+            tot = recv[:, 2 * n_arrays].contiguous().view(torch.int64).view(world, 2).sum(0)
             keep[:] = [TA, TB, *tops, tot]
         else:
             keep[:] = [TA, TB]

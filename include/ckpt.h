@@ -144,6 +144,14 @@ ckpt_status ckpt_tree_build_batch_ex(const void *const *data, const uint64_t *n,
 ckpt_status ckpt_tree_from_digests(const void *digests16, uint64_t count, void *stream,
                                    ckpt_tree **out);
 
+/* n_trees such trees with ONE interior-level launch (the multi-GPU step
+ * builds the top trees of run A and run B together).  digests16: device,
+ * the counts[k] digests of tree k follow those of tree k-1; counts: host,
+ * n_trees entries, each > 0; out: host array of n_trees handles (all NULL on
+ * error).  Same result as n_trees calls of ckpt_tree_from_digests. */
+ckpt_status ckpt_tree_from_digests_batch(const void *digests16, const uint64_t *counts,
+                                         uint32_t n_trees, void *stream, ckpt_tree **out);
+
 /* Release a tree.  ckpt_tree_free orders the release after the work on the
  * tree's build stream (which must still exist); ckpt_tree_free_on orders it
  * on `stream` instead.  NULL is ignored. */

@@ -15,6 +15,7 @@ Function names follow the C ABI:
     compare(arrays_a, arrays_b, ...)          ckpt_compare             (steps 1-4)
     compare_host(...)                         ckpt_compare_host        (host buffers)
     tree_from_digests(digests)                ckpt_tree_from_digests   (top tree, R15)
+    tree_from_digests_batch(digests, counts)  ckpt_tree_from_digests_batch (several, one launch)
 """
 from __future__ import annotations
 
@@ -79,6 +80,7 @@ def lib():
     L.ckpt_tree_params.argtypes = [vp, ctypes.POINTER(i32), ctypes.POINTER(u32),
                                    ctypes.POINTER(dbl), ctypes.POINTER(u32)]
     L.ckpt_tree_from_digests.argtypes = [vp, u64, vp, pp]
+    L.ckpt_tree_from_digests_batch.argtypes = [vp, pu64, u32, vp, pp]
     L.ckpt_tree_free.argtypes = [vp]
     L.ckpt_tree_free.restype = None
     L.ckpt_tree_free_on.argtypes = [vp, vp]
@@ -115,7 +117,7 @@ def lib():
                  "ckpt_tree_build_batch_ex", "ckpt_compare_pair_ex", "ckpt_tree_params",
                  "ckpt_tree_serialized_size", "ckpt_tree_serialize", "ckpt_tree_deserialize",
                  "ckpt_compare_saved", "ckpt_compare_stream",
-                 "ckpt_tree_from_digests",
+                 "ckpt_tree_from_digests", "ckpt_tree_from_digests_batch",
                  "ckpt_tree_diff", "ckpt_tree_diff_async", "ckpt_verify",
                  "ckpt_verify_arrays_async", "ckpt_compare", "ckpt_compare_host",
                  "ckpt_tree_info", "ckpt_tree_root", "ckpt_tree_array_roots", "ckpt_tree_nodes",
@@ -212,8 +214,12 @@ class Tree:
                                     _stream_ptr(stream)), "ckpt_tree_root")
         return bytes(out)
 
-    def array_roots(self, stream=None) -> torch.Tensor:
-        dst = torch.empty((self.n_arrays, 16), dtype=torch.uint8, device="cuda")
+    def array_roots(self, stream=None, out: Optional[torch.Tensor] = None) -> torch.Tensor:
+        """(n_arrays, 16) uint8 array roots; into `out` (a contiguous uint8 CUDA view) if given."""
+        dst = out if out is not None else torch.empty((self.n_arrays, 16), dtype=torch.uint8,
+                                                      device="cuda")
+        if dst.dtype != torch.uint8 or not dst.is_contiguous() or dst.numel() != self.n_arrays * 16:
+            raise ValueError("out must be a contiguous uint8 tensor of n_arrays x 16 bytes")
         _check(lib().ckpt_tree_array_roots(self.handle, dst.data_ptr(), _stream_ptr(stream)),
                "ckpt_tree_array_roots")
         return dst
@@ -312,6 +318,23 @@ def tree_from_digests(digests: torch.Tensor, stream=None) -> Tree:
     _check(lib().ckpt_tree_from_digests(d.data_ptr(), d.shape[0], sp, ctypes.byref(out)),
            "ckpt_tree_from_digests")
     return Tree(out.value, [d], F32, 16, 0.0, sp)
+
+
+def tree_from_digests_batch(digests: torch.Tensor, counts: Sequence[int], stream=None) -> List[Tree]:
+    """Several top trees with one levels launch: rows [sum(counts[:k]), +counts[k]) of the
+    (sum(counts), 16) uint8 `digests` are the leaves of tree k."""
+    if digests.dtype != torch.uint8 or digests.dim() != 2 or digests.shape[1] != 16:
+        raise ValueError("digests must be a (count, 16) uint8 tensor")
+    if sum(counts) != digests.shape[0]:
+        raise ValueError("counts do not add up to the digest rows")
+    d = digests.contiguous()
+    n = len(counts)
+    cnt = (ctypes.c_uint64 * n)(*[int(c) for c in counts])
+    outs = (ctypes.c_void_p * n)()
+    sp = _stream_ptr(stream)
+    _check(lib().ckpt_tree_from_digests_batch(d.data_ptr(), cnt, n, sp, outs),
+           "ckpt_tree_from_digests_batch")
+    return [Tree(outs[k], [d], F32, 16, 0.0, sp) for k in range(n)]
 
 
 def _host_blob(data):

@@ -818,6 +818,41 @@ extern "C" ckpt_status ckpt_tree_from_digests(const void *digests16, uint64_t co
     return CKPT_OK;
 }
 
+extern "C" ckpt_status ckpt_tree_from_digests_batch(const void *digests16, const uint64_t *counts,
+                                                    uint32_t n_trees, void *stream, ckpt_tree **out) {
+    if (!out) return fail(CKPT_EINVAL, "out is NULL");
+    for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
+    if (!digests16 || !counts || n_trees == 0) return fail(CKPT_EINVAL, "no digests");
+    for (uint32_t k = 0; k < n_trees; ++k)
+        if (counts[k] == 0) return fail(CKPT_EINVAL, "empty digest list");
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    cudaStream_t s = (cudaStream_t)stream;
+    ckpt_status st = CKPT_OK;
+    const uint8_t *src = (const uint8_t *)digests16;
+    for (uint32_t k = 0; k < n_trees && st == CKPT_OK; ++k) {
+        ckpt_tree *t = new ckpt_tree();
+        out[k] = t;
+        t->device = dev;
+        t->stream = s;
+        t->from_digests = true;
+        t->chunk_bytes = 16;
+        t->n_elems.assign(1, counts[k]);
+        layout(t, std::vector<uint64_t>{counts[k]});
+        st = prepare_tree(t, s);
+        if (st == CKPT_OK && cudaMemcpyAsync(t->nodes, src, counts[k] * 16, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+            st = fail(CKPT_ECUDA, "digest copy");
+        src += counts[k] * 16;
+    }
+    if (st == CKPT_OK) st = launch_levels(out, (int)n_trees, s);
+    if (st != CKPT_OK) {
+        for (uint32_t k = 0; k < n_trees; ++k) { ckpt_tree_free_on(out[k], stream); out[k] = nullptr; }
+        return st;
+    }
+    return CKPT_OK;
+}
+
 extern "C" void ckpt_tree_free_on(ckpt_tree *t, void *stream) {
     if (!t) return;
     cudaStream_t s = (cudaStream_t)stream;

@@ -90,6 +90,22 @@ def test_levels_from_digests_bit_exact(L):
     assert bad.size == 0, f"{bad.size} nodes differ, first {bad[:5]}"
 
 
+def test_levels_from_digests_batch_equals_single():
+    """ckpt_tree_from_digests_batch (one levels launch, the multi-GPU step's top trees)."""
+    counts = [1, 7, 2049, 48]
+    g = torch.Generator().manual_seed(5)
+    d = torch.randint(0, 256, (sum(counts), 16), dtype=torch.uint8, generator=g)
+    trees = ck.tree_from_digests_batch(d.cuda(), counts)
+    off = 0
+    for t, c in zip(trees, counts):
+        ref = oracle.levels(d[off:off + c].numpy())
+        assert np.array_equal(gpu_tree_nodes(t), ref)
+        assert t.root() == ref[-1].tobytes()
+        off += c
+    with pytest.raises(ValueError):
+        ck.tree_from_digests_batch(d.cuda(), [1, 2])
+
+
 # Multi-array batch: arrays of different heights whose groups end mid-pass.
 def test_levels_multi_array_ragged_groups():
     sizes = [4097 * 4096, 1 * 4096, 2049 * 4096 + 8, 3 * 4096]
