@@ -326,7 +326,37 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         }
     }
     __syncthreads();
-    // top tree: level 0 = array roots in array order (R15), built in L2 (tiny)
+    // top tree: level 0 = array roots in array order (R15).  Up to 2 * kLevelSmemNodes / 3
+    // roots it is built in shared memory (one L2 round trip for the roots, then only
+    // stores); larger tops through L2.
+    if ((uint64_t)na + ((uint64_t)na + 1) / 2 <= (uint64_t)kLevelSmemNodes) {
+        uint4 *cur = sm, *nxt = sm + na;
+        for (int a = tid; a < na; a += kLevelThreads) {
+            const int h = (int)p.height[a];
+            const uint4 v = __ldcg(p.nodes + p.off[(uint64_t)(h - 1) * na + a]);
+            p.nodes[p.top_off + a] = v;
+            cur[a] = v;
+        }
+        __syncthreads();
+        uint64_t n = (uint64_t)na, at = p.top_off;
+        while (n > 1) {
+            const uint64_t up = (n + 1) >> 1;
+            for (uint64_t j = tid; j < up; j += kLevelThreads) {
+                uint4 x = cur[2 * j];
+                if (2 * j + 1 < n) x = hash_children32(x, cur[2 * j + 1]);
+                p.nodes[at + n + j] = x;
+                nxt[j] = x;
+            }
+            __syncthreads();
+            uint4 *t = cur;
+            cur = nxt;
+            nxt = t;
+            at += n;
+            n = up;
+        }
+        if (tid == 0) *p.ticket = 0u;
+        return;
+    }
     for (int a = tid; a < na; a += kLevelThreads) {
         const int h = (int)p.height[a];
         p.nodes[p.top_off + a] = __ldcg(p.nodes + p.off[(uint64_t)(h - 1) * na + a]);
