@@ -1985,3 +1985,9 @@ extern "C" int ckpt_debug_leaf_trace(uint64_t *host_out, int max_warps) {
     return n;
 }
 #endif
+
+#ifdef CKPT_LEVELS_TRACE
+extern "C" int ckpt_debug_levels_trace(uint64_t *host_out) {
+    return cudaMemcpyFromSymbol(host_out, g_lv_trace, sizeof(uint64_t) * (kLvTraceCtas * 4 + 16)) == cudaSuccess ? 0 : -1;
+}
+#endif

@@ -140,8 +140,32 @@ __device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 
     }
 }
 
-__global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_constant__ LevelBatch pb) {
+#ifdef CKPT_LEVELS_TRACE
+// debug build only: per-CTA [entry, after griddepcontrol.wait, phase-1 end, ticket] and the
+// last CTA's [phase-2 levels end, top end] globaltimer stamps (tools/levels_trace.py)
+constexpr int kLvTraceCtas = 4096;
+__device__ uint64_t g_lv_trace[kLvTraceCtas * 4 + 16];
+__device__ __forceinline__ uint64_t gtime() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+#define LV_STAMP(slot, v) do { if (threadIdx.x == 0 && blockIdx.x < kLvTraceCtas) g_lv_trace[blockIdx.x * 4 + (slot)] = (v); } while (0)
+#define LV_STAMP_LAST(slot) do { if (threadIdx.x == 0) g_lv_trace[kLvTraceCtas * 4 + 2 * ti + (slot)] = gtime(); } while (0)
+#else
+#define LV_STAMP(slot, v) do { } while (0)
+#define LV_STAMP_LAST(slot) do { } while (0)
+#endif
+
+__global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_constant__ LevelBatch pb) {
+#ifdef CKPT_LEVELS_TRACE
+    const uint64_t t_entry = gtime();
+#endif
     pdl_enter();
+#ifdef CKPT_LEVELS_TRACE
+    LV_STAMP(0, t_entry);
+    LV_STAMP(1, gtime());
+#endif
     extern __shared__ __align__(16) uint4 sm[];
 #ifdef CKPT_LV_OLD
     __shared__ uint4 s_root[kLevelThreads / 32];
@@ -252,7 +276,44 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         };
         uint4 *buf[2] = {sm, sm + kLevelThreads};       // ping-pong: 512 + 128 nodes
         int cnt = m0;
-        for (int r = 0; r < kLog; r += 2) {
+        if (m0 == kGroup) {
+            // full group (the common case): every level up to kLog exists in the array's
+            // tree and every thread that works has 4 (or 2) valid nodes -- no predicates,
+            // level base pointers formed once per pass
+            for (int r = 0; r < kLog; r += 2) {
+                const bool two = r + 2 <= kLog;
+                const int need = two ? (kGroup >> r) >> 2 : (kGroup >> r) >> 1;
+                const uint4 *in = buf[(r >> 1) & 1];
+                uint4 *out = buf[((r >> 1) + 1) & 1];
+                if (tid < need) {
+                    uint4 *l1 = p.nodes + p.off[(uint64_t)(p.ls + r + 1) * na + a] + (start >> (r + 1));
+                    if (two) {
+                        uint4 *l2 = p.nodes + p.off[(uint64_t)(p.ls + r + 2) * na + a] + (start >> (r + 2));
+                        uint4 x0, x1, x2, x3;
+                        if (r == 0) {
+                            x0 = __ldg(src + 4 * tid); x1 = __ldg(src + 4 * tid + 1);
+                            x2 = __ldg(src + 4 * tid + 2); x3 = __ldg(src + 4 * tid + 3);
+                        } else {
+                            x0 = in[4 * tid]; x1 = in[4 * tid + 1]; x2 = in[4 * tid + 2]; x3 = in[4 * tid + 3];
+                        }
+                        const uint4 y0 = hash_children32(x0, x1);
+                        const uint4 y1 = hash_children32(x2, x3);
+                        l1[2 * tid] = y0;
+                        l1[2 * tid + 1] = y1;
+                        const uint4 z = hash_children32(y0, y1);
+                        l2[tid] = z;
+                        out[tid] = z;
+                    } else {
+                        const uint4 y0 = hash_children32(in[2 * tid], in[2 * tid + 1]);
+                        l1[tid] = y0;
+                        out[tid] = y0;
+                    }
+                }
+                __syncthreads();
+            }
+            cnt = 1;
+        }
+        for (int r = 0; r < kLog && m0 != kGroup; r += 2) {
             const bool two = r + 2 <= kLog;
             const int need = two ? (cnt + 3) >> 2 : (cnt + 1) >> 1;
             const uint4 *in = buf[(r >> 1) & 1];
@@ -287,6 +348,9 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         }
     }
 #endif
+#ifdef CKPT_LEVELS_TRACE
+    LV_STAMP(2, gtime());
+#endif
     // ------------------------------ phase 2 ------------------------------
     // Last-CTA hand-off without sequentially consistent fences (MEMBAR.SC.GPU
     // costs microseconds): the barrier orders every thread's node stores before
@@ -300,6 +364,9 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         s_ticket = t;
     }
     __syncthreads();
+#ifdef CKPT_LEVELS_TRACE
+    LV_STAMP(3, gtime());
+#endif
     if (s_ticket != p.n_groups - 1) return;
     int F = p.ls + kLog;                       // highest level phase 1 completed
     if (F > p.n_levels - 1) F = p.n_levels - 1;
@@ -326,6 +393,7 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
         }
     }
     __syncthreads();
+    LV_STAMP_LAST(0);
     // top tree: level 0 = array roots in array order (R15).  Up to 2 * kLevelSmemNodes / 3
     // roots it is built in shared memory (one L2 round trip for the roots, then only
     // stores); larger tops through L2.
@@ -354,6 +422,7 @@ __global__ void __launch_bounds__(kLevelThreads) levels_kernel(const __grid_cons
             at += n;
             n = up;
         }
+        LV_STAMP_LAST(1);
         if (tid == 0) *p.ticket = 0u;
         return;
     }
