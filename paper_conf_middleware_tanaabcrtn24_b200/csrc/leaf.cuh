@@ -43,8 +43,12 @@ struct LeafArray {            // one array of the checkpoint (device table)
 #ifndef CKPT_LEAF_CH
 #define CKPT_LEAF_CH 1
 #endif
+#ifndef CKPT_LEAF_UNROLL
+#define CKPT_LEAF_UNROLL 2      // f32 stage-loop unroll (see the fast path)
+#endif
 constexpr int kLeafWarps = 8;                  // warps per CTA
 constexpr int kCh = CKPT_LEAF_CH;              // chains (chunks) per lane
+constexpr int kLeafUnroll = CKPT_LEAF_UNROLL;  // f32 stage-loop unroll
 constexpr int kRows = 32 * kCh;                // chunks per warp task
 constexpr int kSeg = CKPT_LEAF_SEG;            // bytes per chunk per stage
 constexpr int kStages = CKPT_LEAF_STAGES;      // ring depth
@@ -412,7 +416,7 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             // stage's + kSeg, an immediate offset (LDGSTS takes +-2 KB), so the 16 64-bit
             // address adds per stage are paid every other stage (86.5 -> 83.1 instructions
             // per 16-byte block; c2 pair launch 722 -> 706 us)
-#pragma unroll (DT == 0 ? 2 : 1)
+#pragma unroll (DT == 0 ? kLeafUnroll : 1)
 #endif
             for (uint32_t s = 0; s < n_stages; ++s) {
                 if (s + kStages - 1 < n_stages) issue(src, nslot);
