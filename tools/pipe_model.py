@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Static pipe-cost model of the K1 hot loop (no GPU needed).
 
-usage: pipe_model.py [-DFLAG ...]
+usage: pipe_model.py [-DFLAG ...]   (-DDTX=1: the f64 instantiation)
 Compiles csrc/leaf.cuh's leaf_kernel<F32, !RAW, 4096, PAIR> alone to a cubin with the given
 defines, finds the chain loop (as tools/sass_loop.py does) and prints per-16-byte-block
 instruction counts and pipe cycles per SMSP under the rates measured on B200 with ncu
@@ -14,8 +14,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 CSRC = os.path.join(ROOT, "paper_conf_middleware_tanaabcrtn24_b200", "csrc")
 defs = [a for a in sys.argv[1:] if a.startswith("-D")]
 src = r'''
+#ifndef DTX
+#define DTX 0
+#endif
 #include "leaf.cuh"
-template __global__ void ckpt::leaf_kernel<0, false, 4096, true, false>(const __grid_constant__ ckpt::LeafParams);
+template __global__ void ckpt::leaf_kernel<DTX, false, 4096, true, false>(const __grid_constant__ ckpt::LeafParams);
 '''
 with tempfile.TemporaryDirectory() as d:
     cu = os.path.join(d, "k.cu"); open(cu, "w").write(src)
