@@ -7,7 +7,7 @@
 //   * 64-bit x constant -> IMAD.WIDE.U32 + 2 x IMAD (fma pipe, 3 instr),
 //   * k ^= k >> 33      -> lo ^= hi >> 1 (SHF + LOP3),
 //   * rotl64 by r       -> two funnel shifts (SHF.L.W) on swapped halves,
-//   * h*5 + c           -> IMAD.WIDE.U32 with a 64-bit addend + IMAD + IADD3.
+//   * h*5 + c           -> IMAD.WIDE.U32 with a 64-bit addend + one IMAD.
 // The leaf kernel is issue-bound, so every instruction
 // of this step is throughput.
 #pragma once
@@ -79,8 +79,8 @@ __device__ __forceinline__ U64p add64(U64p a, U64p b) {
 }
 #endif
 
-// h*5 + c in plain 64-bit C: ptxas folds the 64-bit addend c into IMAD.WIDE.U32
-// (lo*5 + c) and adds hi*5 with one IMAD + IADD3.  (An inline-asm mad.wide with
+// h*5 + c (the default below): lo*5 + c with the 64-bit addend folded into
+// IMAD.WIDE.U32, then hi*5 + that product's high word.  (An inline-asm mad.wide with
 // an immediate multiplier was split by ptxas into IMAD.WIDE + IADD3 + IMAD.X:
 // 2 more instructions per block, measured 1.8% slower in the leaf kernel.)
 #if defined(CKPT_M5ASM)
@@ -111,10 +111,19 @@ __device__ __forceinline__ U64p mul5_add_alu(U64p h, uint64_t c) {
 }
 #if defined(CKPT_M5LEA)
 __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) { return mul5_add_alu(h, c); }
-#elif !defined(CKPT_M5ASM)
+#elif defined(CKPT_M5_64)
+// the whole 64-bit product in C: ptxas emits IMAD.WIDE.U32 + IMAD + IMAD.IADD (it splits
+// hi*5 + carry-word into two instructions)
 __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
     const uint64_t x = (((uint64_t)h.hi << 32) | h.lo) * 5ull + c;
     return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
+}
+#elif !defined(CKPT_M5ASM)
+// lo*5 + c as one IMAD.WIDE.U32 (64-bit addend folded), hi*5 + its high word as ONE IMAD:
+// 2 instructions instead of 3 (81.1 vs 83.1 per block; c2 pair launch 706 -> 692 us)
+__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
+    const uint64_t x = (uint64_t)h.lo * 5u + c;
+    return U64p{(uint32_t)x, h.hi * 5u + (uint32_t)(x >> 32)};
 }
 #endif
 
