@@ -152,7 +152,7 @@ template <int DT, bool RAW>
 __device__ __forceinline__ void chain_block_fast(U64p &h1, U64p &h2, uint4 v, const QuantParams &q,
                                                  bool &ok, float &mx) {
     const uint4 w = words_fast<DT, RAW>(v, q, ok, mx);
-    mm3p_block16(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
+    mm3p_block16<DT == 1>(h1, h2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
 }
 
 // Wide hash blocks (reading R23): a block of B = 16*hb16 bytes is

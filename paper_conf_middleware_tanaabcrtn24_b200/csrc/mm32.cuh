@@ -184,45 +184,56 @@ __device__ __forceinline__ void mm3p_body(U64p &h1, U64p &h2, U64p k1, U64p k2, 
 }
 
 // Murmur3F finalisation for a total length `len` < 2^32.
-#ifdef CKPT_ADD3
-// a + b + b (h2 += h1 right after h1 += h2, as one 3-input add off h1's critical path)
+__device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
+    h1.lo ^= len;
+    h2.lo ^= len;
+    h1 = add64(h1, h2);
+    h2 = add64(h2, h1);
+    h1 = fmix64p(h1);
+    h2 = fmix64p(h2);
+    h1 = add64(h1, h2);
+    h2 = add64(h2, h1);
+}
+
+// a + b + b: "h1 += h2; h2 += h1" as two independent adds, the second a 3-input
+// add that ptxas emits as IADD3 + IADD3.X (ALU pipe) instead of IADD3 + IMAD.X
 __device__ __forceinline__ U64p add64_abb(U64p a, U64p b) {
-    const uint64_t x = (((uint64_t)a.hi << 32) | a.lo) + (((uint64_t)b.hi << 32) | b.lo) +
-                       (((uint64_t)b.hi << 32) | b.lo);
-    return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
+    U64p r;
+    asm("add.cc.u32 %0, %2, %4;\n\taddc.u32 %1, %3, %5;\n\t"
+        "add.cc.u32 %0, %0, %4;\n\taddc.u32 %1, %1, %5;"
+        : "=&r"(r.lo), "=&r"(r.hi)
+        : "r"(a.lo), "r"(a.hi), "r"(b.lo), "r"(b.hi));
+    return r;
 }
-__device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
+
+// The same finalisation with the second add of each pair as add64_abb: the same
+// instruction count, two carries moved from the FMA-heavy pipe to the ALU.  Used by
+// the f64 leaf chain, whose FMA-heavy pipe binds (f64 pair launch 711 -> 663 us);
+// the f32 chain is faster with the default (675 vs 692 us).
+__device__ __forceinline__ void mm3p_final_alu(U64p &h1, U64p &h2, uint32_t len) {
     h1.lo ^= len;
     h2.lo ^= len;
     {
         const U64p a = add64(h1, h2), b = add64_abb(h1, h2);
-        h1 = a; h2 = b;
+        h1 = a;
+        h2 = b;
     }
     h1 = fmix64p(h1);
     h2 = fmix64p(h2);
     {
         const U64p a = add64(h1, h2), b = add64_abb(h1, h2);
-        h1 = a; h2 = b;
+        h1 = a;
+        h2 = b;
     }
 }
-#else
-__device__ __forceinline__ void mm3p_final(U64p &h1, U64p &h2, uint32_t len) {
-    h1.lo ^= len;
-    h2.lo ^= len;
-    h1 = add64(h1, h2);
-    h2 = add64(h2, h1);
-    h1 = fmix64p(h1);
-    h2 = fmix64p(h2);
-    h1 = add64(h1, h2);
-    h2 = add64(h2, h1);
-}
-#endif
 
 // One chained 16-byte block: (h1,h2) <- Murmur3F(k1||k2, len 16, state (h1,h2)).
+template <bool ALU_ADDS = false>
 __device__ __forceinline__ void mm3p_block16(U64p &h1, U64p &h2, U64p k1, U64p k2, uint64_t m1,
                                              uint64_t m2) {
     mm3p_body(h1, h2, k1, k2, m1, m2);
-    mm3p_final(h1, h2, 16u);
+    if (ALU_ADDS) mm3p_final_alu(h1, h2, 16u);
+    else mm3p_final(h1, h2, 16u);
 }
 
 // Interior node: Murmur3F(left || right, 32 bytes, seed 0)  (Alg. 1, R14).
