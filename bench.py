@@ -365,6 +365,9 @@ def run_ours(args):
     for k in ("leaf", "levels", "diff", "verify"):
         pms, pn = ck.profile_read(k)
         phases[k] = {"ms_per_step": round(pms / k_prof, 4), "launches": pn}
+    if phases["diff"]["launches"] == 0:
+        phases["diff"]["note"] = ("fused path: the leaf-level diff and its ordered compaction run inside "
+                                  "the leaf kernel (per-tile), the chunk list is written by verify_mark")
     ck.profile_reset()
     # side reference K5: "Direct" on the device -- verify with every chunk
     # flagged, i.e. 2S bytes compared element-wise with no hashing and no tree
