@@ -79,7 +79,7 @@ def compare_runs(arrays_a: Sequence[torch.Tensor], arrays_b: Sequence[torch.Tens
     """Compare this rank's arrays of run A and run B (steps 1-4) and join the ranks.
 
     With torch.distributed uninitialised (or world size 1) no collective runs."""
-    from . import tree_build, tree_diff_async, tree_from_digests, verify_async
+    from . import tree_build, tree_diff_async, tree_from_digests_batch, verify_async
 
     TA = tree_build(list(arrays_a), chunk_bytes, eps)
     TB = tree_build(list(arrays_b), chunk_bytes, eps)
@@ -94,14 +94,31 @@ def compare_runs(arrays_a: Sequence[torch.Tensor], arrays_b: Sequence[torch.Tens
     chunk_off = elem_off = 0
     local = counts.clone()
     if distributed:
-        roots_a = gather_roots(TA.array_roots(), group)
-        roots_b = gather_roots(TB.array_roots(), group)
-        top_a, top_b = tree_from_digests(roots_a), tree_from_digests(roots_b)
-        sizes = gather_counts([TA.n_leaves, n_elems], group, "cuda")
+        # two collectives: a fixed-size header (array count, sizes, counts), then the roots
+        # of both runs padded to the largest array count; the counts are summed locally and
+        # both top trees are built by one levels launch
+        world = dist.get_world_size(group)
         r = dist.get_rank(group)
-        chunk_off = int(sizes[:r, 0].sum().item()) if r else 0
-        elem_off = int(sizes[:r, 1].sum().item()) if r else 0
-        allreduce_counts(counts, group)
+        na = len(arrays_a)
+        hdr = torch.stack([torch.tensor([na, TA.n_leaves, n_elems], dtype=torch.int64,
+                                        device="cuda"), counts.new_zeros(3)]).view(-1)
+        hdr[3:5] = counts
+        hdrs = torch.empty((world, 6), dtype=torch.int64, device="cuda")
+        dist.all_gather_into_tensor(hdrs.view(-1), hdr, group=group)
+        h = hdrs.cpu()
+        nas = h[:, 0].tolist()
+        m = max(nas)
+        send = torch.zeros((2 * m, 16), dtype=torch.uint8, device="cuda")
+        TA.array_roots(out=send[:na])
+        TB.array_roots(out=send[m:m + na])
+        recv = torch.empty((world, 2 * m, 16), dtype=torch.uint8, device="cuda")
+        dist.all_gather_into_tensor(recv.view(-1), send.view(-1), group=group)
+        ra = torch.cat([recv[k, :nas[k]] for k in range(world)], 0)
+        rb = torch.cat([recv[k, m:m + nas[k]] for k in range(world)], 0)
+        top_a, top_b = tree_from_digests_batch(torch.cat([ra, rb], 0), [ra.shape[0], rb.shape[0]])
+        chunk_off = int(h[:r, 1].sum().item()) if r else 0
+        elem_off = int(h[:r, 2].sum().item()) if r else 0
+        counts.copy_(hdrs[:, 3:5].sum(0))
     else:
         top_a, top_b = TA, TB
     ra = top_a.root() if read_roots else None
