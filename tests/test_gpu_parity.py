@@ -956,6 +956,39 @@ def test_config5_full_size_sampled_parity():
         assert np.array_equal(gpu_tree_nodes(TA, k)[: la.shape[0]], la), k
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("C", [512, 4096, 65536])
+def test_config3_full_size_parity(C):
+    """BASELINE configs[2] at full size (2^29 f64 ~ N(0,1), 4 GiB per run, 1024 clustered
+    divergences) on the fused pair path the bench times, at the smallest, default and largest
+    chunk of the sweep: EVERY leaf of both trees equals the oracle's (full-array oracle leaves),
+    every interior level equals the oracle's levels over them, and the chunk list and element
+    ids equal the oracle's diff + verify; the element count also equals a device brute-force
+    count of |a-b| > eps."""
+    pair = synth.c3_pair(device="cuda")
+    eps, n = pair.eps, pair.a[0].numel()
+    a, b = pair.a[0], pair.b[0]
+    L = -(-n * 8 // C)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(1 << 24, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async([a], [b], C, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    nc, nd = counts.tolist()
+    assert nd == int((a - b).abs().gt(eps).sum().item()) and 0 < nd <= idx.numel()
+    an, bn = np_of(a), np_of(b)
+    th = os.cpu_count() or 8
+    la, lb = oracle.leaves(an, C, eps, threads=th), oracle.leaves(bn, C, eps, threads=th)
+    na, nb = gpu_tree_nodes(TA), gpu_tree_nodes(TB)
+    assert np.array_equal(na[:L], la) and np.array_equal(nb[:L], lb)
+    assert np.array_equal(oracle.levels(la), na) and np.array_equal(oracle.levels(lb), nb)
+    ref_c = np.nonzero(np.any(la != lb, axis=1))[0]
+    ref_i = oracle.verify(an, bn, C, ref_c, eps)
+    assert nc == ref_c.size and np.array_equal(np_of(chunks[:nc]), ref_c)
+    assert nd == ref_i.size and np.array_equal(np_of(idx[:nd]), ref_i)
+    del a, b, pair
+
+
 # -------------------------- latency variant of the leaf kernel (few chains) --
 
 @pytest.mark.parametrize("dt,chunk,n,eps", [(torch.float32, 16384, (1 << 22) + 5, 1e-6),
