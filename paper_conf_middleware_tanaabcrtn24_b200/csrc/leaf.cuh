@@ -57,13 +57,17 @@ constexpr int kSlotBytes = kRows * kPitch;
 constexpr int kWarpSmem = kStages * kSlotBytes;
 constexpr int kLeafSmem = kLeafWarps * kWarpSmem + 16;   // + the two h*5+c addends
 
+// L2 prefetch size hint of the staging copies (tuning knob; 128 B is the product)
+#ifndef CKPT_LEAF_L2PF
+#define CKPT_LEAF_L2PF ".L2::128B"
+#endif
 __device__ __forceinline__ void cp_async16(uint32_t smem, const void *gptr, uint32_t src_bytes) {
-    asm volatile("cp.async.cg.shared.global.L2::128B [%0], [%1], 16, %2;\n" ::"r"(smem), "l"(gptr),
+    asm volatile("cp.async.cg.shared.global" CKPT_LEAF_L2PF " [%0], [%1], 16, %2;\n" ::"r"(smem), "l"(gptr),
                  "r"(src_bytes)
                  : "memory");
 }
 __device__ __forceinline__ void cp_async16_full(uint32_t smem, const void *gptr) {
-    asm volatile("cp.async.cg.shared.global.L2::128B [%0], [%1], 16;\n" ::"r"(smem), "l"(gptr)
+    asm volatile("cp.async.cg.shared.global" CKPT_LEAF_L2PF " [%0], [%1], 16;\n" ::"r"(smem), "l"(gptr)
                  : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
