@@ -46,7 +46,10 @@ struct LeafArray {            // one array of the checkpoint (device table)
 #ifndef CKPT_LEAF_UNROLL
 #define CKPT_LEAF_UNROLL 2      // f32 stage-loop unroll (see the fast path)
 #endif
-constexpr int kLeafWarps = 8;                  // warps per CTA
+#ifndef CKPT_LEAF_WARPS
+#define CKPT_LEAF_WARPS 8
+#endif
+constexpr int kLeafWarps = CKPT_LEAF_WARPS;    // warps per CTA
 constexpr int kCh = CKPT_LEAF_CH;              // chains (chunks) per lane
 constexpr int kLeafUnroll = CKPT_LEAF_UNROLL;  // f32 stage-loop unroll
 constexpr int kRows = 32 * kCh;                // chunks per warp task
