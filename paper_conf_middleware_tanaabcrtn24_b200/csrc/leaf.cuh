@@ -435,8 +435,7 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
                 const uint32_t row = my_row + slot;
 #pragma unroll
                 for (int b = 0; b < kPiecesPerChunk; ++b) {
-                    if constexpr (WIDE) {
-                        static_assert(!WIDE || kCh == 1, "wide blocks assume one chain per lane");
+                    if constexpr (WIDE && kCh == 1) {   // wide blocks: one chain per lane
                         const uint4 w = words_fast<DT, RAW>(lds128(row + b * 16), q, ok, mx);
                         wide_piece(h1[0], h2[0], w, q, left, hb16);
                     } else {
@@ -540,8 +539,8 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             const uint64_t c = c0 + 32 * j + lane;
             if (c < A.n_leaves) A.out[c] = make_uint4(h1[j].lo, h1[j].hi, h2[j].lo, h2[j].hi);
         }
-        if (PAIR) {
-            static_assert(!PAIR || kCh == 1, "pair mode assumes one chain per lane");
+        // pair mode assumes one chain per lane (kCh > 1 is a single-tree tuning build only)
+        if constexpr (PAIR && kCh == 1) {
             const int side = a >= P.pr.m ? 1 : 0;
             const uint64_t pt = task - (side ? P.pr.n_pair : 0);
             // publish my leaves, then count in; the second of the pair does the compare.
