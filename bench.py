@@ -15,6 +15,11 @@ own such checkpoint pair (weak scaling, arrays sharded by rank as HACC writes
 per-rank checkpoints).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+--gpus N > 1 without a torch.distributed environment re-launches this script
+as N ranks (one process per GPU, NCCL) through torch.distributed.run on
+127.0.0.1; under an existing launcher (WORLD_SIZE set) the world size must
+equal N.  Rank 0 prints the one JSON line.
 """
 from __future__ import annotations
 
@@ -45,9 +50,10 @@ CONFIGS = {
                "below-eps changes, 1% chunks below-eps only"),
     "c3": dict(n=1 << 29, workload="configs[2] (C=4 KiB, eps=1e-6 point): 2^29 float64 ~ N(0,1), "
                "1024 geometric clusters (mean 4096) with |d|=10^U(-9,-2)"),
-    "c4": dict(n=1 << 24, workload="configs[3]: one intermediate snapshot (default s=9) of a 64-rank "
-               "HACC run, 2^30 particles x 6 float32 per run (2^24 per rank), ranks sharded over the "
-               "GPUs (strong scaling), 4 KiB chunks, eps=1e-6, clustered divergence 1e-6*4^(s-3)"),
+    "c4": dict(n=1 << 24, workload="configs[3]: intermediate snapshots of a 64-rank HACC run (one "
+               "snapshot, default s=9, or --snapshots all = the 10-snapshot sequence), 2^30 particles "
+               "x 6 float32 per run (2^24 per rank), ranks sharded over the GPUs (strong scaling), "
+               "4 KiB chunks, eps=1e-6, clustered divergence 1e-6*4^(s-3)"),
 }
 SNAPSHOT = 9
 C4_RANKS = 64
@@ -185,20 +191,27 @@ def calibrate_oracle(target_s: float, threads: int):
     return n
 
 
-def cpu_baseline(target_s: float = 12.0):
-    import oracle
-    oracle.build()
-    threads = host_cores()
+def _time_oracle(target_s: float, threads: int):
     n = calibrate_oracle(target_s, threads)
     a, b = oracle_pair_sample(n, SEED)
     t0 = time.perf_counter()
     oracle_step(a, b, threads)
     dt = time.perf_counter() - t0
     nbytes = 2 * sum(x.nbytes for x in a)
-    return {"value": round(nbytes / dt / 1e9, 4), "unit": "GB/s", "cores": threads,
-            "kind": "oracle",
-            "sample": f"same recipe ({CFG}) at {n} elements per array ({nbytes / 1e6:.1f} MB pair), "
-                      f"one full step (build A+B, BFS diff, verify) in {dt:.2f} s"}
+    return nbytes / dt / 1e9, (f"same recipe ({CFG}) at {n} elements per array ({nbytes / 1e6:.1f} MB "
+                               f"pair), one full step (build A+B, BFS diff, verify) in {dt:.2f} s")
+
+
+def cpu_baseline(target_s: float = 8.0):
+    """The oracle as it stands on the host cores: all cores (value) and one thread."""
+    import oracle
+    oracle.build()
+    threads = host_cores()
+    v_all, s_all = _time_oracle(target_s, threads)
+    v_one, s_one = _time_oracle(target_s, 1)
+    return {"value": round(v_all, 4), "unit": "GB/s", "cores": threads, "kind": "oracle",
+            "sample": s_all,
+            "single_thread": {"value": round(v_one, 4), "unit": "GB/s", "cores": 1, "sample": s_one}}
 
 
 def run_reference(args):
@@ -248,17 +261,37 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py --gpus {args.gpus} but the launcher started {world} ranks")
     # CKPT_DIST_BACKEND=gloo + more ranks than GPUs: a functional test of the N>1 path on one
     # GPU (ranks share it; timings are not meaningful).  Production: one rank per GPU, NCCL.
     backend = os.environ.get("CKPT_DIST_BACKEND", "nccl")
+    if backend == "nccl" and world > torch.cuda.device_count():
+        raise SystemExit(f"{world} NCCL ranks need {world} GPUs; this node has "
+                         f"{torch.cuda.device_count()}")
     local = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
     torch.cuda.set_device(local)
-    group = None
-    if world > 1:
+    # the C1/C2 exchange runs for N > 1, and at N = 1 under a launcher with --collectives
+    # (exercises the NCCL path on a one-GPU box)
+    collect = world > 1 or args.collectives
+    nccl_info = None
+    if collect:
+        for k, v in (("MASTER_ADDR", "127.0.0.1"), ("RANK", "0"), ("WORLD_SIZE", "1")):
+            os.environ.setdefault(k, v)
+        os.environ.setdefault("MASTER_PORT", str(free_port()))
         if backend == "nccl":
+            # communicator-init log on stderr (stdout carries only the JSON line)
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+            os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            v = torch.cuda.nccl.version()
+            nccl_info = {"backend": "nccl", "version": ".".join(str(x) for x in v)
+                         if isinstance(v, tuple) else str(v), "world": dist.get_world_size(),
+                         "exchange": "one all_gather_into_tensor per step (C1 roots + C2 counts)"}
         else:
             dist.init_process_group(backend)
+            nccl_info = {"backend": backend, "world": dist.get_world_size()}
     import paper_conf_middleware_tanaabcrtn24_b200 as ck
     from paper_conf_middleware_tanaabcrtn24_b200 import dist as ckd
     import synth
@@ -301,7 +334,7 @@ def run_ours(args):
         else:
             TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS, hash_block=args.hash_block)
             ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # BFS diff, then verify
-        if world > 1:
+        if collect:
             # C1 + C2 in ONE collective: every rank contributes [A roots | B roots | counts]
             # (2*n_arrays*16 + 16 bytes); the counts are summed locally and both top trees
             # are built by one levels launch
@@ -319,41 +352,65 @@ def run_ours(args):
         TA.wait()          # the step ends when both trees are complete (K2 runs on a side stream)
         TB.wait()
 
-    for _ in range(max(3, args.warmup)):
-        step()
-    torch.cuda.synchronize()
-    local_counts = counts.cpu().tolist()
-
-    # timed region
+    # configs[3] as written (--snapshots all): the 10 intermediate snapshots, one at a time
+    # (each generated into HBM before its timed region), every snapshot's trees kept; the
+    # sequence's time is the sum of the snapshots' device times.  Otherwise one snapshot / pair.
+    global SNAPSHOT
+    snaps = list(range(10)) if (CFG == "c4" and args.snapshots == "all") else [SNAPSHOT]
     sampler = ClockSampler(torch.cuda.current_device())
     sampler.start()
     time.sleep(0.2)
-    ck.profile_reset()
-    ck.profile_enable(["leaf"])     # leaf events only: the roofline kernel (events elsewhere end PDL overlap)
-    l0 = ck.launch_count()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record()
-    h0 = time.perf_counter()
-    for _ in range(args.steps):
-        step()
-    host_ms = (time.perf_counter() - h0) * 1e3 / args.steps   # enqueue time per step (host)
-    e1.record()
-    torch.cuda.synchronize()
-    launches = ck.launch_count() - l0
-    ck.profile_enable(False)
+    ms_max = host_ms = leaf_ms = 0.0
+    leaf_n = launches = 0
+    per_snap, kept_trees = [], []
+    for si, snap in enumerate(snaps):
+        if si > 0 or snap != SNAPSHOT:
+            SNAPSHOT = snap
+            A = B = pair = None
+            pair = make_pair(CFG, N_PARTICLES, SEED + 1000 * rank, "cuda")
+            A, B = pair.a, pair.b
+        for _ in range(max(3, args.warmup)):
+            step()
+        torch.cuda.synchronize()
+        local_counts = counts.cpu().tolist()
+        # timed region
+        ck.profile_reset()
+        ck.profile_enable(["leaf"])     # leaf events only: the roofline kernel (events elsewhere end PDL overlap)
+        l0 = ck.launch_count()
+        if collect:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        h0 = time.perf_counter()
+        for _ in range(args.steps):
+            step()
+        host_ms += (time.perf_counter() - h0) * 1e3 / args.steps   # enqueue time per step (host)
+        e1.record()
+        torch.cuda.synchronize()
+        launches += ck.launch_count() - l0
+        ck.profile_enable(False)
+        ms = e0.elapsed_time(e1) / args.steps
+        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        if collect:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dist.barrier()
+        ms_max += float(t.item())
+        lm, ln = ck.profile_read("leaf")
+        leaf_ms += lm
+        leaf_n += ln
+        ck.profile_reset()
+        if len(snaps) > 1:
+            # all trees kept, without references to this snapshot's arrays
+            for t in keep:
+                if isinstance(t, ck.Tree):
+                    t.detach_inputs()
+            kept_trees.append(list(keep))
+            per_snap.append({"snapshot": snap, "ms": round(float(t.item()), 4),
+                             "flagged_chunks_per_gpu": local_counts[0],
+                             "diff_elems_per_gpu": local_counts[1]})
     clocks = sampler.stop()
-    ms = e0.elapsed_time(e1) / args.steps
-    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.barrier()
-    ms_max = float(t.item())
-    leaf_ms, leaf_n = ck.profile_read("leaf")
-    ck.profile_reset()
     # per-phase device times from a separate profiled pass (events around every family)
     k_prof = max(3, min(args.steps, 20))
     ck.profile_enable(True)
@@ -404,7 +461,7 @@ def run_ours(args):
         except Exception:
             traffic = None
 
-    value = bytes_pair * world / (ms_max / 1e3) / 1e9
+    value = bytes_pair * len(snaps) * world / (ms_max / 1e3) / 1e9
 
     # end-to-end through the public API with host buffers (pinned), H2D+D2H inside
     e2e = None
@@ -417,14 +474,14 @@ def run_ours(args):
 
         def timed(fn):
             fn()                                         # warm-up
-            if world > 1:
+            if collect:
                 dist.barrier()
             t0 = time.perf_counter()
             for _ in range(k_e2e):
                 out = fn()
             dt = (time.perf_counter() - t0) / k_e2e
             tt = torch.tensor([dt], dtype=torch.float64, device="cuda")
-            if world > 1:
+            if collect:
                 dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             return float(tt.item()), out
 
@@ -455,10 +512,10 @@ def run_ours(args):
             "dtype": f"{'f64' if A[0].dtype == torch.float64 else 'f32'} in, f64 quantize/compare, u64 hash",
             "data": f"synthetic (seeded, synth {CFG} recipe)",
             "config": {"workload": WORKLOAD, "name": CFG, "elements_per_array": N_PARTICLES,
-                       **({"snapshot": SNAPSHOT, "hacc_ranks_per_gpu": C4_RANKS // world}
+                       **({"snapshots": snaps, "hacc_ranks_per_gpu": C4_RANKS // world}
                           if CFG == "c4" else {}),
                        "arrays_per_run": n_arrays,
-                       "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair,
+                       "chunk_bytes": CHUNK, "eps": EPS, "bytes_per_step_per_gpu": bytes_pair * len(snaps),
                        "l2": f"inputs larger than L2 ({bytes_pair / 1e9:.1f} GB per GPU per step >> 126 MB)",
                        "parallelism": f"dp{world} (checkpoint arrays sharded by rank)",
                        "path": args.path,
@@ -473,12 +530,32 @@ def run_ours(args):
             "phases_profiled_pass": phases, "host_enqueue_ms_per_step": round(host_ms, 4),
             "flagged_chunks_per_gpu": local_counts[0], "diff_elems_per_gpu": local_counts[1],
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
-            "direct_k5": direct_k5,
+            "direct_k5": direct_k5, "dist": nccl_info,
         }
+        if per_snap:
+            line["snapshot_sequence"] = {
+                "what": "one step = the 10-snapshot sequence; per-snapshot device ms summed, every "
+                        "snapshot's trees kept", "per_snapshot": per_snap,
+                "trees_kept": 2 * len(kept_trees)}
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if collect:
         dist.destroy_process_group()
     return 0
+
+
+def free_port() -> int:
+    import socket
+    with socket.socket(socket.AF_INET, socket.SOCK_STREAM) as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def spawn_ranks(n: int) -> int:
+    """Re-launch this command as n ranks (one per GPU) through torch.distributed.run."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()),
+           os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -489,11 +566,18 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--collectives", action="store_true",
+                    help="run the per-step C1/C2 exchange even at N=1 (under a launcher)")
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--path", default="fused", choices=["fused", "unfused", "saved"],
                     help="fused: ckpt_compare_pair_async; unfused: build_batch + diff_verify_async; "
                          "saved: ckpt_compare_saved (A = stored tree + pinned host data)")
     ap.add_argument("--snapshot", type=int, default=9, help="c4: snapshot index 0..9")
+    ap.add_argument("--snapshots", default="one", choices=["one", "all"],
+                    help="c4: 'all' = BASELINE configs[3] as written, the 10-snapshot sequence")
+    ap.add_argument("--n", type=int, default=0,
+                    help="elements per array (0 = the config's full size; smaller sizes are for "
+                         "tests and are marked REDUCED in the workload)")
     ap.add_argument("--chunk", type=int, default=4096, help="chunk bytes (configs[2] sweeps 512..65536)")
     ap.add_argument("--eps", type=float, default=1e-6)
     ap.add_argument("--hash-block", type=int, default=16,
@@ -508,6 +592,11 @@ def main():
     SNAPSHOT = args.snapshot
     N_PARTICLES = CONFIGS[CFG]["n"]
     WORKLOAD = CONFIGS[CFG]["workload"]
+    if args.n:
+        N_PARTICLES = args.n
+        WORKLOAD = f"REDUCED ({args.n} elements per array, not a bench line): " + WORKLOAD
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn_ranks(args.gpus)
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

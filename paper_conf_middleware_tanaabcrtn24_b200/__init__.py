@@ -51,15 +51,20 @@ _lib = None
 
 
 def lib():
-    """Load libckpt.so (in-tree).  Raises if it is missing: there is no fallback."""
+    """Load the in-tree libckpt.so.  Raises if it is missing: there is no fallback."""
     global _lib
     if _lib is not None:
         return _lib
-    path = os.environ.get("CKPT_LIB", _build.LIB)   # CKPT_LIB: a tuning variant of libckpt.so
+    path = _build.LIB
     if not os.path.exists(path):
         raise ImportError(
             f"libckpt.so not built at {path}; run `python -c 'import __graft_entry__ as g; g.build()'`")
-    L = ctypes.CDLL(path)
+    _lib = _declare(ctypes.CDLL(path))
+    return _lib
+
+
+def _declare(L):
+    """Argument and result types of the C ABI (include/ckpt.h)."""
     vp, u64, u32, i32, dbl = (ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int,
                               ctypes.c_double)
     pp = ctypes.POINTER(ctypes.c_void_p)
@@ -123,7 +128,6 @@ def lib():
                  "ckpt_tree_info", "ckpt_tree_root", "ckpt_tree_array_roots", "ckpt_tree_nodes",
                  "ckpt_tree_array_info", "ckpt_tree_wait"):
         getattr(L, name).restype = i32
-    _lib = L
     return L
 
 
@@ -168,6 +172,19 @@ def _check_arrays(arrays: Sequence[torch.Tensor]) -> int:
     return code
 
 
+def _check_out(t: torch.Tensor, what: str, min_numel: int = 0) -> None:
+    """Output / device-count buffers handed to the kernels: int64, contiguous, on the current
+    CUDA device, at least min_numel elements (numel() is passed as the capacity)."""
+    if not isinstance(t, torch.Tensor) or t.dtype != torch.int64:
+        raise TypeError(f"{what} must be an int64 tensor")
+    if not t.is_cuda or t.device.index != torch.cuda.current_device():
+        raise ValueError(f"{what} must live on the current CUDA device")
+    if not t.is_contiguous():
+        raise ValueError(f"{what} must be contiguous")
+    if t.numel() < min_numel:
+        raise ValueError(f"{what} needs at least {min_numel} elements")
+
+
 def _ptr_array(ts: Sequence[torch.Tensor]):
     arr = (ctypes.c_void_p * len(ts))(*[t.data_ptr() for t in ts])
     return ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p)), arr
@@ -197,6 +214,11 @@ class Tree:
         self.n_leaves = nl.value
         self.n_levels = nlev.value
         self.n_nodes = nn.value
+
+    def detach_inputs(self) -> None:
+        """Drop the references to the input arrays: call once the work that built the tree has
+        completed on its stream (e.g. after a synchronize) to keep the tree without its data."""
+        self._keep = []
 
     @property
     def handle(self):
@@ -381,6 +403,9 @@ def compare_saved(saved_a: bytes, arrays_a, arrays_b, chunks: torch.Tensor, idx:
         if not t.is_contiguous():
             raise ValueError("arrays must be contiguous")
     code = _check_arrays(lb)
+    _check_out(chunks, "chunks")
+    _check_out(idx, "idx")
+    _check_out(counts, "counts", 2)
     buf, nbytes = _host_blob(saved_a)
     hdr = ctypes.string_at(buf, 16) if nbytes >= 16 else b""
     if len(hdr) == 16 and int.from_bytes(hdr[12:16], "little") != code:
@@ -413,6 +438,8 @@ def tree_diff(ta: Tree, tb: Tree, cap: Optional[int] = None, stream=None) -> tor
 def tree_diff_async(ta: Tree, tb: Tree, chunks: torch.Tensor, count: torch.Tensor, T: int = 0,
                     stream=None):
     """Step 3 without a host round trip: count lands in count[0] on the device."""
+    _check_out(chunks, "chunks")
+    _check_out(count, "count", 1)
     _check(lib().ckpt_tree_diff_async(ta.handle, tb.handle, T, chunks.data_ptr(), chunks.numel(),
                                       count.data_ptr(), _stream_ptr(stream)), "ckpt_tree_diff_async")
 
@@ -448,6 +475,10 @@ def verify_async(arrays_a, arrays_b, chunks: torch.Tensor, n_chunks_dev: torch.T
     """Step 4 over a multi-array checkpoint; chunk count read on the device."""
     ta, tb = _as_list(arrays_a), _as_list(arrays_b)
     code = _check_arrays(ta + tb)
+    _check_out(chunks, "chunks")
+    _check_out(n_chunks_dev, "n_chunks_dev", 1)
+    _check_out(out, "out")
+    _check_out(count_dev, "count_dev", 1)
     pa, _k1 = _ptr_array(ta)
     pb, _k2 = _ptr_array(tb)
     pn, _k3 = _u64_array([t.numel() for t in ta])
@@ -601,6 +632,9 @@ def diff_verify_async(ta: Tree, tb: Tree, arrays_a, arrays_b, chunks: torch.Tens
     counts[0] / counts[1] (device int64) receive the flagged-chunk and differing-element counts."""
     ta_l, tb_l = _as_list(arrays_a), _as_list(arrays_b)
     _check_arrays(ta_l + tb_l)
+    _check_out(chunks, "chunks")
+    _check_out(idx, "idx")
+    _check_out(counts, "counts", 2)
     pa, _k1 = _ptr_array(ta_l)
     pb, _k2 = _ptr_array(tb_l)
     L = lib()
@@ -629,6 +663,9 @@ def compare_pair_async(arrays_a, arrays_b, chunk_bytes: int, eps: float, chunks:
     if len(la) != len(lb) or any(x.numel() != y.numel() for x, y in zip(la, lb)):
         raise ValueError("A and B must have the same arrays and lengths")
     code = _check_arrays(la + lb)
+    _check_out(chunks, "chunks")
+    _check_out(idx, "idx")
+    _check_out(counts, "counts", 2)
     pa, _k1 = _ptr_array(la)
     pb, _k2 = _ptr_array(lb)
     pn, _k3 = _u64_array([t.numel() for t in la])

@@ -526,8 +526,9 @@ static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
 // One leaf-kernel launch over every array of every tree in `table`.
 static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t tasks,
                                  ckpt_dtype dtype, double eps, uint32_t C, uint32_t hash_block,
-                                 cudaStream_t s, int sms, const PairParams *pair = nullptr,
-                                 unsigned long long *ticket = nullptr) {
+                                 cudaStream_t s, int sms, const PairParams *pair,
+                                 unsigned long long *ticket) {
+    if (!ticket) return fail(CKPT_EINVAL, "leaf launch without a task ticket");
     LeafParams P;
     std::memset(&P, 0, sizeof(P));
     quant_params(eps, &P.q);
@@ -589,15 +590,6 @@ static ckpt_status get_pair_flags(int dev, cudaStream_t s, size_t n, uint8_t **f
 }
 
 constexpr int kLeafTicketSlot = 16;   // 8-byte slot of the per-stream ticket block used by K1
-
-// CKPT_LEAF_STATIC=1: K1 warps stride over tasks statically (A/B measurement only).
-static bool leaf_static_tasks() {
-    static const bool on = [] {
-        const char *e = std::getenv("CKPT_LEAF_STATIC");
-        return e && e[0] == '1';
-    }();
-    return on;
-}
 
 // CKPT_TILE_GATHER=1: always place the fused path's chunk list with tile_gather_kernel
 // (A/B and tests of that path; by default K4a reads the tiles itself).
@@ -726,7 +718,7 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
         pp.n_pair = task / 2;                  // A's tasks; B's are the same count
         st = get_pair_ctr(dev, s, pp.n_pair, &pp.ctr);
     }
-    if (st == CKPT_OK && !leaf_static_tasks()) {   // in-order dynamic tasks (no tail imbalance)
+    if (st == CKPT_OK) {   // in-order dynamic tasks (no tail imbalance)
         uint64_t *unused_states;
         uint32_t unused_epoch;
         st = get_scratch(dev, s, 0, &unused_states, &ticket, &unused_epoch);
@@ -920,6 +912,20 @@ static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_
     *ticket = sc.ticket;
     *epoch = sc.epoch;
     return CKPT_OK;
+}
+
+// Free every scratch buffer of (dev, s) on s and forget the entry: called before a
+// stream the library created for one call (compare_host / compare_stream) is
+// destroyed, so per-call streams do not leave scratch allocations behind.
+static void release_scratch(int dev, cudaStream_t s) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    auto it = g_scr.find(std::make_pair(dev, s));
+    if (it == g_scr.end()) return;
+    Scratch &sc = it->second;
+    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile};
+    for (void *b : bufs)
+        if (b) cudaFreeAsync(b, s);
+    g_scr.erase(it);
 }
 
 // Stream-ordered work buffer of at least `bytes` (grows, never shrinks).
@@ -1471,6 +1477,7 @@ extern "C" ckpt_status ckpt_compare_host(const void *const *a, const void *const
     if (dchunks) cudaFreeAsync(dchunks, sk);
     if (didx) cudaFreeAsync(didx, sk);
     if (dc) cudaFreeAsync(dc, sk);
+    release_scratch(dev, sk);
     cudaStreamSynchronize(sk);
     cudaStreamDestroy(sk);
     if (st != CKPT_OK) return st;
@@ -1671,6 +1678,7 @@ extern "C" ckpt_status ckpt_compare_stream(const void *const *a, const void *con
     if (dchunks) cudaFreeAsync(dchunks, sk);
     if (didx) cudaFreeAsync(didx, sk);
     if (dc) cudaFreeAsync(dc, sk);
+    release_scratch(dev, sk);
     cudaStreamSynchronize(sk);
     for (int i = 0; i < 2; ++i) {
         if (copied[i]) cudaEventDestroy(copied[i]);
@@ -1976,18 +1984,3 @@ extern "C" ckpt_status ckpt_profile_timeline(double *out, uint64_t cap, uint64_t
     }
     return CKPT_OK;
 }
-
-#ifdef CKPT_LEAF_TRACE
-// debug builds only (tools/leaf_trace.py): the last leaf launch's per-warp trace
-extern "C" int ckpt_debug_leaf_trace(uint64_t *host_out, int max_warps) {
-    const int n = max_warps < kTraceWarps ? max_warps : kTraceWarps;
-    if (cudaMemcpyFromSymbol(host_out, g_leaf_trace, (size_t)n * 3 * 8) != cudaSuccess) return -1;
-    return n;
-}
-#endif
-
-#ifdef CKPT_LEVELS_TRACE
-extern "C" int ckpt_debug_levels_trace(uint64_t *host_out) {
-    return cudaMemcpyFromSymbol(host_out, g_lv_trace, sizeof(uint64_t) * (kLvTraceCtas * 4 + 16)) == cudaSuccess ? 0 : -1;
-}
-#endif

@@ -626,7 +626,7 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
     for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + (threadIdx.x >> 5)) * G; q0 < n_chunks;
          q0 += n_warps * G) {
       uint64_t my_off = 0, my_gb = 0, my_key = 0;
-      uint32_t c = 0;
+      uint32_t c = 0, my_groups = 0;
       if (lane < (int)G && q0 + lane < n_chunks) {
           my_key = q0 + lane;
           c = p.cnt[my_key];
@@ -635,6 +635,9 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
               uint64_t len;
               my_off = p.off[q0 + lane];
               verify_locate(p, q0 + lane, ESZ, pa, pb, len, my_gb);
+              // mark_chunk wrote ceil(len/1024) groups; the rest of the chunk's slot holds
+              // stale words (a short last chunk of an array) and must not be read
+              my_groups = (uint32_t)((len + 1023) / 1024);
           }
       }
       // sparse chunks: one lane each
@@ -642,7 +645,7 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
           const uint4 *mw = reinterpret_cast<const uint4 *>(p.mask + my_key * n_words);
           uint64_t o = my_off;
 #pragma unroll 1
-          for (uint32_t w4 = 0; w4 < n_words / 4; ++w4) {
+          for (uint32_t w4 = 0; w4 < my_groups * 8u; ++w4) {
               const uint4 v = __ldcs(mw + w4);
               const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
@@ -659,9 +662,10 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
         const int j = __ffs(todo) - 1;
         const uint64_t gbase = __shfl_sync(kFull, my_gb, j);
         uint64_t pos = __shfl_sync(kFull, my_off, j);
+        const uint32_t groups = __shfl_sync(kFull, my_groups, j);
         const uint32_t *mq = p.mask + __shfl_sync(kFull, my_key, j) * n_words + lane;
 #pragma unroll 1
-        for (uint32_t g = 0; g < p.groups; ++g)
+        for (uint32_t g = 0; g < groups; ++g)
             pos += emit_words(__ldcs(mq + g * 32), gbase + (uint64_t)g * 1024, pos, p.out, p.cap, lane,
                               s_off);
       }

@@ -31,46 +31,27 @@ struct LeafArray {            // one array of the checkpoint (device table)
     uint64_t chunk_base;      // global chunk id of this array's chunk 0 in its tree
 };
 
-#ifndef CKPT_LEAF_SEG
-#define CKPT_LEAF_SEG 128
-#endif
-#ifndef CKPT_LEAF_STAGES
-#define CKPT_LEAF_STAGES 2
-#endif
-#ifndef CKPT_LEAF_MINB
-#define CKPT_LEAF_MINB 3
-#endif
-#ifndef CKPT_LEAF_CH
-#define CKPT_LEAF_CH 1
-#endif
-#ifndef CKPT_LEAF_UNROLL
-#define CKPT_LEAF_UNROLL 2      // f32 stage-loop unroll (see the fast path)
-#endif
-#ifndef CKPT_LEAF_WARPS
-#define CKPT_LEAF_WARPS 8
-#endif
-constexpr int kLeafWarps = CKPT_LEAF_WARPS;    // warps per CTA
-constexpr int kCh = CKPT_LEAF_CH;              // chains (chunks) per lane
-constexpr int kLeafUnroll = CKPT_LEAF_UNROLL;  // f32 stage-loop unroll
-constexpr int kRows = 32 * kCh;                // chunks per warp task
-constexpr int kSeg = CKPT_LEAF_SEG;            // bytes per chunk per stage
-constexpr int kStages = CKPT_LEAF_STAGES;      // ring depth
+// Geometry (measured choices): 8-warp CTAs, 3 CTAs per SM (80
+// registers), 128-byte segments per chunk per stage, a 2-slot ring, the f32 stage loop
+// unrolled x2.
+constexpr int kLeafWarps = 8;                  // warps per CTA
+constexpr int kLeafMinBlocks = 3;              // resident CTAs per SM (register cap)
+constexpr int kLeafUnroll = 2;                 // f32 stage-loop unroll
+constexpr int kRows = 32;                      // chunks per warp task (one chain per lane)
+constexpr int kSeg = 128;                      // bytes per chunk per stage
+constexpr int kStages = 2;                     // ring depth
 constexpr int kPitch = kSeg + 16;    // padded row
 constexpr int kSlotBytes = kRows * kPitch;
 constexpr int kWarpSmem = kStages * kSlotBytes;
 constexpr int kLeafSmem = kLeafWarps * kWarpSmem + 16;   // + the two h*5+c addends
 
-// L2 prefetch size hint of the staging copies (tuning knob; 128 B is the product)
-#ifndef CKPT_LEAF_L2PF
-#define CKPT_LEAF_L2PF ".L2::128B"
-#endif
 __device__ __forceinline__ void cp_async16(uint32_t smem, const void *gptr, uint32_t src_bytes) {
-    asm volatile("cp.async.cg.shared.global" CKPT_LEAF_L2PF " [%0], [%1], 16, %2;\n" ::"r"(smem), "l"(gptr),
+    asm volatile("cp.async.cg.shared.global.L2::128B [%0], [%1], 16, %2;\n" ::"r"(smem), "l"(gptr),
                  "r"(src_bytes)
                  : "memory");
 }
 __device__ __forceinline__ void cp_async16_full(uint32_t smem, const void *gptr) {
-    asm volatile("cp.async.cg.shared.global" CKPT_LEAF_L2PF " [%0], [%1], 16;\n" ::"r"(smem), "l"(gptr)
+    asm volatile("cp.async.cg.shared.global.L2::128B [%0], [%1], 16;\n" ::"r"(smem), "l"(gptr)
                  : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
@@ -123,18 +104,10 @@ __device__ __forceinline__ uint4 words_fast(uint4 v, const QuantParams &q, bool 
         const float x0 = __uint_as_float(v.x), x1 = __uint_as_float(v.y);
         const float x2 = __uint_as_float(v.z), x3 = __uint_as_float(v.w);
         const double d0 = (double)x0, d1 = (double)x1, d2 = (double)x2, d3 = (double)x3;
-#ifdef CKPT_RANGE_F64
-        // range test on the FP64 pipe (DSETP) instead of the ALU pipe
-        ok = ok & (fabs(d0) < q.r64) & (fabs(d1) < q.r64) & (fabs(d2) < q.r64) & (fabs(d3) < q.r64);
-#elif defined(CKPT_RANGE_FSETP)
-        ok = ok & (fabsf(x0) < q.r32) & (fabsf(x1) < q.r32) & (fabsf(x2) < q.r32) &
-             (fabsf(x3) < q.r32);
-#else
         // running NaN-propagating max of |x| (two 3-input FMNMX3.NAN per block instead of
         // four FSETP); compared with r32 once per task
         asm("max.NaN.f32 %0, %1, %2, %3;" : "=f"(mx) : "f"(fabsf(x0)), "f"(fabsf(x1)), "f"(mx));
         asm("max.NaN.f32 %0, %1, %2, %3;" : "=f"(mx) : "f"(fabsf(x2)), "f"(fabsf(x3)), "f"(mx));
-#endif
         // k mod 2^32 = low word of RD(x*inv + 1.5*2^52)   (hash.cuh)
         w.x = (uint32_t)__double2loint(__fma_rd(d0, q.inv, kMagic));
         w.y = (uint32_t)__double2loint(__fma_rd(d1, q.inv, kMagic));
@@ -232,16 +205,6 @@ __device__ __noinline__ void wide_end(uint64_t &h1, uint64_t &h2, const uint8_t 
 
 constexpr int kLeafInline = 16;
 
-#ifdef CKPT_LEAF_TRACE
-constexpr int kTraceWarps = 8192;
-__device__ uint64_t g_leaf_trace[3 * kTraceWarps];
-__device__ __forceinline__ uint32_t smid() {
-    uint32_t r;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
-    return r;
-}
-#endif
-
 // Fused pair mode: the table holds checkpoint A's m
 // arrays then B's m arrays (identical shapes); warp task t < n_pair is A's
 // task t, t >= n_pair is B's task t - n_pair (the usual batch order, so the
@@ -307,8 +270,8 @@ struct LeafParams {
     uint32_t chunk;
     QuantParams q;
     PairParams pr;
-    // non-null: warps draw tasks in order from this counter (0 at launch; the
-    // final draw resets it), so a warp held up by marking takes fewer tasks
+    // warps draw tasks in order from this counter (0 at launch; the final draw
+    // resets it), so a warp held up elsewhere takes fewer tasks
     unsigned long long *ticket;
     // hash block in 16-byte pieces (WIDE kernels only): B = 16*hb16 <= C bytes;
     // B = C is one Murmur3F call per chunk
@@ -325,24 +288,17 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
 }
 
 // CB = chunk bytes if known at compile time (multiple of kSeg), else 0.
-// A task is kRows = 32*kCh consecutive chunks of one array; lane l owns the
-// chains of rows l, l+32, ... (kCh independent chains per lane give the
-// scheduler two interleavable instruction streams).
+// A task is kRows = 32 consecutive chunks of one array; lane l owns the chain
+// of chunk l of the task.
 // WIDE: hash blocks of P.hb16 pieces (reading R23) instead of the paper's
 // default 16-byte blocks.
 // Chunks of >= 32 KB give few, long chains (often fewer than the GPU holds):
 // those instantiations drop the 3-CTA register cap so ptxas keeps more of a
 // chain's independent work in flight (measured +1-7% at 32 KB, +5-22% at 64 KB).
 template <int DT, bool RAW, int CB, bool PAIR, bool WIDE = false>
-__global__ void __launch_bounds__(kLeafWarps * 32, CB >= 32768 ? 1 : CKPT_LEAF_MINB)
+__global__ void __launch_bounds__(kLeafWarps * 32, CB >= 32768 ? 1 : kLeafMinBlocks)
 leaf_kernel(const __grid_constant__ LeafParams P) {
     pdl_enter();
-#ifdef CKPT_LEAF_TRACE
-    // debug build only: per-warp start / end globaltimer and tasks done (tools/leaf_trace.py)
-    uint64_t t_start;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
-    uint32_t n_done = 0;
-#endif
     // small array tables travel in the kernel parameters (no H2D copy per build)
     const LeafArray *arrays = P.n_arrays <= kLeafInline ? P.inl : P.arrays;
     const int n_arrays = P.n_arrays;
@@ -360,7 +316,7 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
     constexpr int kLoads = kRows / kChunksPerInstr;        // cp.async per lane per stage
     const int my_q = lane / kPiecesPerChunk;                // first row I load
     const int my_sub = lane % kPiecesPerChunk;
-    const uint32_t my_row = ring + (uint32_t)lane * kPitch;  // the first row I hash
+    const uint32_t my_row = ring + (uint32_t)lane * kPitch;  // the row I hash
     // keep the h*5+c addends in vector registers (a uniform-register pair cannot be the
     // 64-bit addend of IMAD.WIDE; ptxas would split the add into IADD3 + IADD3.X)
     {
@@ -383,17 +339,14 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
         }
         return __shfl_sync(0xffffffffu, t, 0);
     };
-    for (uint64_t task = P.ticket ? draw() : (uint64_t)blockIdx.x * cta_warps + warp; task < n_tasks;
-         task = P.ticket ? draw() : task + n_warps_grid) {
+    for (uint64_t task = draw(); task < n_tasks; task = draw()) {
         const int a = find_array(arrays, n_arrays, task);
         const LeafArray A = arrays[a];
         const uint64_t c0 = (task - A.task_begin) * kRows;   // first local chunk of the task
         // wide blocks take the fast path only when they tile the chunk exactly
         const bool full_task = (C % kSeg == 0) && (c0 + kRows) <= A.n_full &&
                                (!WIDE || (C / 16) % P.hb16 == 0);
-        U64p h1[kCh], h2[kCh];
-#pragma unroll
-        for (int j = 0; j < kCh; ++j) { h1[j] = U64p{0u, 0u}; h2[j] = U64p{0u, 0u}; }
+        U64p h1{0u, 0u}, h2{0u, 0u};
         bool done = false;
 
         if (full_task) {
@@ -418,13 +371,11 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             src += (kStages - 1) * kSeg;
             uint32_t slot = 0u;                                   // slot of stage s
             uint32_t nslot = (kStages - 1) * kSlotBytes;          // slot of stage s+kStages-1
-#ifndef CKPT_LEAF_NO_UNROLL2
-            // two stages per iteration: the odd stage's cp.async addresses are the even
+            // two stages per iteration (f32): the odd stage's cp.async addresses are the even
             // stage's + kSeg, an immediate offset (LDGSTS takes +-2 KB), so the 16 64-bit
             // address adds per stage are paid every other stage (86.5 -> 83.1 instructions
             // per 16-byte block; c2 pair launch 722 -> 706 us)
 #pragma unroll (DT == 0 ? kLeafUnroll : 1)
-#endif
             for (uint32_t s = 0; s < n_stages; ++s) {
                 if (s + kStages - 1 < n_stages) issue(src, nslot);
                 src += kSeg;
@@ -435,14 +386,11 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
                 const uint32_t row = my_row + slot;
 #pragma unroll
                 for (int b = 0; b < kPiecesPerChunk; ++b) {
-                    if constexpr (WIDE && kCh == 1) {   // wide blocks: one chain per lane
+                    if constexpr (WIDE) {
                         const uint4 w = words_fast<DT, RAW>(lds128(row + b * 16), q, ok, mx);
-                        wide_piece(h1[0], h2[0], w, q, left, hb16);
+                        wide_piece(h1, h2, w, q, left, hb16);
                     } else {
-#pragma unroll
-                        for (int j = 0; j < kCh; ++j)
-                            chain_block_fast<DT, RAW>(h1[j], h2[j], lds128(row + j * 32 * kPitch + b * 16),
-                                                      q, ok, mx);
+                        chain_block_fast<DT, RAW>(h1, h2, lds128(row + b * 16), q, ok, mx);
                     }
                 }
                 __syncwarp();
@@ -454,104 +402,89 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
         }
         if (!done) {
             // ------ exact path: ragged last task of an array, or a retry ------
-#pragma unroll 1
-            for (int j = 0; j < kCh; ++j) {
-                const uint64_t cj = c0 + 32 * j;                  // 32 chunks at a time
-                const uint64_t my_chunk = cj + lane;
-                uint64_t my_len = 0;
-                if (my_chunk < A.n_leaves) {
-                    const uint64_t off = my_chunk * C;
-                    my_len = (A.nbytes - off) < C ? (A.nbytes - off) : C;
-                }
-                U64p e1{0u, 0u}, e2{0u, 0u};
-                auto issue = [&](uint32_t s) {
-                    const uint32_t slot = ring + (s % kStages) * kSlotBytes;
-#pragma unroll
-                    for (int i = 0; i < 32 / kChunksPerInstr; ++i) {
-                        const int qq = my_q + i * kChunksPerInstr;
-                        const uint64_t chunk = cj + qq;
-                        const uint64_t rel = (uint64_t)(s * kSeg + my_sub * 16);
-                        const uint64_t off = chunk * C + rel;
-                        uint32_t nb = 0;
-                        if (chunk < A.n_leaves && off < A.nbytes && rel < C) {
-                            uint64_t rem = A.nbytes - off;
-                            const uint64_t crem = C - rel;
-                            if (crem < rem) rem = crem;
-                            // a piece shorter than 16 bytes is the chunk's Murmur3F tail,
-                            // hashed from global memory (chain_tail / wide_end): not staged
-                            nb = rem >= 16 ? 16u : 0u;
-                        }
-                        const uint8_t *sp = nb ? (A.data + off) : A.data;
-                        cp_async16(slot + qq * kPitch + my_sub * 16, sp, nb);
-                    }
-                };
-#pragma unroll
-                for (int s = 0; s < kStages - 1; ++s) {
-                    if ((uint32_t)s < n_stages) issue(s);
-                    cp_async_commit();
-                }
-                const uint64_t full_blocks = my_len / 16;
-                // wide blocks: bytes in the open block of B = bbytes
-                const uint32_t bbytes = WIDE ? P.hb16 * 16u : 16u;
-                uint32_t blen = 0;
-                for (uint32_t s = 0; s < n_stages; ++s) {
-                    if (s + kStages - 1 < n_stages) issue(s + kStages - 1);
-                    cp_async_commit();
-                    cp_async_wait<kStages - 1>();
-                    __syncwarp();
-                    const uint32_t row = my_row + (s % kStages) * kSlotBytes;
-#pragma unroll
-                    for (int b = 0; b < kPiecesPerChunk; ++b) {
-                        const uint64_t blk = (uint64_t)s * kPiecesPerChunk + b;
-                        if (blk < full_blocks) {
-                            if constexpr (WIDE) {
-                                const uint4 w = words_exact<DT, RAW>(lds128(row + b * 16), q);
-                                mm3p_body(e1, e2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
-                                blen += 16u;
-                                if (blen == bbytes) { mm3p_final(e1, e2, bbytes); blen = 0u; }
-                            } else {
-                                chain_block_exact<DT, RAW>(e1, e2, lds128(row + b * 16), q);
-                            }
-                        }
-                    }
-                    __syncwarp();
-                }
-                cp_async_wait<0>();
-                __syncwarp();
-                const uint32_t tail = (uint32_t)(my_len & 15);
-                if (WIDE ? (tail | blen) != 0u : tail != 0u) {
-                    uint64_t t1 = ((uint64_t)e1.hi << 32) | e1.lo, t2 = ((uint64_t)e2.hi << 32) | e2.lo;
-                    if constexpr (WIDE)
-                        wide_end<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail,
-                                          blen + tail, q);
-                    else
-                        chain_tail<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail, q);
-                    e1 = U64p{(uint32_t)t1, (uint32_t)(t1 >> 32)};
-                    e2 = U64p{(uint32_t)t2, (uint32_t)(t2 >> 32)};
-                }
-#pragma unroll
-                for (int jj = 0; jj < kCh; ++jj)
-                    if (jj == j) { h1[jj] = e1; h2[jj] = e2; }
+            const uint64_t my_chunk = c0 + lane;
+            uint64_t my_len = 0;
+            if (my_chunk < A.n_leaves) {
+                const uint64_t off = my_chunk * C;
+                my_len = (A.nbytes - off) < C ? (A.nbytes - off) : C;
             }
-        }
+            U64p e1{0u, 0u}, e2{0u, 0u};
+            auto issue = [&](uint32_t s) {
+                const uint32_t slot = ring + (s % kStages) * kSlotBytes;
 #pragma unroll
-        for (int j = 0; j < kCh; ++j) {
-            const uint64_t c = c0 + 32 * j + lane;
-            if (c < A.n_leaves) A.out[c] = make_uint4(h1[j].lo, h1[j].hi, h2[j].lo, h2[j].hi);
+                for (int i = 0; i < 32 / kChunksPerInstr; ++i) {
+                    const int qq = my_q + i * kChunksPerInstr;
+                    const uint64_t chunk = c0 + qq;
+                    const uint64_t rel = (uint64_t)(s * kSeg + my_sub * 16);
+                    const uint64_t off = chunk * C + rel;
+                    uint32_t nb = 0;
+                    if (chunk < A.n_leaves && off < A.nbytes && rel < C) {
+                        uint64_t rem = A.nbytes - off;
+                        const uint64_t crem = C - rel;
+                        if (crem < rem) rem = crem;
+                        // a piece shorter than 16 bytes is the chunk's Murmur3F tail,
+                        // hashed from global memory (chain_tail / wide_end): not staged
+                        nb = rem >= 16 ? 16u : 0u;
+                    }
+                    const uint8_t *sp = nb ? (A.data + off) : A.data;
+                    cp_async16(slot + qq * kPitch + my_sub * 16, sp, nb);
+                }
+            };
+#pragma unroll
+            for (int s = 0; s < kStages - 1; ++s) {
+                if ((uint32_t)s < n_stages) issue(s);
+                cp_async_commit();
+            }
+            const uint64_t full_blocks = my_len / 16;
+            // wide blocks: bytes in the open block of B = bbytes
+            const uint32_t bbytes = WIDE ? P.hb16 * 16u : 16u;
+            uint32_t blen = 0;
+            for (uint32_t s = 0; s < n_stages; ++s) {
+                if (s + kStages - 1 < n_stages) issue(s + kStages - 1);
+                cp_async_commit();
+                cp_async_wait<kStages - 1>();
+                __syncwarp();
+                const uint32_t row = my_row + (s % kStages) * kSlotBytes;
+#pragma unroll
+                for (int b = 0; b < kPiecesPerChunk; ++b) {
+                    const uint64_t blk = (uint64_t)s * kPiecesPerChunk + b;
+                    if (blk < full_blocks) {
+                        if constexpr (WIDE) {
+                            const uint4 w = words_exact<DT, RAW>(lds128(row + b * 16), q);
+                            mm3p_body(e1, e2, U64p{w.x, w.y}, U64p{w.z, w.w}, q.m1, q.m2);
+                            blen += 16u;
+                            if (blen == bbytes) { mm3p_final(e1, e2, bbytes); blen = 0u; }
+                        } else {
+                            chain_block_exact<DT, RAW>(e1, e2, lds128(row + b * 16), q);
+                        }
+                    }
+                }
+                __syncwarp();
+            }
+            cp_async_wait<0>();
+            __syncwarp();
+            const uint32_t tail = (uint32_t)(my_len & 15);
+            if (WIDE ? (tail | blen) != 0u : tail != 0u) {
+                uint64_t t1 = ((uint64_t)e1.hi << 32) | e1.lo, t2 = ((uint64_t)e2.hi << 32) | e2.lo;
+                if constexpr (WIDE)
+                    wide_end<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail,
+                                      blen + tail, q);
+                else
+                    chain_tail<DT, RAW>(t1, t2, A.data + my_chunk * C + (my_len - tail), tail, q);
+                e1 = U64p{(uint32_t)t1, (uint32_t)(t1 >> 32)};
+                e2 = U64p{(uint32_t)t2, (uint32_t)(t2 >> 32)};
+            }
+            h1 = e1;
+            h2 = e2;
         }
-        // pair mode assumes one chain per lane (kCh > 1 is a single-tree tuning build only)
-        if constexpr (PAIR && kCh == 1) {
+        {
+            const uint64_t c = c0 + lane;
+            if (c < A.n_leaves) A.out[c] = make_uint4(h1.lo, h1.hi, h2.lo, h2.hi);
+        }
+        if constexpr (PAIR) {
             const int side = a >= P.pr.m ? 1 : 0;
             const uint64_t pt = task - (side ? P.pr.n_pair : 0);
             // publish my leaves, then count in; the second of the pair does the compare.
-#ifdef CKPT_PAIR_FENCES
-            __threadfence();
-            unsigned int order = 0;
-            if (lane == 0) order = atomicInc(&P.pr.ctr[pt], 1u);
-            order = __shfl_sync(0xffffffffu, order, 0);
-            if (order == 1) {
-                __threadfence();
-#else
             // The warp barrier orders every lane's leaf stores before lane 0's
             // acq_rel atomic (release: cumulative over what the barrier made
             // visible to it; acquire: the other run's leaves, published by its
@@ -564,13 +497,12 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             order = __shfl_sync(0xffffffffu, order, 0);
             if (order == 1) {
                 __syncwarp();   // lane 0's acquire, then every lane's loads
-#endif
                 const LeafArray Pa = arrays[side ? a - P.pr.m : a + P.pr.m];   // the other run
                 const uint64_t c = c0 + lane;
                 bool differ = false;
                 if (c < A.n_leaves) {
                     const uint4 o = __ldcg(Pa.out + c);
-                    differ = (o.x != h1[0].lo) | (o.y != h1[0].hi) | (o.z != h2[0].lo) | (o.w != h2[0].hi);
+                    differ = (o.x != h1.lo) | (o.y != h1.hi) | (o.z != h2.lo) | (o.w != h2.hi);
                     P.pr.flags[A.chunk_base + c] = differ ? 1 : 0;
                 }
                 if (P.pr.tmask) {
@@ -595,22 +527,7 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             }
         }
         __syncwarp();
-#ifdef CKPT_LEAF_TRACE
-        ++n_done;
-#endif
     }
-#ifdef CKPT_LEAF_TRACE
-    if ((threadIdx.x & 31) == 0) {
-        uint64_t t_end;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
-        const uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-        if (w < kTraceWarps) {
-            g_leaf_trace[3 * w] = t_start;
-            g_leaf_trace[3 * w + 1] = t_end;
-            g_leaf_trace[3 * w + 2] = ((uint64_t)smid() << 32) | n_done;
-        }
-    }
-#endif
 }
 
 }  // namespace ckpt

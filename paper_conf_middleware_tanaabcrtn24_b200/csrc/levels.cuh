@@ -6,14 +6,11 @@
 // node is promoted unchanged, so any aligned group of 2^G nodes of a level is
 // an exact subtree.
 //
-// Phase 1 (every CTA, no block barrier per level): a CTA of 8 warps takes an
-//   aligned group of 4096 nodes of level ls of one array.  Each thread hashes
-//   its own aligned 16 nodes up 4 levels in registers (15 hashes, every lane
-//   busy, 8-way independent at the first level); each warp then hashes its 32
-//   subtree roots up 5 more levels with register shuffles (the right child of
-//   a level-k node comes from lane + 2^(k-5)), and warp 0 builds the last 3
-//   levels from the 8 warp roots.
-// Phase 2 (last CTA of each tree, atomic ticket): loads the remaining level
+// Phase 1 (every CTA, one per aligned group of 2048 nodes of level ls of one
+//   array): passes of two levels through shared memory -- in each pass the
+//   first ceil(cnt/4) of the 512 threads take 4 consecutive nodes and hash them
+//   two levels up (2 independent hashes, then 1), writing both levels.
+// Phase 2 (last CTA of each tree, acq_rel ticket): loads the remaining level
 //   of every array into shared memory, builds all upper levels there, then
 //   the top tree over the array roots (R15).  Levels that do not fit in
 //   shared memory are walked through L2.
@@ -25,25 +22,14 @@
 
 namespace ckpt {
 
-#ifdef CKPT_LV_OLD
-constexpr int kLevelThreads = 256;
-constexpr int kLogT = 4;                     // levels each thread builds alone
-constexpr int kPerThread = 1 << kLogT;       // nodes of level ls per thread
-constexpr int kLog = 12;
-constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA (256 threads x 16)
-#else
 constexpr int kLevelThreads = 512;
 constexpr int kLog = 11;
 constexpr int kGroup = 1 << kLog;            // nodes of level ls per CTA (512 threads x 4)
-#endif
 constexpr int kLevelSmemNodes = 1536;        // phase-2 shared memory in nodes (24 KiB)
 constexpr int kLevelSmem = kLevelSmemNodes * 16;
 constexpr int kMaxLevelTrees = 4;
 
-#ifndef CKPT_LEVEL_INLINE
-#define CKPT_LEVEL_INLINE 512
-#endif
-constexpr int kLevelInlineWords = CKPT_LEVEL_INLINE;   // 4 KiB of tree metadata in the kernel params
+constexpr int kLevelInlineWords = 512;   // 4 KiB of tree metadata in the kernel params
 
 // Per-tree launch record.  The metadata tables live in one blob (layout below)
 // that is either inline in the kernel parameters (small trees: no H2D copy;
@@ -140,41 +126,12 @@ __device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 
     }
 }
 
-#ifdef CKPT_LEVELS_TRACE
-// debug build only: per-CTA [entry, after griddepcontrol.wait, phase-1 end, ticket] and the
-// last CTA's [phase-2 levels end, top end] globaltimer stamps (tools/levels_trace.py)
-constexpr int kLvTraceCtas = 4096;
-__device__ uint64_t g_lv_trace[kLvTraceCtas * 4 + 16];
-__device__ __forceinline__ uint64_t gtime() {
-    uint64_t t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    return t;
-}
-#define LV_STAMP(slot, v) do { if (threadIdx.x == 0 && blockIdx.x < kLvTraceCtas) g_lv_trace[blockIdx.x * 4 + (slot)] = (v); } while (0)
-#define LV_STAMP_LAST(slot) do { if (threadIdx.x == 0) g_lv_trace[kLvTraceCtas * 4 + 2 * ti + (slot)] = gtime(); } while (0)
-#else
-#define LV_STAMP(slot, v) do { } while (0)
-#define LV_STAMP_LAST(slot) do { } while (0)
-#endif
 
 __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_constant__ LevelBatch pb) {
-#ifdef CKPT_LEVELS_TRACE
-    const uint64_t t_entry = gtime();
-#endif
     pdl_enter();
-#ifdef CKPT_LEVELS_TRACE
-    LV_STAMP(0, t_entry);
-    LV_STAMP(1, gtime());
-#endif
     extern __shared__ __align__(16) uint4 sm[];
-#ifdef CKPT_LV_OLD
-    __shared__ uint4 s_root[kLevelThreads / 32];
-#endif
     __shared__ unsigned int s_ticket;
     const int tid = threadIdx.x;
-#ifdef CKPT_LV_OLD
-    const int lane = tid & 31, warp = tid >> 5;
-#endif
     int ti = 0;
     while (ti + 1 < pb.n && blockIdx.x >= pb.cta_begin[ti + 1]) ++ti;
     const LevelParams &lp = pb.t[ti];
@@ -200,61 +157,6 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
         for (uint32_t w = tid; w < lp.meta_words; w += kLevelThreads) dst[w] = pb.blob[lp.inl + w];
     }
     // ------------------------------ phase 1 ------------------------------
-#ifdef CKPT_LV_OLD
-    {
-        const uint64_t gid = blockIdx.x - pb.cta_begin[ti];
-        const int a = find_le(p.gbegin, na, gid);
-        const uint64_t g = gid - p.gbegin[a];
-        const uint64_t n0 = p.cnt[(uint64_t)p.ls * na + a];
-        const uint64_t start = g * kGroup;
-        const int m0 = (int)((n0 - start) < (uint64_t)kGroup ? (n0 - start) : (uint64_t)kGroup);
-        const int h = (int)p.height[a];
-        const uint4 *src = p.nodes + p.off[(uint64_t)p.ls * na + a] + start;
-        auto write = [&](int k, uint64_t jglob, uint4 v) {
-            if (p.ls + k < h) p.nodes[p.off[(uint64_t)(p.ls + k) * na + a] + (start >> k) + jglob] = v;
-        };
-        // thread t: nodes [16t, 16t+16) of the group, 4 levels in registers
-        int mt = m0 - kPerThread * tid;
-        mt = mt < 0 ? 0 : (mt > kPerThread ? kPerThread : mt);
-        uint4 x[kPerThread / 2];
-#pragma unroll
-        for (int j = 0; j < kPerThread / 2; ++j) {
-            x[j] = make_uint4(0u, 0u, 0u, 0u);
-            if (2 * j < mt) {
-                x[j] = __ldg(src + kPerThread * tid + 2 * j);
-                if (2 * j + 1 < mt) x[j] = hash_children32(x[j], __ldg(src + kPerThread * tid + 2 * j + 1));
-                write(1, (kPerThread / 2) * tid + j, x[j]);
-            }
-        }
-        int m = (mt + 1) >> 1;
-#pragma unroll
-        for (int k = 2; k <= kLogT; ++k) {
-#pragma unroll
-            for (int j = 0; j < (kPerThread >> k); ++j) {
-                if (j < ((m + 1) >> 1)) {
-                    if (2 * j + 1 < m) x[j] = hash_children32(x[2 * j], x[2 * j + 1]);
-                    else x[j] = x[2 * j];
-                    write(k, (uint64_t)(kPerThread >> k) * tid + j, x[j]);
-                }
-            }
-            m = (m + 1) >> 1;
-        }
-        // warp w: its 32 level-kLogT nodes, lane l holding node l, up 5 levels
-        int mw = ((m0 + kPerThread - 1) >> kLogT) - 32 * warp;
-        mw = mw < 0 ? 0 : (mw > 32 ? 32 : mw);
-        constexpr int kWarpSpan = 32 * kPerThread;          // group nodes per warp
-        const uint4 v = warp_levels(x[0], mw, kLogT + 1, kLogT + 5, lane, [&](int k, int j, uint4 y) {
-            write(k, (uint64_t)(kWarpSpan >> k) * warp + j, y);
-        });
-        if (lane == 0) s_root[warp] = v;
-        __syncthreads();
-        if (warp == 0) {
-            const int m9 = (m0 + kWarpSpan - 1) / kWarpSpan;  // valid warp roots
-            uint4 y = lane < m9 ? s_root[lane] : make_uint4(0u, 0u, 0u, 0u);
-            warp_levels(y, m9, kLogT + 6, kLog, lane, [&](int k, int j, uint4 z) { write(k, j, z); });
-        }
-    }
-#else
     {
         // Passes of two levels through shared memory: in pass r/2 the first
         // ceil(cnt/4) threads each take 4 consecutive level-r nodes of the
@@ -347,10 +249,6 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
             __syncthreads();
         }
     }
-#endif
-#ifdef CKPT_LEVELS_TRACE
-    LV_STAMP(2, gtime());
-#endif
     // ------------------------------ phase 2 ------------------------------
     // Last-CTA hand-off without sequentially consistent fences (MEMBAR.SC.GPU
     // costs microseconds): the barrier orders every thread's node stores before
@@ -364,9 +262,6 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
         s_ticket = t;
     }
     __syncthreads();
-#ifdef CKPT_LEVELS_TRACE
-    LV_STAMP(3, gtime());
-#endif
     if (s_ticket != p.n_groups - 1) return;
     int F = p.ls + kLog;                       // highest level phase 1 completed
     if (F > p.n_levels - 1) F = p.n_levels - 1;
@@ -393,7 +288,6 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
         }
     }
     __syncthreads();
-    LV_STAMP_LAST(0);
     // top tree: level 0 = array roots in array order (R15).  Up to 2 * kLevelSmemNodes / 3
     // roots it is built in shared memory (one L2 round trip for the roots, then only
     // stores); larger tops through L2.
@@ -422,7 +316,6 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
             at += n;
             n = up;
         }
-        LV_STAMP_LAST(1);
         if (tid == 0) *p.ticket = 0u;
         return;
     }

@@ -7,10 +7,7 @@
 
 namespace ckpt {
 
-#ifndef CKPT_VERIFY_BATCH
-#define CKPT_VERIFY_BATCH 4
-#endif
-constexpr int kVerifyBatch = CKPT_VERIFY_BATCH;   // warp iterations whose loads are issued together
+constexpr int kVerifyBatch = 4;   // warp iterations whose loads are issued together
 
 // Bits of |a-b| > eps (computed in double, reading R9) for the VEC elements
 // of one 16-byte vector pair.

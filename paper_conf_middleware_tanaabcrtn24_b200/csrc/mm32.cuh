@@ -54,22 +54,6 @@ __device__ __forceinline__ U64p rotl_gt32(U64p a) {
 
 __device__ __forceinline__ U64p xor64(U64p a, U64p b) { return U64p{a.lo ^ b.lo, a.hi ^ b.hi}; }
 
-#ifdef CKPT_ADD_WIDE
-__constant__ uint32_t c_one = 1u;   // opaque to ptxas, so "x * 1" stays an IMAD
-__device__ __forceinline__ uint32_t g_one_reg() { return c_one; }
-// a + b on the FMA pipe: IMAD.WIDE.U32 (a.lo * 1 + b) then IMAD (a.hi * 1 + hi)
-__device__ __forceinline__ U64p add64(U64p a, U64p b) {
-    U64p r;
-    asm("{\n\t.reg .u64 p, q;\n\t"
-        "mov.b64 q, {%4, %5};\n\t"
-        "mad.wide.u32 p, %2, %6, q;\n\t"
-        "mov.b64 {%0, %1}, p;\n\t"
-        "mad.lo.u32 %1, %3, %6, %1;\n\t}"
-        : "=r"(r.lo), "=r"(r.hi)
-        : "r"(a.lo), "r"(a.hi), "r"(b.lo), "r"(b.hi), "r"(g_one_reg()));
-    return r;
-}
-#else
 __device__ __forceinline__ U64p add64(U64p a, U64p b) {
     U64p r;
     asm("add.cc.u32 %0, %2, %4;\n\taddc.u32 %1, %3, %5;"
@@ -77,66 +61,17 @@ __device__ __forceinline__ U64p add64(U64p a, U64p b) {
         : "r"(a.lo), "r"(a.hi), "r"(b.lo), "r"(b.hi));
     return r;
 }
-#endif
 
-// h*5 + c (the default below): lo*5 + c with the 64-bit addend folded into
-// IMAD.WIDE.U32, then hi*5 + that product's high word.  (An inline-asm mad.wide with
-// an immediate multiplier was split by ptxas into IMAD.WIDE + IADD3 + IMAD.X:
-// 2 more instructions per block, measured 1.8% slower in the leaf kernel.)
-#if defined(CKPT_M5ASM)
-__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
-    U64p r;
-    asm("{\n\t.reg .u64 p;\n\t"
-        "mad.wide.u32 p, %2, 5, %4;\n\t"
-        "mov.b64 {%0, %1}, p;\n\t"
-        "mad.lo.u32 %1, %3, 5, %1;\n\t}"
-        : "=r"(r.lo), "=r"(r.hi)
-        : "r"(h.lo), "r"(h.hi), "l"(c));
-    return r;
-}
-#endif
-// h*5 + c on the ALU pipe: (h << 2) + h + c
-__device__ __forceinline__ U64p mul5_add_alu(U64p h, uint64_t c) {
-    U64p r;
-    asm("{\n\t.reg .u32 s, t;\n\t"
-        "shf.l.wrap.b32 t, %2, %3, 2;\n\t"
-        "shl.b32 s, %2, 2;\n\t"
-        "add.cc.u32 s, s, %2;\n\t"
-        "addc.u32 t, t, %3;\n\t"
-        "add.cc.u32 %0, s, %4;\n\t"
-        "addc.u32 %1, t, 0;\n\t}"
-        : "=r"(r.lo), "=r"(r.hi)
-        : "r"(h.lo), "r"(h.hi), "r"((uint32_t)c));
-    return r;
-}
-#if defined(CKPT_M5LEA)
-__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) { return mul5_add_alu(h, c); }
-#elif defined(CKPT_M5_64)
-// the whole 64-bit product in C: ptxas emits IMAD.WIDE.U32 + IMAD + IMAD.IADD (it splits
-// hi*5 + carry-word into two instructions)
-__device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
-    const uint64_t x = (((uint64_t)h.hi << 32) | h.lo) * 5ull + c;
-    return U64p{(uint32_t)x, (uint32_t)(x >> 32)};
-}
-#elif !defined(CKPT_M5ASM)
-// lo*5 + c as one IMAD.WIDE.U32 (64-bit addend folded), hi*5 + its high word as ONE IMAD:
-// 2 instructions instead of 3 (81.1 vs 83.1 per block; c2 pair launch 706 -> 692 us)
+// h*5 + c: lo*5 + c as one IMAD.WIDE.U32 (64-bit addend folded), then hi*5 + that
+// product's high word as ONE IMAD: 2 instructions (81.1 vs 83.1 per block with the plain
+// 64-bit product; an inline-asm mad.wide with an immediate multiplier was split by ptxas
+// into IMAD.WIDE + IADD3 + IMAD.X, measured 1.8% slower)
 __device__ __forceinline__ U64p mul5_add(U64p h, uint64_t c) {
     const uint64_t x = (uint64_t)h.lo * 5u + c;
     return U64p{(uint32_t)x, h.hi * 5u + (uint32_t)(x >> 32)};
 }
-#endif
 
-#ifdef CKPT_XS_IMAD
-// hi >> 1 as IMAD.HI.U32(hi, 2^31): moves the shift from the ALU to the FMA pipe
-__device__ __forceinline__ U64p xorshift33(U64p k) {
-    uint32_t t;
-    asm volatile("mul.hi.u32 %0, %1, 0x80000000;" : "=r"(t) : "r"(k.hi));
-    return U64p{k.lo ^ t, k.hi};
-}
-#else
 __device__ __forceinline__ U64p xorshift33(U64p k) { return U64p{k.lo ^ (k.hi >> 1), k.hi}; }
-#endif
 
 __device__ __forceinline__ U64p fmix64p(U64p k) {
     k = xorshift33(k);
@@ -165,11 +100,7 @@ __device__ __forceinline__ void mm3p_hstep(U64p &h1, U64p &h2, U64p k1, U64p k2,
     h1 = xor64(h1, k1);
     h1 = rotl_lt32<27>(h1);
     h1 = add64(h1, h2);
-#ifdef CKPT_M5MIX
-    h1 = mul5_add_alu(h1, m1);   // ALU pipe: balances the FMA-heavy pipe (IMAD.WIDE = 2 slots)
-#else
     h1 = mul5_add(h1, m1);   // m1 = 0x52dce729
-#endif
     h2 = xor64(h2, k2);
     h2 = rotl_lt32<31>(h2);
     h2 = add64(h2, h1);

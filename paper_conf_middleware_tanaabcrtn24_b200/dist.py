@@ -75,10 +75,11 @@ class RunComparison:
 
 def compare_runs(arrays_a: Sequence[torch.Tensor], arrays_b: Sequence[torch.Tensor],
                  chunk_bytes: int, eps: float, group=None, read_roots: bool = True,
-                 keep_trees: bool = False) -> RunComparison:
+                 keep_trees: bool = False, exchange: Optional[bool] = None) -> RunComparison:
     """Compare this rank's arrays of run A and run B (steps 1-4) and join the ranks.
 
-    With torch.distributed uninitialised (or world size 1) no collective runs."""
+    exchange: run C1/C2 (default: when torch.distributed is initialised with world size > 1;
+    True also at world size 1, e.g. to exercise the NCCL path on one GPU)."""
     from . import tree_build, tree_diff_async, tree_from_digests_batch, verify_async
 
     TA = tree_build(list(arrays_a), chunk_bytes, eps)
@@ -90,7 +91,8 @@ def compare_runs(arrays_a: Sequence[torch.Tensor], arrays_b: Sequence[torch.Tens
     tree_diff_async(TA, TB, chunks, counts[0:1])
     verify_async(list(arrays_a), list(arrays_b), chunks, counts[0:1], chunk_bytes, eps, idx,
                  counts[1:2])
-    distributed = dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1
+    initialised = dist.is_available() and dist.is_initialized()
+    distributed = initialised and (dist.get_world_size(group) > 1 if exchange is None else exchange)
     chunk_off = elem_off = 0
     local = counts.clone()
     if distributed:
@@ -155,15 +157,18 @@ def array_shard(n_elems: int, elem_bytes: int, chunk_bytes: int, world: int,
 
 
 def compare_sharded_array(a_local: torch.Tensor, b_local: torch.Tensor, n_total: int,
-                          chunk_bytes: int, eps: float, group=None) -> RunComparison:
+                          chunk_bytes: int, eps: float, group=None,
+                          exchange: Optional[bool] = None) -> RunComparison:
     """Compare this GPU's shard (array_shard) of ONE large array of run A and run B.
 
     Every rank builds its subtree, C1 all-gathers the shard roots (empty shards send none) and
     every rank builds the same top levels -> the single-GPU root; C2 all-reduces the counts.
     Local ids are shifted to global ones with chunk_offset / elem_offset."""
     from . import compare_pair_async, tree_from_digests
-    world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+    initialised = dist.is_available() and dist.is_initialized()
+    world = dist.get_world_size(group) if initialised else 1
     rank = dist.get_rank(group) if world > 1 else 0
+    collect = initialised and (world > 1 if exchange is None else exchange)
     lo, hi, c_lo, _ = array_shard(n_total, a_local.element_size(), chunk_bytes, world, rank)
     if a_local.numel() != hi - lo or b_local.numel() != hi - lo:
         raise ValueError(f"rank {rank} must hold elements [{lo}, {hi}) of the array")
@@ -178,7 +183,7 @@ def compare_sharded_array(a_local: torch.Tensor, b_local: torch.Tensor, n_total:
         TA = TB = None
         ra = rb = torch.zeros((0, 16), dtype=torch.uint8, device="cuda")
     local = counts.clone()
-    if world > 1:
+    if collect:
         roots_a, roots_b = gather_roots(ra, group), gather_roots(rb, group)
         allreduce_counts(counts, group)
     else:

@@ -20,7 +20,8 @@ Recipes (DESIGN.md "Input recipe"):
       eps 1e-6, C 4 KiB; 1% of particles in 64 contiguous clusters get
       d = +-10^U(-8,-3) on all six fields.
   c3  2^29 f64 ~ N(0,1); 1024 clusters, geometric length (mean 4096),
-      d = +-10^U(-9,-2).
+      d = +-10^U(-9,-2); plus 2^16 isolated d = +-10^U(-10,-1) (eps-dependent
+      flagging and false positives across the sweep).
   c4  per-rank c2-shaped arrays (rank_pair).
   c5  8 ranks x 50*2^20 particles x 6 f32 per GPU; 10% of chunks get 8 above-eps
       and 8 below-eps (bin-straddling) perturbations, another 1% only the
@@ -178,8 +179,13 @@ def c2_pair(n_particles: int = 1 << 26, seed: int = 2, device="cpu", eps: float 
 
 
 def c3_pair(n: int = 1 << 29, seed: int = 3, device="cpu", eps: float = 1e-6,
-            chunk_bytes: int = 4096, n_clusters: int = 1024, mean_len: int = 4096) -> Pair:
-    """Config 3: N(0,1) f64 with geometric-length clustered divergence."""
+            chunk_bytes: int = 4096, n_clusters: int = 1024, mean_len: int = 4096,
+            n_isolated: int = 1 << 16, iso_exp=(-10.0, -1.0)) -> Pair:
+    """Config 3: N(0,1) f64 with geometric-length clustered divergence plus `n_isolated`
+    single-element changes of log-uniform size 10^U(iso_exp) at uniform random indices: around
+    any eps of the sweep some of them exceed eps (true positives) and some smaller ones straddle
+    a bin edge (false positives), so the flagged fraction and the false-positive rate depend on
+    eps (the synthetic analogue of Fig. 7)."""
     a = normal(seed, n, device, dtype=torch.float64)
     b = a.clone()
     rng = np.random.default_rng(seed)
@@ -192,7 +198,16 @@ def c3_pair(n: int = 1 << 29, seed: int = 3, device="cpu", eps: float = 1e-6,
         sg = uniform(seed * 104729 + c, ln, device, dtype=torch.float64)
         d = torch.pow(10.0, -9.0 + 7.0 * u) * torch.where(sg < 0.5, -1.0, 1.0)
         b[sub] = b[sub] + d
-    return Pair("c3", [a], [b], chunk_bytes, eps, {"n": n})
+    if n_isolated > 0:
+        iso = torch.as_tensor(np.unique(rng.integers(0, n, size=n_isolated)), dtype=torch.int64,
+                              device=device)
+        m = iso.numel()
+        u = uniform(seed * 31337 + 1, m, device, dtype=torch.float64)
+        sg = uniform(seed * 31337 + 2, m, device, dtype=torch.float64)
+        lo, hi = iso_exp
+        d = torch.pow(10.0, lo + (hi - lo) * u) * torch.where(sg < 0.5, -1.0, 1.0)
+        b[iso] = b[iso] + d
+    return Pair("c3", [a], [b], chunk_bytes, eps, {"n": n, "n_isolated": n_isolated})
 
 
 def rank_pair(rank: int, n_particles: int, seed_base: int, device="cpu", eps: float = 1e-6,

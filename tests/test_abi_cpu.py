@@ -113,3 +113,16 @@ def test_oracle_written_tree_passes_host_validation(libckpt):
     if torch.cuda.is_available():
         pytest.skip("GPU present: covered by the GPU persistence tests")
     assert _deser(libckpt, _oracle_buf()) == -4
+
+
+def test_product_sources_have_no_tuning_switches():
+    """No compile-time tuning variants inside the product kernels and no way to swap the loaded
+    library from the environment (the product is exactly the in-tree libckpt.so)."""
+    pkg = os.path.join(ROOT, "paper_conf_middleware_tanaabcrtn24_b200")
+    csrc = os.path.join(pkg, "csrc")
+    for f in os.listdir(csrc):
+        src = open(os.path.join(csrc, f)).read()
+        assert not re.search(r"#\s*if(n?def)?\b.*\bCKPT_", src), f
+    init = open(os.path.join(pkg, "__init__.py")).read()
+    assert "CKPT_LIB" not in init
+    assert not os.path.isdir(os.path.join(csrc, "experimental"))

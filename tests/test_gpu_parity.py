@@ -148,8 +148,14 @@ def test_quantizer_specials_and_random_bit_patterns_f64(eps):
                    1.0, -1.0, 1e-5, -1e-5, 2.0 ** 51 * eps, -(2.0 ** 51) * eps, 2.0 ** 63 * eps,
                    -(2.0 ** 63) * eps, np.nextafter(2.0 ** 63 * eps, 0)], dtype=np.float64)
     x[: sp.size] = sp
-    # also values near the fast/slow-path boundary |x| ~ 2^50 * eps
-    x[sp.size: sp.size + 1000] = rng.uniform(-(2.0 ** 52), 2.0 ** 52, 1000) * eps
+    # also values near the fast/slow-path boundary |x| ~ 2^50 * eps (finite: for eps = 1e300
+    # the boundary lies beyond DBL_MAX, so the range is capped there and every value is finite)
+    scale = 2.0 ** 52 * eps
+    if not np.isfinite(scale):
+        scale = np.finfo(np.float64).max
+    near = rng.uniform(-1.0, 1.0, 1000) * scale
+    assert np.all(np.isfinite(near))
+    x[sp.size: sp.size + 1000] = near
     a = torch.from_numpy(x).cuda()
     t = ck.tree_build(a, 16, eps)
     got = gpu_tree_nodes(t)[: x.size // 2]
@@ -231,10 +237,15 @@ def test_config1_pair_end_to_end(n):
     assert np.array_equal(np_of(chunks), ref_chunks)
     truth = oracle.brute(an, bn, eps)
     assert np.array_equal(np_of(idx), truth) and cnt == truth.size
-    # paper invariants: no false negatives; straddlers were flagged and removed
+    # paper invariants: no false negatives; straddlers were flagged and removed.  The recipe
+    # is exact: the 50 "above" changes (>= 2 eps before rounding to f32, whose ulp on [-1, 1)
+    # is <= 6e-8) are exactly the differing elements, the 50 "below" ones (<= 0.5 eps) never are
     per = C // 4
     assert set(np.unique(truth // per)) <= set(ref_chunks.tolist())
-    assert truth.size == pair.meta["n_above"] or truth.size >= pair.meta["n_above"] - 2
+    above = np.sort(pair.meta["perturbed"][: pair.meta["n_above"]])
+    assert truth.size == pair.meta["n_above"] == 50 and np.array_equal(truth, above)
+    straddle = pair.meta["perturbed"][pair.meta["n_above"]: pair.meta["n_above"] + pair.meta["n_straddle"]]
+    assert set(np.unique(straddle // per)) <= set(ref_chunks.tolist())   # flagged, then removed
 
 
 @pytest.mark.parametrize("T", [1, 2, 3, 5, 17, 100, 1000, 4096, 10 ** 9])
@@ -382,31 +393,66 @@ def test_error_paths():
 
 # ------------------------------------------------- full size (configs[1]) --
 
-@pytest.mark.slow
-def test_config2_full_size_sampled_parity():
-    """BASELINE configs[1] at full size (2^26 particles x 6 f32) in the bench's launch
-    configuration: sampled leaves by the oracle, all interior levels recomputed by the
-    oracle from the GPU leaves, verify == brute force over all 805M elements."""
-    pair = synth.c2_pair(device="cuda")
+def full_checkpoint_parity(pair, TA, TB, chunks, idx, counts, brute=True):
+    """Every node of every array tree of both runs, both checkpoint roots, the chunk list and
+    the element ids of a fused compare vs the oracle, one array at a time (host memory stays
+    at one array pair).  Returns (n_chunks, n_diff)."""
     C, eps = pair.chunk_bytes, pair.eps
-    TA, TB = ck.tree_build(pair.a, C, eps), ck.tree_build(pair.b, C, eps)
-    rng = np.random.default_rng(0)
-    per = C // 4
-    for k in range(6):
-        na = gpu_tree_nodes(TA, k)
-        L = pair.a[k].numel() * 4 // C
-        sample = np.sort(rng.choice(L, 512, replace=False))
-        an = pair.a[k]
-        for c in sample:
-            chunk = np_of(an[c * per:(c + 1) * per])
-            assert np.array_equal(oracle.leaves(chunk, C, eps)[0], na[c]), (k, c)
-        assert np.array_equal(oracle.levels(na[:L]), na)
-    chunks = ck.tree_diff(TA, TB)
-    idx, n = ck.verify(pair.a, pair.b, chunks, C, eps)
-    an = [np_of(t) for t in pair.a]
-    bn = [np_of(t) for t in pair.b]
-    truth = oracle.brute_checkpoint(an, bn, eps)
-    assert n == truth.size and np.array_equal(np_of(idx), truth)
+    th = os.cpu_count() or 8
+    nc, nd = counts.tolist()
+    got_c, got_i = np_of(chunks[:nc]), np_of(idx[:nd])
+    ref_c_all, ref_i_all, roots_a, roots_b = [], [], [], []
+    cbase = ebase = 0
+    for k, (x, y) in enumerate(zip(pair.a, pair.b)):
+        an, bn = np_of(x), np_of(y)
+        la = oracle.leaves(an, C, eps, threads=th)
+        lb = oracle.leaves(bn, C, eps, threads=th)
+        na, nb = oracle.levels(la), oracle.levels(lb)
+        assert np.array_equal(gpu_tree_nodes(TA, k), na), ("tree A", k)
+        assert np.array_equal(gpu_tree_nodes(TB, k), nb), ("tree B", k)
+        rc = oracle.diff(na, nb, la.shape[0])
+        ri = oracle.verify(an, bn, C, rc, eps)
+        if brute:
+            assert np.array_equal(ri, oracle.brute(an, bn, eps)), k
+        ref_c_all.append(rc + cbase)
+        ref_i_all.append(ri + ebase)
+        roots_a.append(na[-1])
+        roots_b.append(nb[-1])
+        cbase += la.shape[0]
+        ebase += an.size
+        del an, bn, la, lb, na, nb
+    ref_c, ref_i = np.concatenate(ref_c_all), np.concatenate(ref_i_all)
+    assert nc == ref_c.size and np.array_equal(got_c, ref_c)
+    assert nd == ref_i.size and np.array_equal(got_i, ref_i)
+    assert TA.root() == oracle.levels(np.stack(roots_a))[-1].tobytes()
+    assert TB.root() == oracle.levels(np.stack(roots_b))[-1].tobytes()
+    return nc, nd
+
+
+def fused_compare(pair):
+    """The bench step's call (ckpt_compare_pair_async, default 16-byte hash blocks)."""
+    C, eps = pair.chunk_bytes, pair.eps
+    L = sum(-(-t.numel() * t.element_size() // C) for t in pair.a)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(sum(t.numel() for t in pair.a), dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(pair.a, pair.b, C, eps, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    torch.cuda.synchronize()
+    return TA, TB, chunks, idx, counts
+
+
+@pytest.mark.slow
+def test_config2_full_size_bench_path_parity():
+    """BASELINE configs[1] at full size (2^26 particles x 6 f32 per run) through the exact call
+    and launch configuration bench.py times (ckpt_compare_pair_async: the fused pair leaf kernel
+    leaf_kernel<F32, 4096-byte chunks, PAIR>, K1 tile compaction read by verify_mark): every leaf
+    and interior node of all 6 arrays of both trees, both checkpoint roots, the chunk list and
+    the element ids equal the oracle's; the ids also equal brute force."""
+    pair = synth.c2_pair(device="cuda")
+    TA, TB, chunks, idx, counts = fused_compare(pair)
+    nc, nd = full_checkpoint_parity(pair, TA, TB, chunks, idx, counts, brute=True)
+    assert nc > 0 and nd > 0
 
 
 # ------------------------------------------------ exhaustive f32 quantizer --
@@ -918,42 +964,28 @@ def test_array_beyond_2pow32_elements_fused_path():
 
 
 @pytest.mark.slow
-def test_config5_full_size_sampled_parity():
+def test_config5_full_size_parity():
     """BASELINE configs[4] per-GPU shard at full size (8 ranks x 50*2^20 particles x 6 f32,
-    20 GB per run) on the fused path: every flagged chunk and every element id of a sampled
-    set of arrays equals the oracle's over those arrays, and the global counts equal a
-    brute-force device count of |a-b| > eps (property at full size)."""
+    10 GB per run, verify-heavy: 10% of chunks with true differences, 1% planted false
+    positives) through the bench's fused call: every node of all 48 arrays of both trees, both
+    roots, the chunk list and the element ids equal the oracle's, and the element count equals a
+    device brute-force count of |a-b| > eps over all 2.6e9 element pairs."""
     pair = synth.c5_pair(device="cuda")
-    C, eps = pair.chunk_bytes, pair.eps
-    L = sum(-(-t.numel() * 4 // C) for t in pair.a)
-    n_el = sum(t.numel() for t in pair.a)
-    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
-    idx = torch.empty(n_el, dtype=torch.int64, device="cuda")
-    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
-    TA, TB = ck.compare_pair_async(pair.a, pair.b, C, eps, chunks, idx, counts)
-    TA.wait(); TB.wait()
-    nc, nd = counts.tolist()
-    got_c, got_i = np_of(chunks[:nc]), np_of(idx[:nd])
-    # brute-force property over all 2.5e9 elements (binary64 |a-b| > eps on the device)
+    TA, TB, chunks, idx, counts = fused_compare(pair)
     brute = 0
     for x, y in zip(pair.a, pair.b):
-        brute += int((x.double() - y.double()).abs().gt(eps).sum().item())
+        brute += int((x.double() - y.double()).abs().gt(pair.eps).sum().item())
+    nc, nd = full_checkpoint_parity(pair, TA, TB, chunks, idx, counts, brute=False)
     assert nd == brute
-    # oracle over sampled arrays (global numbering)
-    per = C // 4
-    chunk_base = np.cumsum([0] + [-(-t.numel() * 4 // C) for t in pair.a])
+    # false positives by construction: flagged chunks with no verified difference
+    per = pair.chunk_bytes // 4
+    got_c = np_of(chunks[:nc])
+    got_i = np_of(idx[:nd])
     elem_base = np.cumsum([0] + [t.numel() for t in pair.a])
-    for k in (0, 7, 23, len(pair.a) - 1):
-        an, bn = np_of(pair.a[k]), np_of(pair.b[k])
-        la = oracle.leaves(an, C, eps, threads=os.cpu_count() or 8)
-        lb = oracle.leaves(bn, C, eps, threads=os.cpu_count() or 8)
-        ref_c = np.nonzero(np.any(la != lb, axis=1))[0]
-        ref_i = oracle.verify(an, bn, C, ref_c, eps)
-        sel_c = got_c[(got_c >= chunk_base[k]) & (got_c < chunk_base[k + 1])] - chunk_base[k]
-        sel_i = got_i[(got_i >= elem_base[k]) & (got_i < elem_base[k + 1])] - elem_base[k]
-        assert np.array_equal(sel_c, ref_c), k
-        assert np.array_equal(sel_i, ref_i), k
-        assert np.array_equal(gpu_tree_nodes(TA, k)[: la.shape[0]], la), k
+    chunk_base = np.cumsum([0] + [-(-t.numel() * 4 // pair.chunk_bytes) for t in pair.a])
+    arr = np.searchsorted(elem_base, got_i, side="right") - 1
+    hit_chunks = np.unique(chunk_base[arr] + (got_i - elem_base[arr]) // per)
+    assert np.setdiff1d(got_c, hit_chunks).size > 0
 
 
 @pytest.mark.slow
@@ -1014,3 +1046,43 @@ def test_large_chunk_latency_variant_matches_oracle(dt, chunk, n, eps):
     nc, nd = counts.tolist()
     assert np.array_equal(np_of(chunks[:nc]), ref_c) and np.array_equal(np_of(idx[:nd]), ref_i)
     assert np.array_equal(gpu_tree_nodes(ck.tree_build(a, chunk, eps)), na)
+
+
+# ------------------------------------------ verify work-buffer reuse (emit) --
+
+@pytest.mark.parametrize("dt,chunk", [(torch.float32, 65536), (torch.float64, 16384)])
+def test_flagged_ragged_last_chunk_after_dense_verify(dt, chunk):
+    """A flagged short last chunk (fewer than chunk/elem_size elements, chunk > 1024 elements)
+    must emit only its own ids although the verify work buffer still holds the all-ones masks
+    of a previous, fully differing compare on the same stream."""
+    n = 70_001
+    a = _data(n, dt, 17)
+    L = -(-n * a.element_size() // chunk)
+    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+    idx = torch.empty(n, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async([a], [a + 1.0], chunk, 1e-6, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    assert counts.tolist() == [L, n]
+    b = a.clone()
+    b[-1] += 1.0
+    TA, TB = ck.compare_pair_async([a], [b], chunk, 1e-6, chunks, idx, counts)
+    TA.wait(); TB.wait()
+    assert counts.tolist() == [1, 1]
+    assert chunks[0].item() == L - 1 and idx[0].item() == n - 1
+
+
+def test_async_wrappers_validate_output_buffers():
+    a = _data(1 << 12, torch.float32, 3)
+    good = torch.empty(64, dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    with pytest.raises(TypeError):
+        ck.compare_pair_async([a], [a], 4096, 1e-6, good.int(), good, counts)
+    with pytest.raises(ValueError):
+        ck.compare_pair_async([a], [a], 4096, 1e-6, good, good, counts[:1])
+    with pytest.raises(ValueError):
+        ck.compare_pair_async([a], [a], 4096, 1e-6, good[::2], good, counts)
+    with pytest.raises(ValueError):
+        ck.compare_pair_async([a], [a], 4096, 1e-6, good.cpu(), good, counts)
+    with pytest.raises(ValueError):
+        ck.verify_async([a], [a], good, counts[:0], 4096, 1e-6, good, counts[1:])
