@@ -575,7 +575,7 @@ def main():
     ap.add_argument("--snapshot", type=int, default=9, help="c4: snapshot index 0..9")
     ap.add_argument("--snapshots", default="one", choices=["one", "all"],
                     help="c4: 'all' = BASELINE configs[3] as written, the 10-snapshot sequence")
-    ap.add_argument("--n", type=int, default=0,
+    ap.add_argument("--elems", type=int, default=0,
                     help="elements per array (0 = the config's full size; smaller sizes are for "
                          "tests and are marked REDUCED in the workload)")
     ap.add_argument("--chunk", type=int, default=4096, help="chunk bytes (configs[2] sweeps 512..65536)")
@@ -592,9 +592,9 @@ def main():
     SNAPSHOT = args.snapshot
     N_PARTICLES = CONFIGS[CFG]["n"]
     WORKLOAD = CONFIGS[CFG]["workload"]
-    if args.n:
-        N_PARTICLES = args.n
-        WORKLOAD = f"REDUCED ({args.n} elements per array, not a bench line): " + WORKLOAD
+    if args.elems:
+        N_PARTICLES = args.elems
+        WORKLOAD = f"REDUCED ({args.elems} elements per array, not a bench line): " + WORKLOAD
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         return spawn_ranks(args.gpus)
     if args.impl == "reference":

@@ -82,7 +82,7 @@ def test_bench_runs_n_nccl_ranks(world):
     if torch.cuda.device_count() < world:
         pytest.skip(f"needs {world} GPUs")
     args = [os.path.join(ROOT, "bench.py"), "--gpus", str(world), "--steps", "3", "--warmup", "3",
-            "--no-e2e", "--no-cpu", "--n", str(1 << 20), "--collectives"]
+            "--no-e2e", "--no-cpu", "--elems", str(1 << 20), "--collectives"]
     r = _torchrun(world, args)
     assert r.returncode == 0, r.stderr[-4000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
@@ -102,7 +102,7 @@ def test_bench_spawns_ranks_itself_when_not_launched():
     env = {k: v for k, v in os.environ.items()
            if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "MASTER_ADDR", "MASTER_PORT")}
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "3",
-                        "--warmup", "3", "--no-e2e", "--no-cpu", "--n", str(1 << 20)],
+                        "--warmup", "3", "--no-e2e", "--no-cpu", "--elems", str(1 << 20)],
                        cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-4000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
