@@ -513,8 +513,21 @@ def _pair_cases():
         ("c2_small", lambda: synth.c2_pair(n_particles=(1 << 18) + 77, seed=23, device="cuda")),
         ("c5_small", lambda: synth.c5_pair(n_ranks=2, n_particles=1 << 16, seed=24, device="cuda")),
         ("c3_small", lambda: synth.c3_pair(n=(1 << 20) + 5, seed=25, device="cuda", n_clusters=16,
-                                           mean_len=512)),
+                                           mean_len=512, n_isolated=500)),
+        ("many_ragged", _many_ragged),
     ]
+
+
+def _many_ragged():
+    """20 arrays (device-resident array tables) of ragged sizes: 1 and 3 elements, one chunk,
+    33 chunks, 4097 chunks (levels past one 7-level group), a partial 16-byte block."""
+    sizes = [1, 3, 1024, 33 * 1024 + 1, 4097 * 1024, 5, 77_777, 1 << 16, 2, 129 * 1024 + 3,
+             6, 1025, 99, 4 * 1024, 128 * 1024, 128 * 1024 + 1, 7, 16_383, 300_001, 11]
+    a = [synth.uniform(700 + i, n, "cuda") * 2.0 - 1.0 for i, n in enumerate(sizes)]
+    b = [t.clone() for t in a]
+    for i, t in enumerate(b):
+        t[(3 * i) % t.numel()::max(1, 997 + 31 * i)] += 1e-3 * (1 + (i % 3))
+    return synth.Pair("many_ragged", a, b, 4096, 1e-5)
 
 
 @pytest.mark.parametrize("name,make", _pair_cases(), ids=[c[0] for c in _pair_cases()])
@@ -588,10 +601,11 @@ def test_compare_pair_identical_and_truncated():
         ck.compare_pair_async(a, [b[0]], 4096, 1e-6, chunks, idx, counts)
 
 
-# K1 tile compaction (128 pair-tasks = 4096 chunks per tile) + tile_gather_kernel:
-# ragged arrays (pair-tasks of < 32 chunks), several tiles with a ragged last
-# one, every chunk flagged, no chunk flagged, and a chunk-list cap that cuts
-# through a tile -- all against the plain leaf comparison and brute force.
+# K1 tile compaction (128 pair-tasks = 4096 chunks per tile) + in-kernel marking +
+# pair_emit_kernel: ragged arrays (pair-tasks of < 32 chunks), several tiles with
+# a ragged last one, every chunk flagged (every marking job queued at once), no
+# chunk flagged, and a chunk-list cap that cuts through a tile -- all against the
+# plain leaf comparison and brute force.
 @pytest.mark.parametrize("mode", ["all", "none", "sparse", "cap"])
 def test_compare_pair_tile_compaction(mode):
     sizes = [300 * 1024 + 5, 7 * 1024, 4096 * 1024 + 3, 1]       # f32 elements; C = 4 KiB
@@ -640,18 +654,41 @@ def test_compare_pair_tile_compaction(mode):
     assert np.array_equal(np_of(idx[:nd]), ref_idx)
 
 
-def test_compare_pair_tile_gather_path():
-    """The gather kernel (used past 4096 tiles) in a fresh process with CKPT_TILE_GATHER=1."""
-    import subprocess
-    import sys
-    code = (
-        "import sys; sys.path.insert(0, %r); import test_gpu_parity as t; "
-        "[t.test_compare_pair_tile_compaction(m) for m in ('all', 'none', 'sparse', 'cap')]; print('ok')"
-        % os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, CKPT_TILE_GATHER="1")
-    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
-                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
-    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stdout[-2000:] + r.stderr[-2000:]
+@pytest.mark.parametrize("dt,chunk", [(torch.float32, 2 << 20), (torch.float64, 4 << 20)])
+def test_compare_pair_fallback_path_large_chunks(dt, chunk):
+    """Chunks above 1 MiB take the fallback of the fused call (flags-only leaf kernel, levels
+    kernel, flag compaction, verify kernels): same results as the oracle."""
+    sizes = [3 * chunk // 8 + 5, chunk // 16, 2 * chunk // 4 + 1]
+    a = [_data(n, dt, 300 + i) for i, n in enumerate(sizes)]
+    b = [t.clone() for t in a]
+    b[0][::100_003] += 1e-3
+    b[2][-1] += 1.0
+    pair = synth.Pair("fallback", a, b, chunk, 1e-6)
+    TA, TB, chunks, idx, counts = fused_compare(pair)
+    full_checkpoint_parity(pair, TA, TB, chunks, idx, counts, brute=True)
+
+
+def test_compare_pair_repeated_and_alternating_shapes():
+    """The in-kernel counters, job queue and tile state return to zero after every launch: many
+    compares on one stream, alternating between shapes (per-shape table cache), all exact."""
+    p1 = synth.c1_pair(n=(1 << 19) + 3, seed=61, device="cuda")
+    p2 = synth.c5_pair(n_ranks=1, n_particles=(1 << 15), seed=62, device="cuda")
+    ref = {}
+    for name, p in (("p1", p1), ("p2", p2)):
+        an = [np_of(t) for t in p.a]
+        bn = [np_of(t) for t in p.b]
+        A = oracle.build_checkpoint(an, p.chunk_bytes, p.eps, threads=8)
+        B = oracle.build_checkpoint(bn, p.chunk_bytes, p.eps, threads=8)
+        rc = oracle.diff_checkpoint(A, B)
+        ref[name] = (rc, oracle.verify_checkpoint(an, bn, p.chunk_bytes, rc, p.eps, A), A.root, B.root)
+    for it in range(6):
+        name, p = (("p1", p1), ("p2", p2))[it % 2]
+        TA, TB, chunks, idx, counts = fused_compare(p)
+        nc, nd = counts.tolist()
+        rc, ri, ra, rb = ref[name]
+        assert np.array_equal(np_of(chunks[:nc]), rc), (it, name)
+        assert np.array_equal(np_of(idx[:nd]), ri), (it, name)
+        assert TA.root() == ra and TB.root() == rb, (it, name)
 
 
 # ------------------------------------------- hash block size variant (R23) --
