@@ -1273,7 +1273,7 @@ static ckpt_status get_full_scratch(int dev, cudaStream_t s, uint64_t L, uint64_
     std::lock_guard<std::mutex> lk(g_scr_mu);
     Scratch &sc = g_scr[std::make_pair(dev, s)];
     const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
-    // zero-once block: [qs 4 x u64][acc 2 x u64] | gctr [n_ctr] | tctr [n_tiles]
+    // zero-once block: [qs 5 x u64 @0][acc 2 x u64 @64] | gctr [n_ctr] | tctr [n_tiles]
     if (sc.fz_ctr < n_ctr || sc.fz_tiles < n_tiles) {
         if (sc.fz) CK_CUDA(cudaFreeAsync(sc.fz, s));
         sc.fz_ctr = std::max<size_t>(n_ctr, 2 * sc.fz_ctr);
@@ -1306,7 +1306,7 @@ static ckpt_status get_full_scratch(int dev, cudaStream_t s, uint64_t L, uint64_
         CK_CUDA(cudaMallocAsync((void **)&sc.fbuf, sc.fbuf_cap, s));
     }
     pp->qs = (unsigned long long *)sc.fz;
-    pp->acc = (unsigned long long *)(sc.fz + 32);
+    pp->acc = (unsigned long long *)(sc.fz + 64);
     pp->gctr = (unsigned int *)(sc.fz + 256);
     pp->tctr = (unsigned int *)(sc.fz + 256 + align256(sc.fz_ctr * 4));
     pp->q = (unsigned long long *)sc.fjobs;

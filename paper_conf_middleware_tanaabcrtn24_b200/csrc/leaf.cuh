@@ -280,9 +280,11 @@ __device__ __noinline__ void pair_finish(const LeafParams &P, bool differ, int a
         slot = __shfl_sync(0xffffffffu, slot, 0);
         if (differ)
             pr.q[slot + __popc(m & ((1u << lane) - 1u))] = (((unsigned long long)aa << 44) | (c0 + lane)) + 1ull;
+        __syncwarp();
+        if (lane == 0) atomicAdd(pr.qs + 4, (unsigned long long)nm);   // available to claimers
     }
     __syncwarp();
-    if (lane == 0) atom_add_rel64(pr.qs + 2, 1ull);      // compared (after the tail was raised)
+    if (lane == 0) atom_add_rel64(pr.qs + 2, 1ull);      // compared (after the jobs were counted)
     tile_arrive(pr, pt / kTileTasks, (unsigned int)(kTileUnits - nm), lane);
     climb(pr, aa, c0 / kRows, true, sm, lane);
 }
@@ -335,30 +337,20 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
     uint4 *const wsm = reinterpret_cast<uint4 *>(smem + warp * kWarpSmem);   // the ring, as nodes
     for (;;) {
         // draw the next task; in full pair mode also look at the marking queue (same round trip)
-        unsigned long long t = 0, qh = 0, qt = 0;
+        unsigned long long t = 0;
+        long long avail = 0;
         if (lane == 0) {
             t = atomicAdd(P.ticket, 1ull);
             if (t == n_tasks + n_warps_grid - 1) *P.ticket = 0ull;   // the last draw of the launch
-            if (full) {
-                qh = ld_relaxed64(P.pr.qs);
-                qt = ld_relaxed64(P.pr.qs + 1);
-            }
+            if (full) avail = *reinterpret_cast<volatile long long *>(P.pr.qs + 4);
         }
         const uint64_t task = __shfl_sync(0xffffffffu, t, 0);
-        if (full) {
+        if (full && __shfl_sync(0xffffffffu, avail, 0) > 0) {
             // marking jobs first: they stay few and spread over every warp
-            qh = __shfl_sync(0xffffffffu, qh, 0);
-            qt = __shfl_sync(0xffffffffu, qt, 0);
-            while (qh < qt) {
-                const unsigned long long e = claim_job(P.pr, lane, qh, qt);
+            for (;;) {
+                const unsigned long long e = claim_job(P.pr, lane);
                 if (!e) break;
                 mark_job<DT>(P, arrays, e, lane);
-                if (lane == 0) {
-                    qh = ld_relaxed64(P.pr.qs);
-                    qt = ld_relaxed64(P.pr.qs + 1);
-                }
-                qh = __shfl_sync(0xffffffffu, qh, 0);
-                qt = __shfl_sync(0xffffffffu, qt, 0);
             }
         }
         if (task >= n_tasks) break;
@@ -537,33 +529,29 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
         // empty (the last compares can still queue jobs), then count out; the last warp out
         // empties the queue counters for the next launch
         for (;;) {
-            unsigned long long pd = 0, qh = 0, qt = 0;
+            const unsigned long long e = claim_job(P.pr, lane);
+            if (e) {
+                mark_job<DT>(P, arrays, e, lane);
+                continue;
+            }
+            unsigned long long pd = 0;
+            long long avail = 0;
             if (lane == 0) {
                 pd = ld_acquire64(P.pr.qs + 2);
-                qh = ld_relaxed64(P.pr.qs);
-                qt = ld_relaxed64(P.pr.qs + 1);
+                avail = *reinterpret_cast<volatile long long *>(P.pr.qs + 4);
             }
             pd = __shfl_sync(0xffffffffu, pd, 0);
-            qh = __shfl_sync(0xffffffffu, qh, 0);
-            qt = __shfl_sync(0xffffffffu, qt, 0);
-            if (qh < qt) {
-                const unsigned long long e = claim_job(P.pr, lane, qh, qt);
-                if (e) {
-                    mark_job<DT>(P, arrays, e, lane);
-                    continue;
-                }
-            }
-            if (pd == P.pr.n_pair && qh >= qt) break;
-            __nanosleep(256);
+            avail = __shfl_sync(0xffffffffu, avail, 0);
+            // every pair-task compared (so every job counted) and none left to take; a job whose
+            // take failed transiently is taken by the warp that gave it back
+            if (pd == P.pr.n_pair && avail <= 0) break;
+            __nanosleep(1000);
         }
         __syncwarp();
         if (lane == 0) {
             const unsigned long long out = atomicAdd(P.pr.qs + 3, 1ull);
             if (out == n_warps_grid - 1) {
-                P.pr.qs[0] = 0ull;
-                P.pr.qs[1] = 0ull;
-                P.pr.qs[2] = 0ull;
-                P.pr.qs[3] = 0ull;
+                for (int k = 0; k < 5; ++k) P.pr.qs[k] = 0ull;
             }
         }
     }

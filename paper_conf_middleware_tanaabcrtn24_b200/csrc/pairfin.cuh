@@ -68,7 +68,7 @@ struct PairParams {
     uint4 *tree[2];               // node storage of run A's / run B's tree
     unsigned int *gctr;           // group counters (0 between launches)
     unsigned long long *q;        // [L] marking jobs: ((array << 44) | local chunk) + 1; 0 = empty
-    unsigned long long *qs;       // [4] head, tail, pair-tasks compared, warps exited
+    unsigned long long *qs;       // [5] head, tail, pair-tasks compared, warps exited, jobs available
     unsigned long long *acc;      // [2] flagged chunks, differing elements (the emit kernel resets)
     uint32_t *cnt;                // [L] hits per flagged chunk (global chunk id)
     uint32_t *mask;               // [L * groups * 32] hit bits per flagged chunk (global chunk id)
@@ -246,21 +246,26 @@ __device__ __forceinline__ void tile_arrive(const PairParams &pr, uint64_t tile,
     }
 }
 
-// Claim one marking job (lane 0 CAS on the head); returns the entry (0: none available).
-__device__ __forceinline__ unsigned long long claim_job(const PairParams &pr, int lane,
-                                                        unsigned long long h, unsigned long long t) {
+// Claim one marking job.  Pushers raise the tail, write their entries, then add to the
+// "available" count; a claimer takes one unit of it with a fetch-and-add (no retry loop on
+// a shared word: every claim is one round trip however many warps contend) and, on
+// success, the next head slot, which is then guaranteed to be (or become) a written entry.
+// A failed take (the count was not positive) is given back.  Returns the entry or 0.
+__device__ __forceinline__ unsigned long long claim_job(const PairParams &pr, int lane) {
     unsigned long long e = 0;
     if (lane == 0) {
-        while (h < t) {
-            const unsigned long long o = atomicCAS(pr.qs, h, h + 1);
-            if (o == h) {
-                // the pusher raised the tail before writing its entries: wait for this one
+        long long *avail = reinterpret_cast<long long *>(pr.qs + 4);
+        if (*reinterpret_cast<volatile long long *>(avail) > 0) {
+            const long long before = (long long)atomicAdd(reinterpret_cast<unsigned long long *>(avail),
+                                                          (unsigned long long)-1ll);
+            if (before > 0) {
+                const unsigned long long h = atomicAdd(pr.qs, 1ull);
                 volatile unsigned long long *slot = pr.q + h;
                 do { e = *slot; } while (e == 0ull);
                 *slot = 0ull;                    // empty again for the next launch
-                break;
+            } else {
+                atomicAdd(reinterpret_cast<unsigned long long *>(avail), 1ull);
             }
-            h = o;
         }
     }
     return __shfl_sync(0xffffffffu, e, 0);

@@ -1,5 +1,7 @@
 #!/usr/bin/env python
-"""Fused diff+verify vs separate diff / verify kernels, standalone (trees prebuilt)."""
+"""Leaf-kernel time of the fused pair call (ckpt_compare_pair_async) vs the number of flagged
+chunks: identical runs, the c2 recipe, and k uniformly spread flagged chunks (one element
+changed by 1.0 in each), on the c2 shape (2^26 x 6 f32, 4 KiB chunks)."""
 import os
 import sys
 
@@ -9,37 +11,39 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_middleware_tanaabcrtn24_b200 as ck  # noqa: E402
 import synth  # noqa: E402
 
+n_part = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 26
+pair = synth.c2_pair(n_particles=n_part, seed=5, device="cuda")
+A = pair.a
+L = sum(t.numel() * 4 // 4096 for t in A)
+n = sum(t.numel() for t in A)
+chunks = torch.empty(L, dtype=torch.int64, device="cuda")
+idx = torch.empty(n, dtype=torch.int64, device="cuda")
+cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
 
-def timed(fn, kinds, reps=20):
+
+def run(B, label, reps=10):
     for _ in range(3):
-        fn()
+        ck.compare_pair_async(A, B, 4096, 1e-6, chunks, idx, cnt)
     torch.cuda.synchronize()
     ck.profile_reset()
     ck.profile_enable(True)
     for _ in range(reps):
-        fn()
+        ck.compare_pair_async(A, B, 4096, 1e-6, chunks, idx, cnt)
     torch.cuda.synchronize()
     ck.profile_enable(False)
-    out = []
-    for k in kinds:
-        ms, n = ck.profile_read(k)
-        out.append(ms / max(n, 1) * 1e3)
-    return out
+    lm, ln = ck.profile_read("leaf")
+    vm, vn = ck.profile_read("verify")
+    print(f"{label:>28s}: flagged {int(cnt[0].item()):7d} diffs {int(cnt[1].item()):8d}  "
+          f"leaf {lm / max(ln, 1) * 1e3:8.1f} us  emit {vm / max(vn, 1) * 1e3:6.1f} us", flush=True)
 
 
-for n_part in (1 << 20, 1 << 24, 1 << 26):
-    pair = synth.c2_pair(n_particles=n_part, seed=5, device="cuda")
-    TA, TB = ck.tree_build_batch([pair.a, pair.b], 4096, 1e-6)
-    TA.wait()
-    TB.wait()
-    L = TA.n_leaves
-    n = sum(t.numel() for t in pair.a)
-    chunks = torch.empty(L, dtype=torch.int64, device="cuda")
-    idx = torch.empty(n, dtype=torch.int64, device="cuda")
-    cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
-    f = timed(lambda: ck.diff_verify_async(TA, TB, pair.a, pair.b, chunks, idx, cnt), ["verify"])
-    s = timed(lambda: (ck.tree_diff_async(TA, TB, chunks, cnt[0:1]),
-                       ck.verify_async(pair.a, pair.b, chunks, cnt[0:1], 4096, 1e-6, idx, cnt[1:2])),
-              ["diff", "verify"])
-    print(f"L={L:8d} flagged={int(cnt[0].item()):6d}  fused {f[0]:7.1f} us   separate diff {s[0]:6.1f} + verify {s[1]:6.1f} us",
-          flush=True)
+run([t.clone() for t in A], "identical")
+run(pair.b, "c2 recipe")
+per = 1024
+for k in (64, 1024, 16384):
+    B = [t.clone() for t in A]
+    Lk = A[0].numel() // per
+    for f, t in enumerate(B):
+        ch = torch.arange(f, Lk, max(1, Lk * 6 // k), device="cuda")[: k // 6 + 1]
+        t[ch * per + 7] += 1.0
+    run(B, f"{k} spread chunks")
