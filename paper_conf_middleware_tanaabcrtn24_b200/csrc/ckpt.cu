@@ -26,6 +26,7 @@
 #include "hash.cuh"
 #include "leaf.cuh"
 #include "levels.cuh"
+#include "finish.cuh"
 
 using namespace ckpt;
 
@@ -244,7 +245,6 @@ struct ckpt_tree {
     uint64_t top_off = 0, top_nodes = 0;
     uint4 *nodes = nullptr;                // device
     uint8_t *meta = nullptr;               // device metadata blob
-    bool meta_shared = false;              // meta is a per-shape cache entry (not freed with the tree)
     // device views into meta
     const uint64_t *d_off = nullptr, *d_cnt = nullptr, *d_level_base = nullptr,
                    *d_level_total = nullptr, *d_chunk_base = nullptr;
@@ -424,6 +424,47 @@ static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms, 
 static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_t **states,
                                unsigned long long **ticket, uint32_t *epoch);
 
+// The launch record of up to kMaxLevelTrees trees' level groups (tree metadata inline in
+// the parameters when it fits, else staged to each tree's device blob).
+static ckpt_status fill_level_batch(ckpt_tree *const *trees, int n, cudaStream_t s,
+                                    unsigned long long *tickets, LevelBatch &b) {
+    std::memset(&b, 0, offsetof(LevelBatch, blob));
+    b.n = n;
+    unsigned ctas = 0;
+    uint32_t words = 0;
+    for (int i = 0; i < b.n; ++i) {
+        ckpt_tree *t = trees[i];
+        LevelParams &p = b.t[i];
+        p.nodes = t->nodes;
+        p.meta = t->meta;
+        p.meta_words = (uint32_t)t->meta_host.size();
+        if (words + p.meta_words <= (uint32_t)kLevelInlineWords) {
+            std::memcpy(b.blob + words, t->meta_host.data(), (size_t)p.meta_words * 8);
+            p.inl = (int)words;
+            words += p.meta_words;
+        } else {
+            p.inl = -1;
+            CK_TRY(g_ring.copy(t->meta, t->meta_host.data(), t->meta_host.size() * 8, s));
+        }
+        p.o_off = t->o_off;
+        p.o_cnt = t->o_cnt;
+        p.o_lb = t->o_lb;
+        p.o_lt = t->o_lt;
+        p.o_h = t->o_h;
+        p.o_g = t->o_g;
+        p.top_off = t->top_off;
+        p.ticket = reinterpret_cast<unsigned int *>(tickets + 1 + i);   // slot 0: compactions
+        p.n_arrays = (int)t->n_arrays;
+        p.n_levels = (int)t->n_levels;
+        p.ls = 0;
+        p.n_groups = (unsigned)t->n_groups;
+        b.cta_begin[i] = ctas;
+        ctas += (unsigned)t->n_groups;
+    }
+    b.cta_begin[b.n] = ctas;
+    return CKPT_OK;
+}
+
 static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s) {
     static std::atomic<int> attr_done{0};
     if (!attr_done.load()) {
@@ -440,50 +481,17 @@ static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s)
     static std::mutex b_mu;
     std::lock_guard<std::mutex> lk(b_mu);
     for (int k0 = 0; k0 < n; k0 += kMaxLevelTrees) {
-        std::memset(&b, 0, offsetof(LevelBatch, blob));
-        b.n = std::min(kMaxLevelTrees, n - k0);
-        unsigned ctas = 0;
-        uint32_t words = 0;
-        for (int i = 0; i < b.n; ++i) {
-            ckpt_tree *t = trees[k0 + i];
-            LevelParams &p = b.t[i];
-            p.nodes = t->nodes;
-            p.meta = t->meta;
-            p.meta_words = (uint32_t)t->meta_host.size();
-            if (words + p.meta_words <= (uint32_t)kLevelInlineWords) {
-                std::memcpy(b.blob + words, t->meta_host.data(), (size_t)p.meta_words * 8);
-                p.inl = (int)words;
-                words += p.meta_words;
-            } else {
-                p.inl = -1;
-                CK_TRY(g_ring.copy(t->meta, t->meta_host.data(), t->meta_host.size() * 8, s));
-            }
-            p.o_off = t->o_off;
-            p.o_cnt = t->o_cnt;
-            p.o_lb = t->o_lb;
-            p.o_lt = t->o_lt;
-            p.o_h = t->o_h;
-            p.o_g = t->o_g;
-            p.top_off = t->top_off;
-            p.ticket = reinterpret_cast<unsigned int *>(tickets + 1 + i);   // slot 0: compactions
-            p.n_arrays = (int)t->n_arrays;
-            p.n_levels = (int)t->n_levels;
-            p.ls = 0;
-            p.n_groups = (unsigned)t->n_groups;
-            b.cta_begin[i] = ctas;
-            ctas += (unsigned)t->n_groups;
-        }
-        b.cta_begin[b.n] = ctas;
+        CK_TRY(fill_level_batch(trees + k0, std::min(kMaxLevelTrees, n - k0), s, tickets, b));
         ProfScope prof(1, s);
-        CK_CUDA(launch_k(levels_kernel, dim3(ctas), dim3(kLevelThreads), kLevelSmem, s, b));
+        CK_CUDA(launch_k(levels_kernel, dim3(b.cta_begin[b.n]), dim3(kLevelThreads), kLevelSmem, s, b));
         CK_LAUNCH();
     }
     return CKPT_OK;
 }
 
-// The device metadata blob of a laid-out tree, on the host (t->meta_host):
-// [off][cnt][level_base][level_total][chunk_base][height][gbegin]
-static void meta_layout(ckpt_tree *t) {
+// Allocate a laid-out tree's node storage and device metadata blob:
+// [off][cnt][level_base][level_total][chunk_base][height][gbegin][ticket]
+static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
     const uint32_t na = t->n_arrays;
     std::vector<uint64_t> gbegin(na);
     uint64_t groups = 0;
@@ -501,7 +509,8 @@ static void meta_layout(ckpt_tree *t) {
     t->o_cb = (uint32_t)o;  o = al8(o + (size_t)na * 8);
     t->o_h = (uint32_t)o;   o = al8(o + (size_t)na * 4);
     t->o_g = (uint32_t)o;   o = al8(o + (size_t)na * 8);
-    t->meta_host.assign(o / 8, 0);
+    const size_t total = o;
+    t->meta_host.assign(total / 8, 0);
     uint8_t *blob = reinterpret_cast<uint8_t *>(t->meta_host.data());
     std::memcpy(blob + t->o_off, t->off.data(), t->off.size() * 8);
     std::memcpy(blob + t->o_cnt, t->cnt.data(), t->cnt.size() * 8);
@@ -510,20 +519,8 @@ static void meta_layout(ckpt_tree *t) {
     std::memcpy(blob + t->o_cb, t->chunk_base.data(), (size_t)na * 8);
     std::memcpy(blob + t->o_h, t->height.data(), (size_t)na * 4);
     std::memcpy(blob + t->o_g, gbegin.data(), (size_t)na * 8);
-}
-
-// Allocate a laid-out tree's node storage and device metadata blob.
-// shared_meta != null: the blob already holds this layout on the device (a per-shape cache
-// entry of the fused pair path) and is used instead of a per-tree copy.
-static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s, uint8_t *shared_meta = nullptr) {
-    meta_layout(t);
     CK_CUDA(cudaMallocAsync((void **)&t->nodes, (t->array_nodes + t->top_nodes) * 16, s));
-    if (shared_meta) {
-        t->meta = shared_meta;
-        t->meta_shared = true;
-    } else {
-        CK_CUDA(cudaMallocAsync((void **)&t->meta, t->meta_host.size() * 8, s));
-    }
+    CK_CUDA(cudaMallocAsync((void **)&t->meta, total, s));
     // the blob reaches `meta` through K2 (inline parameters) or a staging copy there
     t->d_off = (const uint64_t *)(t->meta + t->o_off);
     t->d_cnt = (const uint64_t *)(t->meta + t->o_cnt);
@@ -582,13 +579,8 @@ struct Scratch {
     size_t pair_cap = 0;
     uint8_t *pair_flags = nullptr;      // fused pair mode: one flag byte per chunk
     size_t flags_cap = 0;
-    // fused pair path, full mode (pairfin.cuh)
-    uint8_t *fz = nullptr;              // zero-once block: queue state + totals, group + tile counters
-    size_t fz_ctr = 0, fz_tiles = 0;    // counters it holds
-    uint8_t *fjobs = nullptr;           // marking-job queue entries (zero once, self-clearing)
-    size_t fjobs_cap = 0;
-    uint8_t *fbuf = nullptr;            // per-chunk / per-pair-task / per-tile buffers (no init)
-    size_t fbuf_cap = 0;
+    uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
+    size_t tile_pairs = 0;              // pair-tasks the buffers hold
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -607,6 +599,49 @@ static ckpt_status get_pair_flags(int dev, cudaStream_t s, size_t n, uint8_t **f
 }
 
 constexpr int kLeafTicketSlot = 16;   // 8-byte slot of the per-stream ticket block used by K1
+
+// CKPT_TILE_GATHER=1: always place the fused path's chunk list with tile_gather_kernel
+// (A/B and tests of that path; by default K4a reads the tiles itself).
+static bool tile_gather_forced() {
+    static const bool on = [] {
+        const char *e = std::getenv("CKPT_TILE_GATHER");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
+// K1 tile-compaction buffers for n_pair pair-tasks (leaf.cuh PairParams):
+// [tctr: n_tiles u32, zeroed once; self-resetting] [tagg: n_tiles u32]
+// [tmask: n_pair u32] [tbase: n_pair u64] [tids: n_tiles * kTileTasks * 32 u64]
+static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, PairParams *pp) {
+    std::lock_guard<std::mutex> lk(g_scr_mu);
+    Scratch &sc = g_scr[std::make_pair(dev, s)];
+    n_pair = std::max<uint64_t>(n_pair, 1);
+    auto layout_of = [](uint64_t np, size_t o[5]) {
+        const uint64_t nt = (np + kTileTasks - 1) / kTileTasks;
+        o[0] = 0;
+        o[1] = align256(nt * 4);
+        o[2] = o[1] + align256(nt * 4);
+        o[3] = o[2] + align256(np * 4);
+        o[4] = o[3] + align256(np * 8);
+        return o[4] + nt * kTileTasks * 32 * 8;
+    };
+    size_t o[5];
+    if (sc.tile_pairs < n_pair) {
+        if (sc.tile) CK_CUDA(cudaFreeAsync(sc.tile, s));
+        sc.tile_pairs = std::max<uint64_t>(n_pair, 2 * sc.tile_pairs);
+        const size_t bytes = layout_of(sc.tile_pairs, o);
+        CK_CUDA(cudaMallocAsync((void **)&sc.tile, bytes, s));
+        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters
+    }
+    layout_of(sc.tile_pairs, o);
+    pp->tctr = (unsigned int *)(sc.tile + o[0]);
+    pp->tagg = (uint32_t *)(sc.tile + o[1]);
+    pp->tmask = (uint32_t *)(sc.tile + o[2]);
+    pp->tbase = (uint64_t *)(sc.tile + o[3]);
+    pp->tids = (uint64_t *)(sc.tile + o[4]);
+    return CKPT_OK;
+}
 
 // Zero-initialised pair-task counters (they return to 0 after every launch).
 static ckpt_status get_pair_ctr(int dev, cudaStream_t s, size_t n, unsigned int **ctr) {
@@ -629,7 +664,7 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
                                     const uint32_t *arrays_per_tree, uint32_t n_trees,
                                     ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
                                     uint32_t hash_block, void *stream, ckpt_tree **out,
-                                    const PairParams *pair) {
+                                    const PairParams *pair, bool defer_levels = false) {
     if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
     for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
     if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
@@ -701,7 +736,7 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
     if (st == CKPT_OK)
         st = launch_leaves(table, task, dtype, eps, chunk_bytes, hash_block, s, di.sms,
                            pair ? &pp : nullptr, ticket);
-    if (st == CKPT_OK) {
+    if (st == CKPT_OK && !defer_levels) {
         // K2 on the side stream, after the leaves; each tree records its own event
         cudaStream_t ss = nullptr;
         cudaEvent_t leaves_done = nullptr;
@@ -830,7 +865,7 @@ extern "C" void ckpt_tree_free_on(ckpt_tree *t, void *stream) {
         cudaEventDestroy(t->levels_done);
     }
     if (t->nodes) cudaFreeAsync(t->nodes, s);
-    if (t->meta && !t->meta_shared) cudaFreeAsync(t->meta, s);
+    if (t->meta) cudaFreeAsync(t->meta, s);
     if (cur != t->device) cudaSetDevice(cur);
     delete t;
 }
@@ -896,7 +931,7 @@ static void release_scratch(int dev, cudaStream_t s) {
     auto it = g_scr.find(std::make_pair(dev, s));
     if (it == g_scr.end()) return;
     Scratch &sc = it->second;
-    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.fz, sc.fjobs, sc.fbuf};
+    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile};
     for (void *b : bufs)
         if (b) cudaFreeAsync(b, s);
     g_scr.erase(it);
@@ -1067,15 +1102,79 @@ extern "C" ckpt_status ckpt_tree_diff(const ckpt_tree *a, const ckpt_tree *b, ui
 // it may replace the output buffer and its capacity (exact-size outputs).
 using EmitHook = std::function<ckpt_status(uint64_t **idx, uint64_t *cap)>;
 
+// The verify parameters, table and scratch for `max_tiles` look-back tiles of `tile`
+// list positions (the finish kernel's tiles; the scan kernel's otherwise).
+static ckpt_status verify_setup(const void *const *a, const void *const *b, const uint64_t *n,
+                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
+                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
+                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
+                                uint64_t chunk_base0, uint64_t elem_base0, const PairParams *tiles,
+                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out);
+
 static ckpt_status verify_impl(const void *const *a, const void *const *b, const uint64_t *n,
                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
                                const EmitHook &before_emit = nullptr, uint64_t chunk_base0 = 0,
-                               uint64_t elem_base0 = 0) {
-    if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
+                               uint64_t elem_base0 = 0, const PairParams *tiles = nullptr) {
     if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
+    VerifyParams p;
+    uint8_t *tab = nullptr;
+    uint64_t max_chunks = 0;
+    CK_TRY(verify_setup(a, b, n, na, dtype, chunk_bytes, chunks, n_chunks_dev, n_chunks_host, chunks_cap,
+                        eps, idx, cap, n_diff_dev, s, chunk_base0, elem_base0, tiles, kVerifyScanTile, p,
+                        &tab, &max_chunks));
+    int dev;
+    DevInfo di;
+    CK_TRY(dev_info(&dev, &di));
+    static std::atomic<int> occ[5] = {{0}, {0}, {0}, {0}, {0}};
+    const int d = dtype == CKPT_F32 ? 0 : 1;
+    if (occ[d].load() == 0) {
+        int m = 0, e = 0, sc = 0;
+        if (d == 0) {
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<0>, kVerifyThreads, 0));
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<0>, kVerifyThreads, 0));
+        } else {
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<1>, kVerifyThreads, 0));
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<1>, kVerifyThreads, 0));
+        }
+        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sc, verify_scan_kernel, kVerifyThreads, 0));
+        occ[4].store(std::max(sc, 1));
+        occ[2 + d].store(std::max(e, 1));
+        occ[d].store(std::max(m, 1));
+    }
+    const uint64_t warp_ctas = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
+    const unsigned g_mark = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[d].load()));
+    const unsigned g_emit = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[2 + d].load()));
+    // co-resident grid (the look-back relies on it); tiles are strided statically
+    const uint64_t max_tiles = (max_chunks + kVerifyScanTile - 1) / kVerifyScanTile;
+    const unsigned g_scan = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * occ[4].load()));
+    {
+        ProfScope prof(3, s);
+        CK_CUDA(launch_k(d == 0 ? verify_mark_kernel<0> : verify_mark_kernel<1>, dim3(g_mark),
+                         dim3(kVerifyThreads), 0, s, p));
+        CK_LAUNCH();
+        CK_CUDA(launch_k(verify_scan_kernel, dim3(g_scan), dim3(kVerifyThreads), 0, s, p));
+        CK_LAUNCH();
+        if (before_emit) CK_TRY(before_emit(&p.out, &p.cap));
+        CK_CUDA(launch_k(d == 0 ? verify_emit_kernel<0> : verify_emit_kernel<1>, dim3(g_emit),
+                         dim3(kVerifyThreads), 0, s, p));
+    }
+    CK_LAUNCH();
+    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
+    return CKPT_OK;
+}
+
+static ckpt_status verify_setup(const void *const *a, const void *const *b, const uint64_t *n,
+                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
+                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
+                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
+                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
+                                uint64_t chunk_base0, uint64_t elem_base0, const PairParams *tiles,
+                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out) {
+    if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
     std::vector<VerifyArray> va(na);
@@ -1100,7 +1199,6 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
     const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c - chunk_base0);
-    VerifyParams p;
     std::memset(&p, 0, sizeof(p));
     uint8_t *tab = nullptr;
     if (na <= (uint32_t)kVerifyInline) {
@@ -1127,28 +1225,16 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     p.out = idx;
     p.cap = cap;
     p.count = n_diff_dev;
-    static std::atomic<int> occ[5] = {{0}, {0}, {0}, {0}, {0}};
-    const int d = dtype == CKPT_F32 ? 0 : 1;
-    if (occ[d].load() == 0) {
-        int m = 0, e = 0, sc = 0;
-        if (d == 0) {
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<0>, kVerifyThreads, 0));
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<0>, kVerifyThreads, 0));
-        } else {
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<1>, kVerifyThreads, 0));
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<1>, kVerifyThreads, 0));
-        }
-        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sc, verify_scan_kernel, kVerifyThreads, 0));
-        occ[4].store(std::max(sc, 1));
-        occ[2 + d].store(std::max(e, 1));
-        occ[d].store(std::max(m, 1));
+    if (tiles) {
+        // fused pair path: K4a reads K1's tile compaction and writes the chunk list + its count
+        p.tagg = tiles->tagg;
+        p.tids = tiles->tids;
+        p.n_tiles = (uint32_t)((tiles->n_pair + kTileTasks - 1) / kTileTasks);
+        p.tile_ids = (uint32_t)kTileTasks * 32;
+        p.list_out = const_cast<uint64_t *>(chunks);
+        p.n_chunks_out = const_cast<uint64_t *>(n_chunks_dev);
     }
-    const uint64_t warp_ctas = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
-    const unsigned g_mark = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[d].load()));
-    const unsigned g_emit = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[2 + d].load()));
-    // co-resident grid (the look-back relies on it); tiles are strided statically
-    const uint64_t max_tiles = (max_chunks + kVerifyScanTile - 1) / kVerifyScanTile;
-    const unsigned g_scan = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * occ[4].load()));
+    const uint64_t max_tiles = (max_chunks + tile - 1) / tile;
     unsigned long long *ticket_unused = nullptr;
     CK_TRY(get_scratch(dev, s, max_tiles, &p.states, &ticket_unused, &p.epoch));
     const size_t o_off = align256((size_t)max_chunks * 4);
@@ -1158,19 +1244,8 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     p.cnt = (uint32_t *)work;
     p.off = (uint64_t *)(work + o_off);
     p.mask = (uint32_t *)(work + o_mask);
-    {
-        ProfScope prof(3, s);
-        CK_CUDA(launch_k(d == 0 ? verify_mark_kernel<0> : verify_mark_kernel<1>, dim3(g_mark),
-                         dim3(kVerifyThreads), 0, s, p));
-        CK_LAUNCH();
-        CK_CUDA(launch_k(verify_scan_kernel, dim3(g_scan), dim3(kVerifyThreads), 0, s, p));
-        CK_LAUNCH();
-        if (before_emit) CK_TRY(before_emit(&p.out, &p.cap));
-        CK_CUDA(launch_k(d == 0 ? verify_emit_kernel<0> : verify_emit_kernel<1>, dim3(g_emit),
-                         dim3(kVerifyThreads), 0, s, p));
-    }
-    CK_LAUNCH();
-    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
+    *tab_out = tab;
+    *max_chunks_out = max_chunks;
     return CKPT_OK;
 }
 
@@ -1191,133 +1266,57 @@ extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tr
 }
 
 // ---------------------------------------------------------------------------
-// fused pair compare
-//   full mode: ONE leaf-kernel launch hashes both runs, compares the leaf digests,
-//     builds both trees' interior levels, marks the flagged chunks' elements and
-//     compacts them per tile (pairfin.cuh); one emit kernel then writes the chunk
-//     list and the element ids.
-//   fallback (more than kMaxTiles tiles, chunks > 1 MiB): K1 in flags-only pair
-//     mode, levels on the side stream, flag compaction, verify.
+// fused pair compare: K1 in pair mode (digest compare and
+// element marking in-kernel), then the ordered chunk list and the element ids
 // ---------------------------------------------------------------------------
-
-// Per-shape tables of the full mode (device, kept for the process lifetime: a
-// handful of KB per distinct checkpoint shape): the tree layout's metadata blob
-// shared by every tree of that shape, and the TreeTab of pairfin.cuh.
-struct PairShape {
-    uint8_t *meta = nullptr;
+// K5 (finish.cuh): both trees' level groups and the verify tiles over K1's tile compaction,
+// one launch on the compute stream after K1.
+static ckpt_status launch_finish(const void *const *a, const void *const *b, const uint64_t *n,
+                                 uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                 uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                                 uint64_t *counts_dev, cudaStream_t s, ckpt_tree *const *trees,
+                                 const PairParams &pp, int sms) {
+    int dev = 0;
+    CK_CUDA(cudaGetDevice(&dev));
+    static FinishParams fp;                   // large (kernel parameters); filled per launch
+    static std::mutex fp_mu;
+    std::lock_guard<std::mutex> lk(fp_mu);
+    std::memset(&fp, 0, sizeof(fp));
     uint8_t *tab = nullptr;
-    size_t o_cb = 0, o_nl = 0;
-    uint32_t n_ctr = 0;
-};
-static std::mutex g_shape_mu;
-static std::map<std::pair<int, std::vector<uint64_t>>, PairShape> g_shapes;
-
-static ckpt_status pair_shape(int dev, const ckpt_tree *t, PairShape *out) {
-    std::lock_guard<std::mutex> lk(g_shape_mu);
-    const auto key = std::make_pair(dev, t->n_leaves);
-    auto it = g_shapes.find(key);
-    if (it != g_shapes.end()) { *out = it->second; return CKPT_OK; }
-    const uint32_t m = t->n_arrays;
-    if (t->n_levels > (uint32_t)kMaxLv) return fail(CKPT_EINVAL, "tree too tall for the fused path");
-    std::vector<uint64_t> lvl((size_t)(m + 1) * kMaxLv, 0), nl(m + 1);
-    std::vector<uint32_t> cb((size_t)(m + 1) * kMaxSteps, 0);
-    uint64_t n_ctr = 0;
-    auto steps = [&](uint32_t a, uint64_t L) {
-        const uint32_t H = tree_height(L);
-        for (uint32_t j = 0; j < (uint32_t)kMaxSteps && H - 1 > (uint32_t)kGrpLog * j; ++j) {
-            cb[(size_t)a * kMaxSteps + j] = (uint32_t)n_ctr;
-            const uint32_t sh = (uint32_t)kGrpLog * (j + 1);
-            n_ctr += sh >= 64 ? 1 : (L + (1ull << sh) - 1) >> sh;     // nodes of level 7(j+1)
-        }
-    };
-    for (uint32_t a = 0; a < m; ++a) {
-        nl[a] = t->n_leaves[a];
-        for (uint32_t k = 0; k < t->height[a]; ++k) lvl[(size_t)a * kMaxLv + k] = t->off[(size_t)k * m + a];
-        steps(a, nl[a]);
-    }
-    nl[m] = m;
+    uint64_t max_chunks = 0;
+    CK_TRY(verify_setup(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps, idx,
+                        idx_cap, counts_dev + 1, s, 0, 0, &pp, kFinTile, fp.v, &tab, &max_chunks));
+    uint64_t *unused_states;
+    unsigned long long *tickets;
+    uint32_t unused_epoch;
     {
-        uint64_t at = t->top_off, n = m;
-        for (uint32_t k = 0;; ++k) {
-            lvl[(size_t)m * kMaxLv + k] = at;
-            if (n == 1) break;
-            at += n;
-            n = (n + 1) / 2;
-        }
-        steps(m, m);
+        // the level tickets (slots 1..2) and the finish ticket (slot 24) share the block
+        std::lock_guard<std::mutex> lk2(g_scr_mu);
+        Scratch &sc = g_scr[std::make_pair(dev, s)];
+        tickets = sc.ticket;
+        (void)unused_states;
+        (void)unused_epoch;
     }
-    if (n_ctr >= (1ull << 32)) return fail(CKPT_EINVAL, "too many level groups");
-    PairShape ps;
-    ps.n_ctr = (uint32_t)n_ctr;
-    ps.o_cb = align256(lvl.size() * 8);
-    ps.o_nl = ps.o_cb + align256(cb.size() * 4);
-    const size_t bytes = ps.o_nl + nl.size() * 8;
-    std::vector<uint8_t> host(bytes, 0);
-    std::memcpy(host.data(), lvl.data(), lvl.size() * 8);
-    std::memcpy(host.data() + ps.o_cb, cb.data(), cb.size() * 4);
-    std::memcpy(host.data() + ps.o_nl, nl.data(), nl.size() * 8);
-    CK_CUDA(cudaMalloc((void **)&ps.tab, bytes));
-    CK_CUDA(cudaMemcpy(ps.tab, host.data(), bytes, cudaMemcpyHostToDevice));
-    const size_t mb = t->meta_host.size() * 8;
-    CK_CUDA(cudaMalloc((void **)&ps.meta, mb));
-    CK_CUDA(cudaMemcpy(ps.meta, t->meta_host.data(), mb, cudaMemcpyHostToDevice));
-    g_shapes[key] = ps;
-    *out = ps;
-    return CKPT_OK;
-}
-
-// Full-mode scratch on (dev, s): counters and the job queue are zeroed once when allocated
-// (every launch returns them to zero); the other buffers are written before they are read.
-static ckpt_status get_full_scratch(int dev, cudaStream_t s, uint64_t L, uint64_t n_pair, uint32_t n_ctr,
-                                    uint32_t groups, PairParams *pp) {
-    std::lock_guard<std::mutex> lk(g_scr_mu);
-    Scratch &sc = g_scr[std::make_pair(dev, s)];
-    const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
-    // zero-once block: [qs 5 x u64 @0][acc 2 x u64 @64] | gctr [n_ctr] | tctr [n_tiles]
-    if (sc.fz_ctr < n_ctr || sc.fz_tiles < n_tiles) {
-        if (sc.fz) CK_CUDA(cudaFreeAsync(sc.fz, s));
-        sc.fz_ctr = std::max<size_t>(n_ctr, 2 * sc.fz_ctr);
-        sc.fz_tiles = std::max<size_t>(n_tiles, 2 * sc.fz_tiles);
-        const size_t bytes = 256 + align256(sc.fz_ctr * 4) + sc.fz_tiles * 4;
-        CK_CUDA(cudaMallocAsync((void **)&sc.fz, bytes, s));
-        CK_CUDA(cudaMemsetAsync(sc.fz, 0, bytes, s));
+    CK_TRY(fill_level_batch(trees, 2, s, tickets, fp.lv));
+    fp.n_level = fp.lv.cta_begin[fp.lv.n];
+    fp.ticket = tickets + 24;
+    const int d = dtype == CKPT_F32 ? 0 : 1;
+    auto kern = d == 0 ? finish_kernel<0> : finish_kernel<1>;
+    static std::atomic<int> occ[2] = {{0}, {0}};
+    if (occ[d].load() == 0) {
+        int o = 0;
+        CK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFinSmem));
+        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, kFinThreads, kFinSmem));
+        occ[d].store(std::max(o, 1));
     }
-    if (sc.fjobs_cap < L) {
-        if (sc.fjobs) CK_CUDA(cudaFreeAsync(sc.fjobs, s));
-        sc.fjobs_cap = std::max<size_t>(L, 2 * sc.fjobs_cap);
-        CK_CUDA(cudaMallocAsync((void **)&sc.fjobs, sc.fjobs_cap * 8, s));
-        CK_CUDA(cudaMemsetAsync(sc.fjobs, 0, sc.fjobs_cap * 8, s));
+    const uint64_t work = (uint64_t)fp.n_level + (max_chunks + kFinTile - 1) / kFinTile;
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(work, (uint64_t)sms * occ[d].load()));
+    {
+        ProfScope prof(3, s);
+        CK_CUDA(launch_k(kern, dim3(grid), dim3(kFinThreads), kFinSmem, s, fp));
     }
-    // [cnt L u32][mask L*groups*32 u32][tmask n_pair u32][tbase n_pair u64][tagg n_tiles u32]
-    // [thits n_tiles u64][tids n_tiles*kTileIds u64][tpos n_tiles*kTileIds u32]
-    size_t o[9];
-    o[0] = 0;
-    o[1] = align256(L * 4);
-    o[2] = o[1] + align256(L * groups * 128);
-    o[3] = o[2] + align256(n_pair * 4);
-    o[4] = o[3] + align256(n_pair * 8);
-    o[5] = o[4] + align256(n_tiles * 4);
-    o[6] = o[5] + align256(n_tiles * 8);
-    o[7] = o[6] + align256(n_tiles * kTileIds * 8);
-    o[8] = o[7] + n_tiles * kTileIds * 4;
-    if (sc.fbuf_cap < o[8]) {
-        if (sc.fbuf) CK_CUDA(cudaFreeAsync(sc.fbuf, s));
-        sc.fbuf_cap = std::max<size_t>(o[8], std::min<size_t>(2 * sc.fbuf_cap, o[8] + (64u << 20)));
-        CK_CUDA(cudaMallocAsync((void **)&sc.fbuf, sc.fbuf_cap, s));
-    }
-    pp->qs = (unsigned long long *)sc.fz;
-    pp->acc = (unsigned long long *)(sc.fz + 64);
-    pp->gctr = (unsigned int *)(sc.fz + 256);
-    pp->tctr = (unsigned int *)(sc.fz + 256 + align256(sc.fz_ctr * 4));
-    pp->q = (unsigned long long *)sc.fjobs;
-    pp->cnt = (uint32_t *)(sc.fbuf + o[0]);
-    pp->mask = (uint32_t *)(sc.fbuf + o[1]);
-    pp->tmask = (uint32_t *)(sc.fbuf + o[2]);
-    pp->tbase = (uint64_t *)(sc.fbuf + o[3]);
-    pp->tagg = (uint32_t *)(sc.fbuf + o[4]);
-    pp->thits = (uint64_t *)(sc.fbuf + o[5]);
-    pp->tids = (uint64_t *)(sc.fbuf + o[6]);
-    pp->tpos = (uint32_t *)(sc.fbuf + o[7]);
+    CK_LAUNCH();
+    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
     return CKPT_OK;
 }
 
@@ -1335,24 +1334,21 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
         return fail(CKPT_EINVAL, "NULL argument");
     if (n_arrays >= (1u << 20)) return fail(CKPT_EINVAL, "too many arrays");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
-    CK_TRY(norm_block(hash_block, chunk_bytes, &hash_block));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
-    uint64_t L = 0, n_pair = 0;
-    for (uint32_t k = 0; k < n_arrays; ++k) {
-        if (!a[k] || !b[k]) return fail(CKPT_EINVAL, "NULL data pointer");
-        if (n[k] == 0) return fail(CKPT_EINVAL, "empty array (n == 0)");
-        if ((uintptr_t)a[k] % 16 || (uintptr_t)b[k] % 16) return fail(CKPT_EINVAL, "data must be 16-byte aligned");
-        if (n[k] > (1ull << 50)) return fail(CKPT_EINVAL, "array too large");
-        const uint64_t l = (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
-        L += l;
-        n_pair += (l + kRows - 1) / kRows;
-    }
+    uint64_t L = 0;
+    for (uint32_t k = 0; k < n_arrays; ++k) L += (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
     int dev;
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
     cudaStream_t s = (cudaStream_t)stream;
-    const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
-    const bool full = n_tiles <= (uint64_t)kMaxTiles && chunk_bytes <= (1u << 20) && L < (1ull << 44);
+    PairParams pp;
+    std::memset(&pp, 0, sizeof(pp));
+    pp.m = (int)n_arrays;
+    // flag bytes live in their own per-stream buffer (verify's work buffer may regrow)
+    CK_TRY(get_pair_flags(dev, s, L, &pp.flags));
+    uint64_t n_pair = 0;                          // pair-tasks: kRows chunks of one array each
+    for (uint32_t k = 0; k < n_arrays; ++k) n_pair += ((n[k] * esz + chunk_bytes - 1) / chunk_bytes + kRows - 1) / kRows;
+    CK_TRY(get_tile_scratch(dev, s, n_pair, &pp));
     std::vector<const void *> data(2 * (size_t)n_arrays);
     std::vector<uint64_t> nn(2 * (size_t)n_arrays);
     for (uint32_t k = 0; k < n_arrays; ++k) {
@@ -1360,23 +1356,21 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
         data[n_arrays + k] = b[k];
         nn[k] = nn[n_arrays + k] = n[k];
     }
-    PairParams pp;
-    std::memset(&pp, 0, sizeof(pp));
-    pp.m = (int)n_arrays;
-    pp.n_pair = n_pair;
-    CK_TRY(get_pair_ctr(dev, s, n_pair, &pp.ctr));
+    const uint32_t apt[2] = {n_arrays, n_arrays};
+    ckpt_tree *trees[2] = {nullptr, nullptr};
+    // the ordered chunk list from K1's per-tile compaction: read directly by the finish kernel
+    // (or, with an exact-size output hook, K4a) up to kVerifyMaxTiles tiles, else placed by one
+    // gather pass
+    const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
+    const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
+    const bool finish = tiles_in_mark && !before_emit;
+    CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
+                            trees, &pp, finish));
     ckpt_status st = CKPT_OK;
-    if (!full) {
-        // flags-only K1 (+ levels on the side stream), flag compaction, verify
-        CK_TRY(get_pair_flags(dev, s, L, &pp.flags));
-        const uint32_t apt[2] = {n_arrays, n_arrays};
-        ckpt_tree *trees[2] = {nullptr, nullptr};
-        CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block,
-                                stream, trees, &pp));
-        st = launch_compact(1, nullptr, nullptr, pp.flags, L, chunks, chunks_cap, counts_dev, s, di.sms);
-        if (st == CKPT_OK)
-            st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
-                             idx, idx_cap, counts_dev + 1, s, before_emit);
+    pp.n_pair = n_pair;
+    if (finish) {
+        st = launch_finish(a, b, n, n_arrays, dtype, chunk_bytes, eps, chunks, chunks_cap, idx, idx_cap,
+                           counts_dev, s, trees, pp, di.sms);
         if (st != CKPT_OK) {
             ckpt_tree_free_on(trees[0], stream);
             ckpt_tree_free_on(trees[1], stream);
@@ -1386,150 +1380,30 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
         *out_b = trees[1];
         return CKPT_OK;
     }
-    // ---- full mode ----
-    ckpt_tree *tt[2] = {nullptr, nullptr};
-    auto cleanup = [&]() {
-        ckpt_tree_free_on(tt[0], stream);
-        ckpt_tree_free_on(tt[1], stream);
-    };
-    std::vector<uint64_t> leaves(n_arrays);
-    for (uint32_t k = 0; k < n_arrays; ++k) leaves[k] = (n[k] * esz + chunk_bytes - 1) / chunk_bytes;
-    PairShape ps;
-    for (int r = 0; r < 2 && st == CKPT_OK; ++r) {
-        ckpt_tree *t = new ckpt_tree();
-        tt[r] = t;
-        t->device = dev;
-        t->stream = s;
-        t->dtype = dtype;
-        t->chunk_bytes = chunk_bytes;
-        t->eps = eps;
-        t->hash_block = hash_block;
-        t->n_elems.assign(n, n + n_arrays);
-        layout(t, leaves);
-        if (r == 0) {
-            meta_layout(t);                      // the layout's blob on the host, then the cache
-            st = pair_shape(dev, t, &ps);
-        }
-        if (st == CKPT_OK) st = prepare_tree(t, s, ps.meta);
+    if (!tiles_in_mark) {
+        TileGatherParams g;
+        g.tagg = pp.tagg;
+        g.tids = pp.tids;
+        g.n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
+        g.tile_ids = (uint64_t)kTileTasks * 32;
+        g.out = chunks;
+        g.cap = chunks_cap;
+        g.count = counts_dev;
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(g.n_tiles, (uint64_t)di.sms * 8));
+        ProfScope prof(2, s);
+        if (launch_k(tile_gather_kernel, dim3(grid), dim3(kGatherThreads), 0, s, g) != cudaSuccess)
+            st = fail(CKPT_ECUDA, "tile gather launch");
     }
-    if (st != CKPT_OK) { cleanup(); return st; }
-    const uint32_t per = chunk_bytes / (uint32_t)esz;
-    const uint32_t groups = (per + 1023) / 1024;
-    st = get_full_scratch(dev, s, L, n_pair, ps.n_ctr, groups, &pp);
-    if (st != CKPT_OK) { cleanup(); return st; }
-    pp.tab.lvl = (const uint64_t *)ps.tab;
-    pp.tab.cb = (const uint32_t *)(ps.tab + ps.o_cb);
-    pp.tab.nl = (const uint64_t *)(ps.tab + ps.o_nl);
-    pp.tree[0] = tt[0]->nodes;
-    pp.tree[1] = tt[1]->nodes;
-    pp.groups = groups;
-    pp.per = per;
-    pp.eps = eps;
-    // the leaf table: A's arrays then B's, tasks in that order
-    std::vector<LeafArray> table;
-    table.reserve(2 * (size_t)n_arrays);
-    uint64_t task = 0;
-    for (int r = 0; r < 2; ++r) {
-        for (uint32_t k = 0; k < n_arrays; ++k) {
-            LeafArray e;
-            e.data = (const uint8_t *)(r ? b[k] : a[k]);
-            e.nbytes = n[k] * esz;
-            e.n_leaves = leaves[k];
-            e.n_full = e.nbytes / chunk_bytes;
-            e.task_begin = task;
-            e.out = tt[r]->nodes + tt[r]->off[k];
-            e.chunk_base = tt[r]->chunk_base[k];
-            table.push_back(e);
-            task += (leaves[k] + kRows - 1) / kRows;
-        }
+    if (st == CKPT_OK)
+        st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
+                         idx, idx_cap, counts_dev + 1, s, before_emit, 0, 0, tiles_in_mark ? &pp : nullptr);
+    if (st != CKPT_OK) {
+        ckpt_tree_free_on(trees[0], stream);
+        ckpt_tree_free_on(trees[1], stream);
+        return st;
     }
-    unsigned long long *ticket = nullptr;
-    {
-        uint64_t *unused_states;
-        uint32_t unused_epoch;
-        st = get_scratch(dev, s, 0, &unused_states, &ticket, &unused_epoch);
-        ticket += kLeafTicketSlot;
-    }
-    if (st == CKPT_OK) st = launch_leaves(table, task, dtype, eps, chunk_bytes, hash_block, s, di.sms, &pp, ticket);
-    if (st != CKPT_OK) { cleanup(); return st; }
-    // the emit kernel: chunk list, element ids, counts
-    VerifyParams p;
-    std::memset(&p, 0, sizeof(p));
-    uint8_t *vtab = nullptr;
-    {
-        std::vector<VerifyArray> va(n_arrays);
-        std::vector<uint64_t> cb(n_arrays);
-        uint64_t c = 0, e = 0;
-        for (uint32_t k = 0; k < n_arrays; ++k) {
-            va[k].a = (const uint8_t *)a[k];
-            va[k].b = (const uint8_t *)b[k];
-            va[k].n = n[k];
-            va[k].chunk_base = c;
-            va[k].elem_base = e;
-            cb[k] = c;
-            c += leaves[k];
-            e += n[k];
-        }
-        if (n_arrays <= (uint32_t)kVerifyInline) {
-            for (uint32_t k = 0; k < n_arrays; ++k) { p.inl[k] = va[k]; p.inl_base[k] = cb[k]; }
-        } else {
-            const size_t o_cb = align256((size_t)n_arrays * sizeof(VerifyArray));
-            std::vector<uint8_t> tbl(o_cb + (size_t)n_arrays * 8, 0);
-            std::memcpy(tbl.data(), va.data(), (size_t)n_arrays * sizeof(VerifyArray));
-            std::memcpy(tbl.data() + o_cb, cb.data(), (size_t)n_arrays * 8);
-            if (cudaMallocAsync((void **)&vtab, tbl.size(), s) != cudaSuccess) { cleanup(); return fail(CKPT_ENOMEM, "verify table"); }
-            st = g_ring.copy(vtab, tbl.data(), tbl.size(), s);
-            p.arrays = (const VerifyArray *)vtab;
-            p.chunk_base = (const uint64_t *)(vtab + o_cb);
-        }
-    }
-    p.n_arrays = (int)n_arrays;
-    p.chunks_cap = chunks_cap;
-    p.per = per;
-    p.groups = groups;
-    p.eps = eps;
-    p.cnt = pp.cnt;
-    p.mask = pp.mask;
-    p.out = idx;
-    p.cap = idx_cap;
-    p.tagg = pp.tagg;
-    p.thits = pp.thits;
-    p.tids = pp.tids;
-    p.tpos = pp.tpos;
-    p.n_tiles = (uint32_t)n_tiles;
-    p.list_out = chunks;
-    p.counts = counts_dev;
-    p.acc = pp.acc;
-    if (st == CKPT_OK && before_emit) {
-        // exact-size outputs: the totals of K1 reach counts_dev before the hook reads them
-        if (cudaMemcpyAsync(counts_dev, pp.acc, 16, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
-            st = fail(CKPT_ECUDA, "totals copy");
-        if (st == CKPT_OK) st = before_emit(&p.out, &p.cap);
-    }
-    if (st == CKPT_OK) {
-        static std::atomic<int> occ[2] = {{0}, {0}};
-        const int d = dtype == CKPT_F32 ? 0 : 1;
-        auto kern = d == 0 ? pair_emit_kernel<0> : pair_emit_kernel<1>;
-        if (occ[d].load() == 0) {
-            int o = 0;
-            if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPairEmitSmem) != cudaSuccess ||
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, kVerifyThreads, kPairEmitSmem) != cudaSuccess)
-                st = fail(CKPT_ECUDA, "pair emit kernel attributes");
-            occ[d].store(std::max(o, 1));
-        }
-        const uint64_t want = std::max<uint64_t>(1, (std::min<uint64_t>(L, chunks_cap) + kVerifyWarps - 1) / kVerifyWarps);
-        const unsigned grid = (unsigned)std::min<uint64_t>(want, (uint64_t)di.sms * occ[d].load());
-        if (st == CKPT_OK) {
-            ProfScope prof(3, s);
-            if (launch_k(kern, dim3(grid), dim3(kVerifyThreads), kPairEmitSmem, s, p) != cudaSuccess)
-                st = fail(CKPT_ECUDA, "pair emit launch");
-        }
-        if (st == CKPT_OK) g_launches.fetch_add(1, std::memory_order_relaxed);
-    }
-    if (vtab) cudaFreeAsync(vtab, s);
-    if (st != CKPT_OK) { cleanup(); return st; }
-    *out_a = tt[0];
-    *out_b = tt[1];
+    *out_a = trees[0];
+    *out_b = trees[1];
     return CKPT_OK;
 }
 

@@ -11,7 +11,6 @@
 
 #include "hash.cuh"
 #include "mark.cuh"
-#include "pairfin.cuh"
 
 namespace ckpt {
 
@@ -204,6 +203,52 @@ __global__ void __launch_bounds__(kCompactThreads) compact_kernel(const __grid_c
 }
 
 // ---------------------------------------------------------------------------
+// Ordered chunk list of the fused pair path from K1's tile compaction
+// (leaf.cuh, tile_compact): tile t's ids go to out[sum of tagg[0..t) ..].
+// One pass, no look-back; CTA 0 also writes the total count.
+// ---------------------------------------------------------------------------
+struct TileGatherParams {
+    const uint32_t *tagg;         // [n_tiles] flagged chunks per tile
+    const uint64_t *tids;         // [n_tiles * tile_ids] tile-compacted chunk ids
+    uint64_t n_tiles;
+    uint64_t tile_ids;            // id slots per tile
+    uint64_t *out;
+    uint64_t cap;
+    uint64_t *count;              // device: total flagged chunks
+};
+
+constexpr int kGatherThreads = 256;
+
+__global__ void __launch_bounds__(kGatherThreads) tile_gather_kernel(const __grid_constant__ TileGatherParams p) {
+    pdl_enter();
+    __shared__ uint64_t s_red[kGatherThreads / 32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    auto block_sum = [&](uint64_t upto) -> uint64_t {   // sum of tagg[0..upto)
+        uint64_t x = 0;
+        for (uint64_t i = threadIdx.x; i < upto; i += kGatherThreads) x += p.tagg[i];
+        x = warp_sum_u64(x);
+        if (lane == 0) s_red[warp] = x;
+        __syncthreads();
+        uint64_t t = 0;
+#pragma unroll
+        for (int w = 0; w < kGatherThreads / 32; ++w) t += s_red[w];
+        __syncthreads();
+        return t;
+    };
+    if (blockIdx.x == 0) {
+        const uint64_t total = block_sum(p.n_tiles);
+        if (threadIdx.x == 0) *p.count = total;
+    }
+    for (uint64_t t = blockIdx.x; t < p.n_tiles; t += gridDim.x) {
+        const uint64_t base = block_sum(t);
+        const uint32_t n = p.tagg[t];
+        const uint64_t *src = p.tids + t * p.tile_ids;
+        for (uint32_t k = threadIdx.x; k < n; k += kGatherThreads)
+            if (base + k < p.cap) p.out[base + k] = src[k];
+    }
+}
+
+// ---------------------------------------------------------------------------
 // BFS steps for a start level above the leaves.
 // Frontier entry: array (20 bits) | level (6 bits) | node (38 bits).
 // ---------------------------------------------------------------------------
@@ -344,17 +389,18 @@ struct VerifyParams {
     uint64_t *count;
     uint64_t *states;             // look-back state words (K4b)
     uint32_t epoch;
-    // fused pair path (pair_emit_kernel): K1's per-tile compaction (pairfin.cuh); cnt and
-    // mask are indexed by global chunk id there
-    const uint32_t *tagg;         // [n_tiles] flagged chunks per tile
-    const uint64_t *thits;        // [n_tiles] differing elements per tile
-    const uint64_t *tids;         // [n_tiles * kTileIds] flagged chunk ids
-    const uint32_t *tpos;         // [n_tiles * kTileIds] first hit of each chunk inside its tile
+    // fused pair path: the chunk list is K1's tile compaction (leaf.cuh
+    // tile_compact) read directly by K4a, which also writes it out (list_out,
+    // n_chunks_out = the device count every later kernel reads as n_chunks_dev)
+    const uint32_t *tagg;         // [n_tiles] flagged chunks per tile, or null
+    const uint64_t *tids;         // [n_tiles * tile_ids]
     uint32_t n_tiles;
-    uint64_t *list_out;           // the chunk list (chunks_cap entries)
-    uint64_t *counts;             // [2] flagged chunks, differing elements
-    unsigned long long *acc;      // K1's running totals, reset here
+    uint32_t tile_ids;
+    uint64_t *list_out;
+    uint64_t *n_chunks_out;
 };
+
+constexpr int kVerifyMaxTiles = 4096;   // tile prefix table of K4a in shared memory
 
 __device__ __forceinline__ uint64_t verify_n_chunks(const VerifyParams &p) {
     const uint64_t n = p.n_chunks_dev ? *p.n_chunks_dev : p.n_chunks_host;
@@ -381,6 +427,48 @@ __device__ __forceinline__ void verify_locate(const VerifyParams &p, uint64_t q,
                                               const uint8_t *&pa, const uint8_t *&pb,
                                               uint64_t &len, uint64_t &gbase) {
     verify_locate_g(p, p.chunks[q], esz, pa, pb, len, gbase);
+}
+
+// Tile mode: exclusive prefix of the tile counts into s_tpre[0..n_tiles]
+// (s_tpre[n_tiles] = total).  Called by all NT threads of the CTA.
+template <int NT = kVerifyThreads>
+__device__ __forceinline__ void tile_prefix(const VerifyParams &p, uint32_t *s_tpre) {
+    constexpr int NW = NT / 32;
+    __shared__ uint32_t s_w[NW];
+    constexpr int kPer = kVerifyMaxTiles / NT;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t nt = p.n_tiles;
+    const uint32_t t0 = threadIdx.x * kPer;
+    uint32_t v[kPer], sum = 0;
+#pragma unroll
+    for (int k = 0; k < kPer; ++k) {
+        v[k] = t0 + k < nt ? __ldcg(p.tagg + t0 + k) : 0u;
+        sum += v[k];
+    }
+    uint32_t wt;
+    uint32_t ex = warp_excl_scan_u32(sum, lane, wt);
+    if (lane == 0) s_w[warp] = wt;
+    __syncthreads();
+#pragma unroll
+    for (int w = 0; w < NW; ++w) ex += w < warp ? s_w[w] : 0u;
+#pragma unroll
+    for (int k = 0; k < kPer; ++k) {
+        if (t0 + k <= nt) s_tpre[t0 + k] = ex;
+        ex += v[k];
+    }
+    if (threadIdx.x == NT - 1 && nt == kVerifyMaxTiles) s_tpre[nt] = ex;
+    __syncthreads();
+}
+
+// Tile mode: chunk id of list position q (q < total).
+__device__ __forceinline__ uint64_t tile_chunk(const VerifyParams &p, const uint32_t *s_tpre, uint64_t q) {
+    uint32_t lo = 0, hi = p.n_tiles - 1;               // last tile with s_tpre[t] <= q
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (s_tpre[mid] <= q) lo = mid; else hi = mid - 1;
+    }
+    return __ldcg(reinterpret_cast<const unsigned long long *>(p.tids) + (uint64_t)lo * p.tile_ids +
+                  (q - s_tpre[lo]));
 }
 
 // Chunks per warp group: the largest power of two <= 32 that still gives
@@ -411,15 +499,31 @@ template <int DT>
 __global__ void __launch_bounds__(kVerifyThreads) verify_mark_kernel(const __grid_constant__ VerifyParams p) {
     pdl_enter();
     constexpr int ESZ = DT == 0 ? 4 : 8;
+    __shared__ uint32_t s_tpre[kVerifyMaxTiles + 1];
     const int lane = threadIdx.x & 31;
-    const uint64_t n_chunks = verify_n_chunks(p);
+    uint64_t n_chunks;
+    if (p.tagg) {
+        tile_prefix(p, s_tpre);
+        const uint64_t total = s_tpre[p.n_tiles];
+        if (blockIdx.x == 0 && threadIdx.x == 0) *p.n_chunks_out = total;
+        n_chunks = total < p.chunks_cap ? total : p.chunks_cap;
+    } else {
+        n_chunks = verify_n_chunks(p);
+    }
     const uint64_t n_warps = (uint64_t)gridDim.x * kVerifyWarps;
     const uint32_t G = verify_group(n_chunks, n_warps);
     for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + (threadIdx.x >> 5)) * G; q0 < n_chunks;
          q0 += n_warps * G) {
       ChunkLoc mine{nullptr, nullptr, 0, 0};
-      if (lane < (int)G && q0 + lane < n_chunks)
-          verify_locate(p, q0 + lane, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+      if (lane < (int)G && q0 + lane < n_chunks) {
+          if (p.tagg) {
+              const uint64_t g = tile_chunk(p, s_tpre, q0 + lane);
+              p.list_out[q0 + lane] = g;
+              verify_locate_g(p, g, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+          } else {
+              verify_locate(p, q0 + lane, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
+          }
+      }
       const uint32_t nq = (n_chunks - q0) < G ? (uint32_t)(n_chunks - q0) : G;
       for (uint32_t j = 0; j < nq; ++j) {
         const uint64_t q = q0 + j;
@@ -535,142 +639,6 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
               verify_locate(p, q0 + lane, ESZ, pa, pb, len, my_gb);
               // mark_chunk wrote ceil(len/1024) groups; the rest of the chunk's slot holds
               // stale words (a short last chunk of an array) and must not be read
-              my_groups = (uint32_t)((len + 1023) / 1024);
-          }
-      }
-      // sparse chunks: one lane each
-      if (c && c <= kEmitSparse) {
-          const uint4 *mw = reinterpret_cast<const uint4 *>(p.mask + my_key * n_words);
-          uint64_t o = my_off;
-#pragma unroll 1
-          for (uint32_t w4 = 0; w4 < my_groups * 8u; ++w4) {
-              const uint4 v = __ldcs(mw + w4);
-              const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-              for (int k = 0; k < 4; ++k) {
-                  const uint64_t e = my_gb + (uint64_t)(w4 * 4 + k) * 32;
-                  for (uint32_t mm = wv[k]; mm; mm &= mm - 1, ++o)
-                      if (o < p.cap) p.out[o] = e + (__ffs(mm) - 1);
-              }
-          }
-      }
-      // dense chunks: the whole warp
-#pragma unroll 1
-      for (uint32_t todo = __ballot_sync(kFull, c > kEmitSparse); todo; todo &= todo - 1) {
-        const int j = __ffs(todo) - 1;
-        const uint64_t gbase = __shfl_sync(kFull, my_gb, j);
-        uint64_t pos = __shfl_sync(kFull, my_off, j);
-        const uint32_t groups = __shfl_sync(kFull, my_groups, j);
-        const uint32_t *mq = p.mask + __shfl_sync(kFull, my_key, j) * n_words + lane;
-#pragma unroll 1
-        for (uint32_t g = 0; g < groups; ++g)
-            pos += emit_words(__ldcs(mq + g * 32), gbase + (uint64_t)g * 1024, pos, p.out, p.cap, lane,
-                              s_off);
-      }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// Fused pair path, the one kernel after K1: the ordered chunk list and the element
-// ids.  Every CTA prefixes the tiles' chunk and hit counts in shared memory; list
-// position q is found by binary search over the tile prefix, and its ids come from
-// the hit mask its marking job wrote (pairfin.cuh).  CTA 0 writes the two counts
-// and resets K1's running totals.
-// ---------------------------------------------------------------------------
-constexpr size_t kPairEmitSmem = (size_t)(kMaxTiles + 1) * 8 + (size_t)(kMaxTiles + 1) * 4;
-
-template <int DT>
-__global__ void __launch_bounds__(kVerifyThreads) pair_emit_kernel(const __grid_constant__ VerifyParams p) {
-    pdl_enter();
-    constexpr int ESZ = DT == 0 ? 4 : 8;
-    extern __shared__ __align__(16) uint8_t esm[];
-    uint64_t *s_hpre = reinterpret_cast<uint64_t *>(esm);
-    uint32_t *s_tpre = reinterpret_cast<uint32_t *>(esm + (size_t)(kMaxTiles + 1) * 8);
-    __shared__ uint16_t s_off_all[kVerifyWarps][1024];
-    __shared__ uint32_t s_wc[kVerifyWarps];
-    __shared__ uint64_t s_wh[kVerifyWarps];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    {
-        // exclusive prefix of the tiles' chunk and hit counts
-        constexpr int kPer = kMaxTiles / kVerifyThreads;
-        const uint32_t nt = p.n_tiles;
-        const uint32_t t0 = threadIdx.x * kPer;
-        uint32_t vc[kPer], sc = 0;
-        uint64_t vh[kPer], sh = 0;
-#pragma unroll
-        for (int k = 0; k < kPer; ++k) {
-            vc[k] = t0 + k < nt ? __ldcg(p.tagg + t0 + k) : 0u;
-            vh[k] = t0 + k < nt ? __ldcg(reinterpret_cast<const unsigned long long *>(p.thits) + t0 + k) : 0ull;
-            sc += vc[k];
-            sh += vh[k];
-        }
-        uint32_t xc = sc;
-        uint64_t xh = sh;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t yc = __shfl_up_sync(kFull, xc, o);
-            const uint64_t yh = __shfl_up_sync(kFull, xh, o);
-            if (lane >= o) { xc += yc; xh += yh; }
-        }
-        if (lane == 31) { s_wc[warp] = xc; s_wh[warp] = xh; }
-        __syncthreads();
-        uint32_t ec = xc - sc;
-        uint64_t eh = xh - sh;
-#pragma unroll
-        for (int w = 0; w < kVerifyWarps; ++w) {
-            if (w < warp) { ec += s_wc[w]; eh += s_wh[w]; }
-        }
-#pragma unroll
-        for (int k = 0; k < kPer; ++k) {
-            if (t0 + k <= nt) { s_tpre[t0 + k] = ec; s_hpre[t0 + k] = eh; }
-            ec += vc[k];
-            eh += vh[k];
-        }
-        if (threadIdx.x == kVerifyThreads - 1 && nt == kMaxTiles) { s_tpre[nt] = ec; s_hpre[nt] = eh; }
-        __syncthreads();
-    }
-    // the listed chunks: the first chunks_cap; the element ids (and their count) are those
-    // of the listed chunks, as in the unfused path
-    const uint64_t total_c = s_tpre[p.n_tiles];
-    const uint64_t n_chunks = total_c < p.chunks_cap ? total_c : p.chunks_cap;
-    auto tile_of = [&](uint64_t q) -> uint32_t {            // last tile with s_tpre[t] <= q
-        uint32_t lo = 0, hi = p.n_tiles - 1;
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi + 1) >> 1;
-            if (s_tpre[mid] <= q) lo = mid; else hi = mid - 1;
-        }
-        return lo;
-    };
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        uint64_t n_hits = s_hpre[p.n_tiles];
-        if (n_chunks < total_c) {                           // hits before list position n_chunks
-            const uint32_t t = tile_of(n_chunks);
-            n_hits = s_hpre[t] + __ldcg(p.tpos + (uint64_t)t * kTileIds + (n_chunks - s_tpre[t]));
-        }
-        p.counts[0] = total_c;
-        p.counts[1] = n_hits;
-        p.acc[0] = 0ull;
-        p.acc[1] = 0ull;
-    }
-    uint16_t *s_off = s_off_all[warp];
-    const uint64_t n_warps = (uint64_t)gridDim.x * kVerifyWarps;
-    const uint32_t G = verify_group(n_chunks, n_warps);
-    const uint32_t n_words = p.groups * 32;
-    for (uint64_t q0 = ((uint64_t)blockIdx.x * kVerifyWarps + warp) * G; q0 < n_chunks; q0 += n_warps * G) {
-      uint64_t my_off = 0, my_gb = 0, my_key = 0;
-      uint32_t c = 0, my_groups = 0;
-      if (lane < (int)G && q0 + lane < n_chunks) {
-          const uint64_t q = q0 + lane;
-          const uint32_t lo = tile_of(q);
-          const uint64_t slot = (uint64_t)lo * kTileIds + (q - s_tpre[lo]);
-          my_key = __ldcg(reinterpret_cast<const unsigned long long *>(p.tids) + slot);
-          p.list_out[q] = my_key;
-          c = __ldcg(p.cnt + my_key);
-          if (c) {
-              my_off = s_hpre[lo] + __ldcg(p.tpos + slot);
-              const uint8_t *pa, *pb;
-              uint64_t len;
-              verify_locate_g(p, my_key, ESZ, pa, pb, len, my_gb);
               my_groups = (uint32_t)((len + 1023) / 1024);
           }
       }

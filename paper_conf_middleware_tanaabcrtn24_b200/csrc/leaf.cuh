@@ -17,9 +17,7 @@
 #include <cstdint>
 
 #include "hash.cuh"
-#include "mark.cuh"
 #include "mm32.cuh"
-#include "pairfin.cuh"
 
 namespace ckpt {
 
@@ -211,11 +209,59 @@ constexpr int kLeafInline = 16;
 // arrays then B's m arrays (identical shapes); warp task t < n_pair is A's
 // task t, t >= n_pair is B's task t - n_pair (the usual batch order, so the
 // warps in flight stream one checkpoint at a time).  Whichever of the two
-// warps of a pair-task finishes second (a self-resetting counter per
-// pair-task) compares the 32 leaf digests: the diff at start level 0 happens
-// inside K1.  Flags-only mode (pr.tmask == null) writes one flag byte per
-// chunk; full mode also builds both trees' interior levels, marks the flagged
-// chunks' elements and compacts them per tile (pairfin.cuh).
+// warps of a pair-task finishes second (a self-resetting atomicInc counter per
+// pair-task) compares the 32 leaf digests and writes one flag byte per chunk:
+// the diff at start level 0 happens inside K1.  (Marking the flagged chunks'
+// elements here as well was measured slower than K4a: flagged chunks cluster,
+// so the marking serialises in the few warps that own them.)
+// Tile compaction (optional, tmask != null): pair-tasks are grouped in tiles
+// of kTileTasks; the warp that completes a tile's last pair-task (a
+// self-resetting acq_rel counter per tile) writes the tile's flagged chunk ids,
+// ascending, to tids[tile * kTileTasks * 32 ..] and their number to tagg[tile].
+// The ordered chunk list is then one gather pass (tile_gather_kernel) with no
+// look-back: the digest compare, the flags AND their compaction happen in K1.
+constexpr int kTileTasks = 128;                // pair-tasks per tile (4096 chunks)
+struct PairParams {
+    uint8_t *flags;               // [L] 1 if the chunk's leaf digests differ
+    unsigned int *ctr;            // [n_pair] 0 between launches (atomicInc wraps 1 -> 0)
+    uint64_t n_pair;              // pair-tasks (A's warp tasks)
+    int m;                        // arrays per checkpoint
+    uint32_t *tmask;              // [n_pair] differing-chunk mask per pair-task, or null
+    uint64_t *tbase;              // [n_pair] global chunk id of the pair-task's chunk 0
+    unsigned int *tctr;           // [n_tiles] 0 between launches
+    uint32_t *tagg;               // [n_tiles] flagged chunks per tile
+    uint64_t *tids;               // [n_tiles * kTileTasks * 32] tile-compacted chunk ids
+};
+
+// The tile's ordered chunk ids, by the warp that completed its last pair-task
+// (after an acquire of every pair-task's release).
+__device__ __noinline__ void tile_compact(const PairParams &pr, uint64_t tile, int lane) {
+    const uint64_t t0 = tile * kTileTasks;
+    const uint64_t t1 = (t0 + kTileTasks) < pr.n_pair ? t0 + kTileTasks : pr.n_pair;
+    uint64_t *dst = pr.tids + t0 * 32;
+    uint32_t run = 0;
+    for (uint64_t k = t0; k < t1; k += 32) {
+        const uint64_t pt = k + lane;
+        uint32_t m = 0;
+        uint64_t b = 0;
+        if (pt < t1) {
+            m = __ldcg(pr.tmask + pt);
+            b = __ldcg(reinterpret_cast<const unsigned long long *>(pr.tbase) + pt);
+        }
+        uint32_t x = __popc(m);
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        const uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
+        uint32_t pos = run + x - __popc(m);
+        for (uint32_t mm = m; mm; mm &= mm - 1) dst[pos++] = b + (uint64_t)(__ffs(mm) - 1);
+        run += tot;
+    }
+    if (lane == 0) pr.tagg[tile] = run;
+}
+
 struct LeafParams {
     const LeafArray *arrays;      // device table when n_arrays > kLeafInline
     LeafArray inl[kLeafInline];
@@ -239,54 +285,6 @@ __device__ __forceinline__ int find_array(const LeafArray *arr, int n_arrays, ui
         if (arr[mid].task_begin <= task) lo = mid; else hi = mid - 1;
     }
     return lo;
-}
-
-// One marking job of the full pair mode: the element test |a_i - b_i| > eps (R11) over
-// flagged chunk c of array aa (A's table index), hit bits and count stored by global chunk id.
-template <int DT>
-__device__ __noinline__ void mark_job(const LeafParams &P, const LeafArray *arrays,
-                                      unsigned long long e, int lane) {
-    e -= 1ull;
-    const int aa = (int)(e >> 44);
-    const uint64_t c = e & ((1ull << 44) - 1);
-    const LeafArray &XA = arrays[aa];
-    const LeafArray &XB = arrays[aa + P.pr.m];
-    constexpr uint64_t esz = DT == 0 ? 4 : 8;
-    const uint64_t n = XA.nbytes / esz;
-    const uint64_t e0 = c * P.pr.per;
-    const uint64_t len = (n - e0) < P.pr.per ? (n - e0) : P.pr.per;
-    const uint64_t gid = XA.chunk_base + c;
-    const uint32_t hits = mark_chunk<DT>(XA.data + e0 * esz, XB.data + e0 * esz, len, P.pr.eps,
-                                         P.pr.mask + gid * P.pr.groups * 32, lane);
-    if (lane == 0) P.pr.cnt[gid] = hits;
-    tile_arrive(P.pr, (XA.task_begin + c / kRows) / kTileTasks, 1u, lane);
-}
-
-// Full pair mode, by the warp that compared pair-task pt (array aa of A's table, local chunks
-// c0..c0+31): record the differing-chunk mask, queue one marking job per differing chunk,
-// count the compare into its tile, then climb both trees' levels from this pair-task.
-__device__ __noinline__ void pair_finish(const LeafParams &P, bool differ, int aa, uint64_t chunk_base,
-                                         uint64_t c0, uint64_t pt, uint4 *sm, int lane) {
-    const PairParams &pr = P.pr;
-    const uint32_t m = __ballot_sync(0xffffffffu, differ);
-    const int nm = __popc(m);
-    if (lane == 0) {
-        pr.tmask[pt] = m;
-        pr.tbase[pt] = chunk_base + c0;
-    }
-    if (nm) {
-        unsigned long long slot = 0;
-        if (lane == 0) slot = atomicAdd(pr.qs + 1, (unsigned long long)nm);
-        slot = __shfl_sync(0xffffffffu, slot, 0);
-        if (differ)
-            pr.q[slot + __popc(m & ((1u << lane) - 1u))] = (((unsigned long long)aa << 44) | (c0 + lane)) + 1ull;
-        __syncwarp();
-        if (lane == 0) atomicAdd(pr.qs + 4, (unsigned long long)nm);   // available to claimers
-    }
-    __syncwarp();
-    if (lane == 0) atom_add_rel64(pr.qs + 2, 1ull);      // compared (after the jobs were counted)
-    tile_arrive(pr, pt / kTileTasks, (unsigned int)(kTileUnits - nm), lane);
-    climb(pr, aa, c0 / kRows, true, sm, lane);
 }
 
 // CB = chunk bytes if known at compile time (multiple of kSeg), else 0.
@@ -333,27 +331,15 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
     // host then launches one CTA per task so that every SM gets the same number of chains)
     const uint32_t cta_warps = blockDim.x >> 5;
     const uint64_t n_warps_grid = (uint64_t)gridDim.x * cta_warps;
-    const bool full = PAIR && P.pr.tmask != nullptr;
-    uint4 *const wsm = reinterpret_cast<uint4 *>(smem + warp * kWarpSmem);   // the ring, as nodes
-    for (;;) {
-        // draw the next task; in full pair mode also look at the marking queue (same round trip)
+    auto draw = [&]() -> uint64_t {
         unsigned long long t = 0;
-        long long avail = 0;
         if (lane == 0) {
             t = atomicAdd(P.ticket, 1ull);
             if (t == n_tasks + n_warps_grid - 1) *P.ticket = 0ull;   // the last draw of the launch
-            if (full) avail = *reinterpret_cast<volatile long long *>(P.pr.qs + 4);
         }
-        const uint64_t task = __shfl_sync(0xffffffffu, t, 0);
-        if (full && __shfl_sync(0xffffffffu, avail, 0) > 0) {
-            // marking jobs first: they stay few and spread over every warp
-            for (;;) {
-                const unsigned long long e = claim_job(P.pr, lane);
-                if (!e) break;
-                mark_job<DT>(P, arrays, e, lane);
-            }
-        }
-        if (task >= n_tasks) break;
+        return __shfl_sync(0xffffffffu, t, 0);
+    };
+    for (uint64_t task = draw(); task < n_tasks; task = draw()) {
         const int a = find_array(arrays, n_arrays, task);
         const LeafArray A = arrays[a];
         const uint64_t c0 = (task - A.task_begin) * kRows;   // first local chunk of the task
@@ -511,49 +497,36 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
             order = __shfl_sync(0xffffffffu, order, 0);
             if (order == 1) {
                 __syncwarp();   // lane 0's acquire, then every lane's loads
-                const LeafArray &Pa = arrays[side ? a - P.pr.m : a + P.pr.m];   // the other run
+                const LeafArray Pa = arrays[side ? a - P.pr.m : a + P.pr.m];   // the other run
                 const uint64_t c = c0 + lane;
                 bool differ = false;
                 if (c < A.n_leaves) {
                     const uint4 o = __ldcg(Pa.out + c);
                     differ = (o.x != h1.lo) | (o.y != h1.hi) | (o.z != h2.lo) | (o.w != h2.hi);
-                    if (P.pr.flags) P.pr.flags[A.chunk_base + c] = differ ? 1 : 0;
+                    P.pr.flags[A.chunk_base + c] = differ ? 1 : 0;
                 }
-                if (full) pair_finish(P, differ, side ? a - P.pr.m : a, A.chunk_base, c0, pt, wsm, lane);
+                if (P.pr.tmask) {
+                    // publish this pair-task's mask, then count it into its tile
+                    const uint32_t m = __ballot_sync(0xffffffffu, differ);
+                    const uint64_t tile = pt / kTileTasks;
+                    const uint64_t rest = P.pr.n_pair - tile * kTileTasks;
+                    const unsigned int in_tile = (unsigned int)(rest < kTileTasks ? rest : kTileTasks);
+                    unsigned int done = 0;
+                    if (lane == 0) {
+                        P.pr.tmask[pt] = m;
+                        P.pr.tbase[pt] = A.chunk_base + c0;
+                        asm volatile("atom.acq_rel.gpu.global.inc.u32 %0, [%1], %2;"
+                                     : "=r"(done) : "l"(P.pr.tctr + tile), "r"(in_tile - 1u) : "memory");
+                    }
+                    done = __shfl_sync(0xffffffffu, done, 0);
+                    if (done == in_tile - 1u) {
+                        __syncwarp();
+                        tile_compact(P.pr, tile, lane);
+                    }
+                }
             }
         }
         __syncwarp();
-    }
-    if (full) {
-        // no leaf task left: keep marking until every pair-task is compared and the queue is
-        // empty (the last compares can still queue jobs), then count out; the last warp out
-        // empties the queue counters for the next launch
-        for (;;) {
-            const unsigned long long e = claim_job(P.pr, lane);
-            if (e) {
-                mark_job<DT>(P, arrays, e, lane);
-                continue;
-            }
-            unsigned long long pd = 0;
-            long long avail = 0;
-            if (lane == 0) {
-                pd = ld_acquire64(P.pr.qs + 2);
-                avail = *reinterpret_cast<volatile long long *>(P.pr.qs + 4);
-            }
-            pd = __shfl_sync(0xffffffffu, pd, 0);
-            avail = __shfl_sync(0xffffffffu, avail, 0);
-            // every pair-task compared (so every job counted) and none left to take; a job whose
-            // take failed transiently is taken by the warp that gave it back
-            if (pd == P.pr.n_pair && avail <= 0) break;
-            __nanosleep(1000);
-        }
-        __syncwarp();
-        if (lane == 0) {
-            const unsigned long long out = atomicAdd(P.pr.qs + 3, 1ull);
-            if (out == n_warps_grid - 1) {
-                for (int k = 0; k < 5; ++k) P.pr.qs[k] = 0ull;
-            }
-        }
     }
 }
 

@@ -127,13 +127,14 @@ __device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 
 }
 
 
-__global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_constant__ LevelBatch pb) {
-    pdl_enter();
-    extern __shared__ __align__(16) uint4 sm[];
-    __shared__ unsigned int s_ticket;
+// The work of level CTA `cta` (0 .. cta_begin[n]-1) of a batch: phase 1 for its group,
+// phase 2 if it is the last of its tree.  Called by all kLevelThreads threads of a CTA;
+// `sm` = kLevelSmem bytes of shared memory, s_ticket a shared word.
+__device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int cta, uint4 *sm,
+                                        unsigned int &s_ticket) {
     const int tid = threadIdx.x;
     int ti = 0;
-    while (ti + 1 < pb.n && blockIdx.x >= pb.cta_begin[ti + 1]) ++ti;
+    while (ti + 1 < pb.n && cta >= pb.cta_begin[ti + 1]) ++ti;
     const LevelParams &lp = pb.t[ti];
     const uint8_t *mb = lp.inl >= 0 ? reinterpret_cast<const uint8_t *>(pb.blob + lp.inl) : lp.meta;
     LvView p;
@@ -151,7 +152,7 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
     p.ls = lp.ls;
     p.n_groups = lp.n_groups;
     const int na = p.n_arrays;
-    if (lp.inl >= 0 && blockIdx.x == pb.cta_begin[ti]) {
+    if (lp.inl >= 0 && cta == pb.cta_begin[ti]) {
         // publish the inline tables to device memory for later BFS launches
         uint64_t *dst = reinterpret_cast<uint64_t *>(lp.meta);
         for (uint32_t w = tid; w < lp.meta_words; w += kLevelThreads) dst[w] = pb.blob[lp.inl + w];
@@ -165,7 +166,7 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
         // Every pass but the last few keeps whole warps busy, so the CTA's
         // 2047 hashes cost ~2047/32 warp-hashes instead of a lane-halving
         // shuffle tree, and 16 warps per CTA hide the hash latency.
-        const uint64_t gid = blockIdx.x - pb.cta_begin[ti];
+        const uint64_t gid = cta - pb.cta_begin[ti];
         const int a = find_le(p.gbegin, na, gid);
         const uint64_t g = gid - p.gbegin[a];
         const uint64_t n0 = p.cnt[(uint64_t)p.ls * na + a];
@@ -337,6 +338,13 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
         n = up;
     }
     if (tid == 0) *p.ticket = 0u;
+}
+
+__global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_constant__ LevelBatch pb) {
+    pdl_enter();
+    extern __shared__ __align__(16) uint4 sm[];
+    __shared__ unsigned int s_ticket;
+    levels_cta(pb, blockIdx.x, sm, s_ticket);
 }
 
 }  // namespace ckpt

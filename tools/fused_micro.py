@@ -11,7 +11,18 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_middleware_tanaabcrtn24_b200 as ck  # noqa: E402
 import synth  # noqa: E402
 
-n_part = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 26
+import argparse  # noqa: E402
+import ctypes  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--n", type=int, default=1 << 26)
+ap.add_argument("--lib", default="", help="an A/B variant library (tools/variant.py)")
+ap.add_argument("--quick", action="store_true", help="identical + c2 recipe only")
+args = ap.parse_args()
+if args.lib:
+    ck._lib = ck._declare(ctypes.CDLL(args.lib))
+    print("library:", args.lib, flush=True)
+n_part = args.n
 pair = synth.c2_pair(n_particles=n_part, seed=5, device="cuda")
 A = pair.a
 L = sum(t.numel() * 4 // 4096 for t in A)
@@ -39,6 +50,8 @@ def run(B, label, reps=10):
 
 run([t.clone() for t in A], "identical")
 run(pair.b, "c2 recipe")
+if args.quick:
+    sys.exit(0)
 per = 1024
 for k in (64, 1024, 16384):
     B = [t.clone() for t in A]
