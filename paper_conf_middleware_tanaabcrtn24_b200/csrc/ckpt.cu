@@ -452,6 +452,7 @@ static ckpt_status fill_level_batch(ckpt_tree *const *trees, int n, cudaStream_t
         p.o_lt = t->o_lt;
         p.o_h = t->o_h;
         p.o_g = t->o_g;
+        p.o_cb = t->o_cb;
         p.top_off = t->top_off;
         p.ticket = reinterpret_cast<unsigned int *>(tickets + 1 + i);   // slot 0: compactions
         p.n_arrays = (int)t->n_arrays;
@@ -581,6 +582,7 @@ struct Scratch {
     size_t flags_cap = 0;
     uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
     size_t tile_pairs = 0;              // pair-tasks the buffers hold
+    uint32_t tepoch = 0;                // tag of the last fused compare's tile flags
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -617,29 +619,33 @@ static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, Pa
     std::lock_guard<std::mutex> lk(g_scr_mu);
     Scratch &sc = g_scr[std::make_pair(dev, s)];
     n_pair = std::max<uint64_t>(n_pair, 1);
-    auto layout_of = [](uint64_t np, size_t o[5]) {
+    // [tctr: n_tiles u32][tdone: n_tiles u32] (zeroed once) [tagg][tmask][tbase][tids]
+    auto layout_of = [](uint64_t np, size_t o[6]) {
         const uint64_t nt = (np + kTileTasks - 1) / kTileTasks;
         o[0] = 0;
         o[1] = align256(nt * 4);
         o[2] = o[1] + align256(nt * 4);
-        o[3] = o[2] + align256(np * 4);
-        o[4] = o[3] + align256(np * 8);
-        return o[4] + nt * kTileTasks * 32 * 8;
+        o[3] = o[2] + align256(nt * 4);
+        o[4] = o[3] + align256(np * 4);
+        o[5] = o[4] + align256(np * 8);
+        return o[5] + nt * kTileTasks * 32 * 8;
     };
-    size_t o[5];
+    size_t o[6];
     if (sc.tile_pairs < n_pair) {
         if (sc.tile) CK_CUDA(cudaFreeAsync(sc.tile, s));
         sc.tile_pairs = std::max<uint64_t>(n_pair, 2 * sc.tile_pairs);
         const size_t bytes = layout_of(sc.tile_pairs, o);
         CK_CUDA(cudaMallocAsync((void **)&sc.tile, bytes, s));
-        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters
+        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[2], s));      // tile counters and flags
+        sc.tepoch = 0;
     }
     layout_of(sc.tile_pairs, o);
     pp->tctr = (unsigned int *)(sc.tile + o[0]);
-    pp->tagg = (uint32_t *)(sc.tile + o[1]);
-    pp->tmask = (uint32_t *)(sc.tile + o[2]);
-    pp->tbase = (uint64_t *)(sc.tile + o[3]);
-    pp->tids = (uint64_t *)(sc.tile + o[4]);
+    pp->tdone = (uint32_t *)(sc.tile + o[1]);
+    pp->tagg = (uint32_t *)(sc.tile + o[2]);
+    pp->tmask = (uint32_t *)(sc.tile + o[3]);
+    pp->tbase = (uint64_t *)(sc.tile + o[4]);
+    pp->tids = (uint64_t *)(sc.tile + o[5]);
     return CKPT_OK;
 }
 
@@ -664,7 +670,8 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
                                     const uint32_t *arrays_per_tree, uint32_t n_trees,
                                     ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
                                     uint32_t hash_block, void *stream, ckpt_tree **out,
-                                    const PairParams *pair, bool defer_levels = false) {
+                                    const PairParams *pair, bool defer_levels = false,
+                                    const std::function<ckpt_status(ckpt_tree **, PairParams *)> &pre_launch = nullptr) {
     if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
     for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
     if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
@@ -733,6 +740,9 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
         st = get_scratch(dev, s, 0, &unused_states, &ticket, &unused_epoch);
         ticket += kLeafTicketSlot;
     }
+    // work the caller stages between the trees' creation and the leaf launch (host->device
+    // copies must precede K1: a copy node after it would end the overlap with K1's tail)
+    if (st == CKPT_OK && pre_launch) st = pre_launch(out, pair ? &pp : nullptr);
     if (st == CKPT_OK)
         st = launch_leaves(table, task, dtype, eps, chunk_bytes, hash_block, s, di.sms,
                            pair ? &pp : nullptr, ticket);
@@ -1110,7 +1120,8 @@ static ckpt_status verify_setup(const void *const *a, const void *const *b, cons
                                 uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
                                 uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
                                 uint64_t chunk_base0, uint64_t elem_base0, const PairParams *tiles,
-                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out);
+                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out,
+                                uint64_t mask_slots = 0, uint64_t n_states = 0);
 
 static ckpt_status verify_impl(const void *const *a, const void *const *b, const uint64_t *n,
                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
@@ -1173,7 +1184,8 @@ static ckpt_status verify_setup(const void *const *a, const void *const *b, cons
                                 uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
                                 uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
                                 uint64_t chunk_base0, uint64_t elem_base0, const PairParams *tiles,
-                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out) {
+                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out,
+                                uint64_t mask_slots, uint64_t n_states) {
     if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
@@ -1234,13 +1246,14 @@ static ckpt_status verify_setup(const void *const *a, const void *const *b, cons
         p.list_out = const_cast<uint64_t *>(chunks);
         p.n_chunks_out = const_cast<uint64_t *>(n_chunks_dev);
     }
-    const uint64_t max_tiles = (max_chunks + tile - 1) / tile;
+    const uint64_t max_tiles = n_states ? n_states : (max_chunks + tile - 1) / tile;
     unsigned long long *ticket_unused = nullptr;
     CK_TRY(get_scratch(dev, s, max_tiles, &p.states, &ticket_unused, &p.epoch));
     const size_t o_off = align256((size_t)max_chunks * 4);
     const size_t o_mask = o_off + align256((size_t)max_chunks * 8);
     uint8_t *work = nullptr;
-    CK_TRY(get_work(dev, s, o_mask + (size_t)max_chunks * p.groups * 128, &work));
+    const uint64_t slots = mask_slots ? mask_slots : max_chunks;
+    CK_TRY(get_work(dev, s, o_mask + (size_t)slots * p.groups * 128, &work));
     p.cnt = (uint32_t *)work;
     p.off = (uint64_t *)(work + o_off);
     p.mask = (uint32_t *)(work + o_mask);
@@ -1269,37 +1282,49 @@ extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tr
 // fused pair compare: K1 in pair mode (digest compare and
 // element marking in-kernel), then the ordered chunk list and the element ids
 // ---------------------------------------------------------------------------
-// K5 (finish.cuh): both trees' level groups and the verify tiles over K1's tile compaction,
-// one launch on the compute stream after K1.
-static ckpt_status launch_finish(const void *const *a, const void *const *b, const uint64_t *n,
-                                 uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
-                                 uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
-                                 uint64_t *counts_dev, cudaStream_t s, ckpt_tree *const *trees,
-                                 const PairParams &pp, int sms) {
-    int dev = 0;
-    CK_CUDA(cudaGetDevice(&dev));
-    static FinishParams fp;                   // large (kernel parameters); filled per launch
-    static std::mutex fp_mu;
-    std::lock_guard<std::mutex> lk(fp_mu);
-    std::memset(&fp, 0, sizeof(fp));
+// K5 (finish.cuh): both trees' level groups and the verify items over K1's tiles, launched
+// right after K1 and running alongside its tail.  prepare_finish runs before K1 is launched
+// (its table copies must not sit between the two kernels), launch_finish after.
+struct FinishStage {
+    FinishParams fp;
     uint8_t *tab = nullptr;
     uint64_t max_chunks = 0;
+};
+
+static ckpt_status prepare_finish(const void *const *a, const void *const *b, const uint64_t *n,
+                                  uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
+                                  uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
+                                  uint64_t *counts_dev, cudaStream_t s, ckpt_tree *const *trees,
+                                  PairParams &pp, FinishStage &fs) {
+    int dev = 0;
+    CK_CUDA(cudaGetDevice(&dev));
+    std::memset(&fs.fp, 0, sizeof(fs.fp));
+    const uint64_t n_tiles = (pp.n_pair + kTileTasks - 1) / kTileTasks;
+    // look-back states: [0, n_tiles) element ids (p.states), [n_tiles, 2 n_tiles) chunk positions
     CK_TRY(verify_setup(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps, idx,
-                        idx_cap, counts_dev + 1, s, 0, 0, &pp, kFinTile, fp.v, &tab, &max_chunks));
-    uint64_t *unused_states;
-    unsigned long long *tickets;
-    uint32_t unused_epoch;
+                        idx_cap, counts_dev + 1, s, 0, 0, &pp, kTileIdsFin, fs.fp.v, &fs.tab, &fs.max_chunks,
+                        n_tiles * (uint64_t)kTileIdsFin, 2 * n_tiles));
+    fs.fp.states_c = fs.fp.v.states + n_tiles;
+    unsigned long long *tickets = nullptr;
     {
-        // the level tickets (slots 1..2) and the finish ticket (slot 24) share the block
-        std::lock_guard<std::mutex> lk2(g_scr_mu);
+        std::lock_guard<std::mutex> lk(g_scr_mu);
         Scratch &sc = g_scr[std::make_pair(dev, s)];
-        tickets = sc.ticket;
-        (void)unused_states;
-        (void)unused_epoch;
+        tickets = sc.ticket;                  // allocated by verify_setup's get_scratch
+        if (++sc.tepoch == 0) {               // epoch wrap: clear the tile flags once
+            CK_CUDA(cudaMemsetAsync(pp.tdone, 0, n_tiles * 4, s));
+            sc.tepoch = 1;
+        }
+        pp.tepoch = sc.tepoch;
     }
-    CK_TRY(fill_level_batch(trees, 2, s, tickets, fp.lv));
-    fp.n_level = fp.lv.cta_begin[fp.lv.n];
-    fp.ticket = tickets + 24;
+    CK_TRY(fill_level_batch(trees, 2, s, tickets, fs.fp.lv));
+    fs.fp.n_level = fs.fp.lv.cta_begin[fs.fp.lv.n];
+    fs.fp.ticket = tickets + 24;              // slots 1..4: level trees, 16: K1
+    fs.fp.tdone = pp.tdone;
+    fs.fp.tepoch = pp.tepoch;
+    return CKPT_OK;
+}
+
+static ckpt_status launch_finish(ckpt_dtype dtype, cudaStream_t s, FinishStage &fs, int sms) {
     const int d = dtype == CKPT_F32 ? 0 : 1;
     auto kern = d == 0 ? finish_kernel<0> : finish_kernel<1>;
     static std::atomic<int> occ[2] = {{0}, {0}};
@@ -1309,14 +1334,14 @@ static ckpt_status launch_finish(const void *const *a, const void *const *b, con
         CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, kFinThreads, kFinSmem));
         occ[d].store(std::max(o, 1));
     }
-    const uint64_t work = (uint64_t)fp.n_level + (max_chunks + kFinTile - 1) / kFinTile;
+    const uint64_t work = (uint64_t)fs.fp.n_level + fs.fp.v.n_tiles;
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(work, (uint64_t)sms * occ[d].load()));
     {
         ProfScope prof(3, s);
-        CK_CUDA(launch_k(kern, dim3(grid), dim3(kFinThreads), kFinSmem, s, fp));
+        CK_CUDA(launch_k(kern, dim3(grid), dim3(kFinThreads), kFinSmem, s, fs.fp));
     }
     CK_LAUNCH();
-    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
+    if (fs.tab) CK_CUDA(cudaFreeAsync(fs.tab, s));
     return CKPT_OK;
 }
 
@@ -1363,14 +1388,25 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     // gather pass
     const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
     const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
-    const bool finish = tiles_in_mark && !before_emit;
+    const bool finish = chunks_cap > 0 && !before_emit && !tile_gather_forced();
+    if (!finish) pp.tdone = nullptr;          // tile flags: only for the finish kernel
+    static FinishStage fs;                    // large (kernel parameters); one call at a time
+    static std::mutex fs_mu;
+    std::unique_lock<std::mutex> fs_lk(fs_mu, std::defer_lock);
+    std::function<ckpt_status(ckpt_tree **, PairParams *)> pre = nullptr;
+    if (finish) {
+        fs_lk.lock();
+        pre = [&](ckpt_tree **tt, PairParams *kp) -> ckpt_status {
+            return prepare_finish(a, b, n, n_arrays, dtype, chunk_bytes, eps, chunks, chunks_cap, idx,
+                                  idx_cap, counts_dev, s, tt, *kp, fs);
+        };
+    }
     CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
-                            trees, &pp, finish));
+                            trees, &pp, finish, pre));
     ckpt_status st = CKPT_OK;
     pp.n_pair = n_pair;
     if (finish) {
-        st = launch_finish(a, b, n, n_arrays, dtype, chunk_bytes, eps, chunks, chunks_cap, idx, idx_cap,
-                           counts_dev, s, trees, pp, di.sms);
+        st = launch_finish(dtype, s, fs, di.sms);
         if (st != CKPT_OK) {
             ckpt_tree_free_on(trees[0], stream);
             ckpt_tree_free_on(trees[1], stream);

@@ -1,24 +1,29 @@
-// finish.cuh -- K5: everything the fused pair path does after the leaf kernel, ONE launch.
+// finish.cuh -- K5: everything the fused pair path does after the leaves, ONE launch that
+// runs alongside the leaf kernel's tail.
 //
-// K1 (leaf.cuh, PAIR mode) leaves the leaves of both trees and, per tile of 4096 chunks,
-// the ascending ids of the chunks whose digests differ (the BFS of P:555-566 at start level
-// 0).  What remains is latency-bound: the interior levels of both trees (Alg. 1)
-// and the element test of the flagged chunks with the ordered output.  Doing it
-// inside K1 was measured 2-4x costlier than its instruction count (profiles/r2/inK1_finish_ab.md:
-// K1 is issue-bound at its register-limited 24 warps per SM, and latency-bound side work there
-// idles warp slots nothing else can fill), so it runs here, at full occupancy, with both
-// parts in one grid instead of a levels kernel on a side stream plus three verify kernels:
+// K1 (leaf.cuh, PAIR mode) leaves the leaves of both trees and, per tile of 128 pair-tasks
+// (4096 chunks), the ascending ids of the chunks whose digests differ (the BFS of P:555-566
+// at start level 0), publishing each finished tile with a release flag (tdone[tile] = the
+// launch's epoch).  What remains is latency-bound: the interior levels of both trees
+// (Alg. 1) and the element test of the flagged chunks with the ordered output
+// (P:568-578).  Doing it inside K1 was measured 2-4x costlier than its instruction count
+// (profiles/r2/inK1_finish_ab.md: K1 is issue-bound at its register-limited 24 warps per SM,
+// and latency-bound side work there idles warp slots nothing else can fill).  Here it runs in
+// its own grid, launched with programmatic dependent launch and WITHOUT waiting for K1 to
+// complete: its CTAs take the SM slots K1's CTAs free during K1's tail (the last ~10% of K1,
+// where warps run out of tasks) and consume K1's tiles as they are published.
 //
-//  * tickets [0, n_level_ctas): level groups of both trees (levels.cuh, levels_cta: 2048-node
-//    groups in shared memory, the last CTA of a tree builds the rest and the top tree);
-//  * the following tickets: verify tiles of kFinTile consecutive positions of the flagged
-//    chunk list, in list order.  A tile marks its chunks (one warp per chunk: binary64
-//    |a-b| > eps, R11, hit bits to the work buffer), scans their hit counts, finds its output
-//    offset by a decoupled look-back over the preceding tiles, and writes the element ids --
-//    a single pass, no grid-wide step between marking and emitting.
+//  * tickets [0, n_tiles): verify item k = K1 tile k.  Wait for tdone[k]; mark the tile's
+//    flagged chunks (one warp per chunk: binary64 |a-b| > eps, R11; hit bits to the work
+//    buffer), scan their hit counts in the CTA, then a decoupled look-back over the preceding
+//    items gives both the tile's first chunk-list position and its first element-id position;
+//    write the chunk ids and the element ids (ascending, coalesced).
+//  * tickets [n_tiles, n_tiles + n_level): level groups of both trees (levels.cuh,
+//    levels_cta: 2048 leaves of one array per CTA, the last CTA of a tree builds the rest and
+//    the top tree), each after the K1 tiles holding its leaves are published.
 //
-// Tickets are drawn in order by co-resident CTAs, so a look-back only waits on tiles that
-// running CTAs already hold.
+// Tickets are drawn in order by running CTAs and every wait is on work that K1 (resident from
+// its start) or an earlier ticket's CTA completes, so nothing waits on a CTA that cannot run.
 #pragma once
 #include <cstdint>
 
@@ -31,14 +36,20 @@ namespace ckpt {
 
 constexpr int kFinThreads = kLevelThreads;         // 512 (the level groups' CTA shape)
 constexpr int kFinWarps = kFinThreads / 32;
-constexpr int kFinPerWarp = 2;                     // list positions per warp and tile
-constexpr int kFinTile = kFinWarps * kFinPerWarp;  // 32 flagged chunks per verify tile
+constexpr int kTileIdsFin = 4096;                  // chunk slots per K1 tile (kTileTasks * 32)
+// dynamic shared memory: per-chunk hit counts of a tile (16 KB) + per-warp emit scratch
+// (2 KB each), or the level groups' kLevelSmem
+constexpr size_t kFinSmemVerify = (size_t)kTileIdsFin * 4 + (size_t)kFinWarps * 2048;
+constexpr size_t kFinSmem = kFinSmemVerify > (size_t)kLevelSmem ? kFinSmemVerify : (size_t)kLevelSmem;
 
 struct FinishParams {
     LevelBatch lv;                // both trees' level groups (lv.cta_begin[lv.n] CTAs)
-    VerifyParams v;               // tile mode (v.tagg != null): the list comes from K1's tiles
+    VerifyParams v;               // tagg / tids / n_tiles: K1's tiles; mask: per tile slot
     unsigned long long *ticket;   // 0 on entry; the last draw resets it
     unsigned int n_level;         // level tickets
+    const uint32_t *tdone;        // [n_tiles] K1's tile flags
+    uint32_t tepoch;              // this pair compare's tag in tdone
+    uint64_t *states_c;           // look-back states of the chunk-list positions (p.states: element ids)
 };
 
 __device__ __forceinline__ uint64_t fin_draw(unsigned long long *ticket, uint64_t n_total,
@@ -53,85 +64,130 @@ __device__ __forceinline__ uint64_t fin_draw(unsigned long long *ticket, uint64_
     return *s_t;
 }
 
-constexpr size_t kFinSmem = (size_t)kFinWarps * 1024 * 2 > (size_t)kLevelSmem
-                               ? (size_t)kFinWarps * 1024 * 2 : (size_t)kLevelSmem;
+// Thread 0 waits (acquire, growing sleep) until K1 published tiles [lo, hi]; then a barrier.
+__device__ __forceinline__ void fin_wait_tiles(const FinishParams &P, uint64_t lo, uint64_t hi) {
+    if (threadIdx.x == 0) {
+        unsigned int nap = 64;
+        for (uint64_t k = lo; k <= hi; ++k) {
+            for (;;) {
+                uint32_t v;
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.tdone + k) : "memory");
+                if (v == P.tepoch) break;
+                __nanosleep(nap);
+                nap = nap < 2048u ? 2u * nap : 2048u;
+            }
+        }
+    }
+    __syncthreads();
+}
 
 template <int DT>
 __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_constant__ FinishParams P) {
-    pdl_enter();
+    // no griddepcontrol.wait: this grid runs while K1 still does (see above); its successor
+    // waits for it as usual
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     constexpr int ESZ = DT == 0 ? 4 : 8;
-    extern __shared__ __align__(16) uint4 fin_sm[];              // kFinSmem: level groups / emit scratch
-    __shared__ uint32_t s_tpre[kVerifyMaxTiles + 1];             // K1 tile prefix (list positions)
-    __shared__ uint32_t s_cnt[kFinTile], s_ex[kFinTile], s_len[kFinTile];
-    __shared__ uint64_t s_gb[kFinTile];
-    __shared__ const uint8_t *s_pa[kFinTile], *s_pb[kFinTile];
-    __shared__ uint32_t s_sum;
+    extern __shared__ __align__(16) uint4 fin_sm[];
+    __shared__ uint32_t s_w[kFinWarps];
     __shared__ uint64_t s_t;
     __shared__ unsigned int s_ticket;
     const VerifyParams &p = P.v;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    // the flagged-chunk list: K1's per-tile compaction, prefixed once per CTA
-    tile_prefix<kFinThreads>(p, s_tpre);
-    const uint64_t total = s_tpre[p.n_tiles];
-    const uint64_t n_list = total < p.chunks_cap ? total : p.chunks_cap;
-    const uint64_t n_vt = (n_list + kFinTile - 1) / kFinTile;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        *p.n_chunks_out = total;
-        if (n_vt == 0) *p.count = 0;
-    }
-    const uint64_t n_total = P.n_level + n_vt;
+    const uint64_t n_tiles = p.n_tiles;
+    const uint64_t n_total = n_tiles + P.n_level;
     for (uint64_t t = fin_draw(P.ticket, n_total, &s_t); t < n_total; t = fin_draw(P.ticket, n_total, &s_t)) {
-        if (t < P.n_level) {
-            levels_cta(P.lv, (unsigned int)t, fin_sm, s_ticket);
+        if (t >= n_tiles) {
+            // ------------------------------ a level group ------------------------------
+            const unsigned int cta = (unsigned int)(t - n_tiles);
+            int ti = 0;
+            while (ti + 1 < P.lv.n && cta >= P.lv.cta_begin[ti + 1]) ++ti;
+            const LevelParams &lp = P.lv.t[ti];
+            const uint8_t *mb = lp.inl >= 0 ? reinterpret_cast<const uint8_t *>(P.lv.blob + lp.inl) : lp.meta;
+            const uint64_t *gbegin = reinterpret_cast<const uint64_t *>(mb + lp.o_g);
+            const uint64_t *cnt0 = reinterpret_cast<const uint64_t *>(mb + lp.o_cnt);   // level 0
+            const int na = lp.n_arrays;
+            const uint64_t gid = cta - P.lv.cta_begin[ti];
+            const int a = find_le(gbegin, na, gid);
+            // pair-tasks (32 chunks of one array each, array-major) holding the group's leaves
+            uint64_t tb = 0;
+            for (int k = 0; k < a; ++k) tb += (cnt0[k] + 31) / 32;
+            const uint64_t g = gid - gbegin[a];
+            const uint64_t c_lo = g * kGroup;
+            const uint64_t c_hi = (c_lo + kGroup < cnt0[a] ? c_lo + kGroup : cnt0[a]) - 1;
+            fin_wait_tiles(P, (tb + c_lo / 32) / kTileTasks, (tb + c_hi / 32) / kTileTasks);
+            levels_cta(P.lv, cta, fin_sm, s_ticket);
             continue;
         }
-        // ---------------- verify tile vt: list positions [q0, q0 + kFinTile) ----------------
-        const uint64_t vt = t - P.n_level;
-        const uint64_t q0 = vt * kFinTile;
-        const uint32_t nq = (uint32_t)((n_list - q0) < (uint64_t)kFinTile ? (n_list - q0) : kFinTile);
-        if (threadIdx.x < kFinTile) {                  // locate the tile's chunks, one thread each
-            const uint32_t j = threadIdx.x;
-            const uint8_t *pa = nullptr, *pb = nullptr;
-            uint64_t len = 0, gb = 0;
-            if (j < nq) {
-                const uint64_t g = tile_chunk(p, s_tpre, q0 + j);
-                p.list_out[q0 + j] = g;
-                verify_locate_g(p, g, ESZ, pa, pb, len, gb);
-            }
-            s_pa[j] = pa;
-            s_pb[j] = pb;
-            s_len[j] = (uint32_t)len;
-            s_gb[j] = gb;
-        }
-        __syncthreads();
-        for (int k = 0; k < kFinPerWarp; ++k) {        // mark: one warp per chunk
-            const uint32_t j = warp * kFinPerWarp + k;
-            uint32_t c = 0;
-            if (j < nq)
-                c = mark_chunk<DT>(s_pa[j], s_pb[j], s_len[j], p.eps, p.mask + (q0 + j) * p.groups * 32, lane);
+        // ------------------------------ verify item k ------------------------------
+        const uint64_t k = t;
+        fin_wait_tiles(P, k, k);
+        const uint32_t n = __ldcg(p.tagg + k);
+        uint32_t *s_cnt = reinterpret_cast<uint32_t *>(fin_sm);           // [kTileIdsFin]
+        const uint64_t *ids = p.tids + k * kTileIdsFin;
+        for (uint32_t j = warp; j < n; j += kFinWarps) {                  // mark: a warp per chunk
+            const uint64_t g = __ldcg(reinterpret_cast<const unsigned long long *>(ids) + j);
+            const uint8_t *pa, *pb;
+            uint64_t len, gb;
+            verify_locate_g(p, g, ESZ, pa, pb, len, gb);
+            const uint32_t c = mark_chunk<DT>(pa, pb, len, p.eps, p.mask + (k * kTileIdsFin + j) * p.groups * 32, lane);
             if (lane == 0) s_cnt[j] = c;
         }
         __syncthreads();
-        if (warp == 0) {                               // the tile's exclusive prefix of hit counts
-            uint32_t tot;
-            const uint32_t ex = warp_excl_scan_u32(lane < kFinTile ? s_cnt[lane] : 0u, lane, tot);
-            if (lane < kFinTile) s_ex[lane] = ex;
-            if (lane == 0) s_sum = tot;
+        // exclusive prefix of the hit counts over the tile's chunks (8 per thread)
+        constexpr int kPer = kTileIdsFin / kFinThreads;
+        uint32_t v[kPer], sum = 0;
+        const uint32_t j0 = threadIdx.x * kPer;
+#pragma unroll
+        for (int i = 0; i < kPer; ++i) {
+            v[i] = j0 + i < n ? s_cnt[j0 + i] : 0u;
+            sum += v[i];
+        }
+        uint32_t wtot;
+        uint32_t ex = warp_excl_scan_u32(sum, lane, wtot);
+        if (lane == 0) s_w[warp] = wtot;
+        __syncthreads();
+        uint32_t hits = 0;
+#pragma unroll
+        for (int w = 0; w < kFinWarps; ++w) {
+            const uint32_t x = s_w[w];
+            if (w < warp) ex += x;
+            hits += x;
+        }
+#pragma unroll
+        for (int i = 0; i < kPer; ++i) {
+            if (j0 + i < n) s_cnt[j0 + i] = ex;                // now: first hit of chunk j inside the tile
+            ex += v[i];
         }
         __syncthreads();
-        const uint64_t excl = cta_lookback<kFinThreads>(p.states, vt, s_sum, p.epoch);
-        if (threadIdx.x == 0 && vt == n_vt - 1) *p.count = excl + s_sum;
-        // ids: each warp writes its own chunks' (ascending, coalesced)
-        uint16_t *s_off = reinterpret_cast<uint16_t *>(fin_sm) + warp * 1024;
-        for (int k = 0; k < kFinPerWarp; ++k) {
-            const uint32_t j = warp * kFinPerWarp + k;
-            if (j >= nq || s_cnt[j] == 0) continue;    // warp-uniform
-            uint64_t pos = excl + s_ex[j];
-            const uint32_t groups = (s_len[j] + 1023) / 1024;
-            const uint32_t *mq = p.mask + (q0 + j) * p.groups * 32 + lane;
-            for (uint32_t g = 0; g < groups; ++g)
-                pos += emit_words(__ldcs(mq + g * 32), s_gb[j] + (uint64_t)g * 1024, pos, p.out, p.cap, lane,
-                                  s_off);
+        // the tile's place: chunk-list positions and element-id positions of all earlier tiles
+        const uint64_t excl_c = cta_lookback<kFinThreads>(P.states_c, k, n, p.epoch);
+        const uint64_t excl_h = cta_lookback<kFinThreads>(p.states, k, hits, p.epoch);
+        const uint64_t cap_c = p.chunks_cap;
+        if (threadIdx.x == 0) {
+            if (k == n_tiles - 1) {
+                *p.n_chunks_out = excl_c + n;
+                if (excl_c + n <= cap_c) *p.count = excl_h + hits;
+            }
+            // the chunk-list capacity cuts this tile: the element ids are those of listed chunks
+            if (excl_c < cap_c && cap_c < excl_c + n) *p.count = excl_h + s_cnt[cap_c - excl_c];
+        }
+        const uint32_t n_listed = excl_c >= cap_c ? 0u : (uint32_t)((cap_c - excl_c) < n ? (cap_c - excl_c) : n);
+        for (uint32_t j = threadIdx.x; j < n_listed; j += kFinThreads)
+            p.list_out[excl_c + j] = __ldcg(reinterpret_cast<const unsigned long long *>(ids) + j);
+        uint16_t *s_off = reinterpret_cast<uint16_t *>(reinterpret_cast<uint8_t *>(fin_sm) + kTileIdsFin * 4) + warp * 1024;
+        for (uint32_t j = warp; j < n_listed; j += kFinWarps) {           // ids: a warp per chunk
+            const uint32_t c0 = s_cnt[j];
+            const uint32_t c1 = j + 1 < n ? s_cnt[j + 1] : hits;
+            if (c1 == c0) continue;                                       // warp-uniform
+            const uint64_t g = __ldcg(reinterpret_cast<const unsigned long long *>(ids) + j);
+            const uint8_t *pa, *pb;
+            uint64_t len, gb;
+            verify_locate_g(p, g, ESZ, pa, pb, len, gb);
+            uint64_t pos = excl_h + c0;
+            const uint32_t groups = (uint32_t)((len + 1023) / 1024);
+            const uint32_t *mq = p.mask + (k * kTileIdsFin + j) * p.groups * 32 + lane;
+            for (uint32_t gr = 0; gr < groups; ++gr)
+                pos += emit_words(__ldcs(mq + gr * 32), gb + (uint64_t)gr * 1024, pos, p.out, p.cap, lane, s_off);
         }
     }
 }

@@ -47,6 +47,7 @@ struct LevelParams {
     uint32_t o_lt;                // u64 [level]: nodes in level (all arrays)
     uint32_t o_h;                 // u32 [a]: number of levels of array a
     uint32_t o_g;                 // u64 [a]: first group of array a
+    uint32_t o_cb;                // u64 [a]: global chunk id of array a's leaf 0
     uint64_t top_off;             // node index of the top tree's level 0
     unsigned int *ticket;         // zero on entry, reset to zero by the last CTA
     int n_arrays;
@@ -194,8 +195,8 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
                         uint4 *l2 = p.nodes + p.off[(uint64_t)(p.ls + r + 2) * na + a] + (start >> (r + 2));
                         uint4 x0, x1, x2, x3;
                         if (r == 0) {
-                            x0 = __ldg(src + 4 * tid); x1 = __ldg(src + 4 * tid + 1);
-                            x2 = __ldg(src + 4 * tid + 2); x3 = __ldg(src + 4 * tid + 3);
+                            x0 = __ldcg(src + 4 * tid); x1 = __ldcg(src + 4 * tid + 1);
+                            x2 = __ldcg(src + 4 * tid + 2); x3 = __ldcg(src + 4 * tid + 3);
                         } else {
                             x0 = in[4 * tid]; x1 = in[4 * tid + 1]; x2 = in[4 * tid + 2]; x3 = in[4 * tid + 3];
                         }
@@ -229,7 +230,7 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
                     x[j] = make_uint4(0u, 0u, 0u, 0u);
-                    if (j < mt) x[j] = r == 0 ? __ldg(src + per * tid + j) : in[per * tid + j];
+                    if (j < mt) x[j] = r == 0 ? __ldcg(src + per * tid + j) : in[per * tid + j];
                 }
                 const uint4 y0 = mt >= 2 ? hash_children32(x[0], x[1]) : x[0];
                 write(r + 1, (uint64_t)(per / 2) * tid, y0);
