@@ -583,6 +583,8 @@ struct Scratch {
     uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
     size_t tile_pairs = 0;              // pair-tasks the buffers hold
     uint32_t tepoch = 0;                // tag of the last fused compare's tile flags
+    unsigned int *lctr = nullptr;       // finish kernel level arrivals (zeroed once, self-resetting)
+    size_t lctr_cap = 0;
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -941,7 +943,7 @@ static void release_scratch(int dev, cudaStream_t s) {
     auto it = g_scr.find(std::make_pair(dev, s));
     if (it == g_scr.end()) return;
     Scratch &sc = it->second;
-    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile};
+    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile, sc.lctr};
     for (void *b : bufs)
         if (b) cudaFreeAsync(b, s);
     g_scr.erase(it);
@@ -1315,6 +1317,14 @@ static ckpt_status prepare_finish(const void *const *a, const void *const *b, co
             sc.tepoch = 1;
         }
         pp.tepoch = sc.tepoch;
+        const size_t need = 2 * (size_t)n_arrays + 2;
+        if (sc.lctr_cap < need) {
+            if (sc.lctr) CK_CUDA(cudaFreeAsync(sc.lctr, s));
+            sc.lctr_cap = std::max(need, 2 * sc.lctr_cap);
+            CK_CUDA(cudaMallocAsync((void **)&sc.lctr, sc.lctr_cap * 4, s));
+            CK_CUDA(cudaMemsetAsync(sc.lctr, 0, sc.lctr_cap * 4, s));
+        }
+        fs.fp.lctr = sc.lctr;
     }
     CK_TRY(fill_level_batch(trees, 2, s, tickets, fs.fp.lv));
     fs.fp.n_level = fs.fp.lv.cta_begin[fs.fp.lv.n];

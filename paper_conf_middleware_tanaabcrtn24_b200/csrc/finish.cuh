@@ -18,9 +18,10 @@
 //    buffer), scan their hit counts in the CTA, then a decoupled look-back over the preceding
 //    items gives both the tile's first chunk-list position and its first element-id position;
 //    write the chunk ids and the element ids (ascending, coalesced).
-//  * tickets [n_tiles, n_tiles + n_level): level groups of both trees (levels.cuh,
-//    levels_cta: 2048 leaves of one array per CTA, the last CTA of a tree builds the rest and
-//    the top tree), each after the K1 tiles holding its leaves are published.
+//  * tickets [n_tiles, n_tiles + n_level): level groups of both trees, each after the K1
+//    tiles holding its leaves are published: 2048 leaves of one array per CTA reduced 11
+//    levels up (reduce.cuh: registers, shuffles, one barrier); the last group of an array
+//    builds the array's remaining levels, the last array of a tree the top tree (R15).
 //
 // Tickets are drawn in order by running CTAs and every wait is on work that K1 (resident from
 // its start) or an earlier ticket's CTA completes, so nothing waits on a CTA that cannot run.
@@ -31,6 +32,7 @@
 #include "hash.cuh"
 #include "levels.cuh"
 #include "mark.cuh"
+#include "reduce.cuh"
 
 namespace ckpt {
 
@@ -50,7 +52,14 @@ struct FinishParams {
     const uint32_t *tdone;        // [n_tiles] K1's tile flags
     uint32_t tepoch;              // this pair compare's tag in tdone
     uint64_t *states_c;           // look-back states of the chunk-list positions (p.states: element ids)
+    unsigned int *lctr;           // [2 * na + 2] level arrivals per (tree, array), per tree; 0 between launches
 };
+
+__device__ __forceinline__ unsigned int atom_add_acq_rel_u32(unsigned int *p, unsigned int v) {
+    unsigned int old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
 
 __device__ __forceinline__ uint64_t fin_draw(unsigned long long *ticket, uint64_t n_total,
                                              uint64_t *s_t) {
@@ -115,7 +124,47 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
             const uint64_t c_lo = g * kGroup;
             const uint64_t c_hi = (c_lo + kGroup < cnt0[a] ? c_lo + kGroup : cnt0[a]) - 1;
             fin_wait_tiles(P, (tb + c_lo / 32) / kTileTasks, (tb + c_hi / 32) / kTileTasks);
-            levels_cta(P.lv, cta, fin_sm, s_ticket);
+            if (lp.inl >= 0 && gid == 0) {
+                // publish the inline tables to device memory for later BFS launches
+                uint64_t *dst = reinterpret_cast<uint64_t *>(lp.meta);
+                for (uint32_t w = threadIdx.x; w < lp.meta_words; w += kFinThreads) dst[w] = P.lv.blob[lp.inl + w];
+            }
+            TreeRef T;
+            T.nodes = lp.nodes;
+            T.off = reinterpret_cast<const uint64_t *>(mb + lp.o_off);
+            T.cnt = cnt0;
+            T.height = reinterpret_cast<const uint32_t *>(mb + lp.o_h);
+            T.top_off = lp.top_off;
+            T.na = na;
+            uint4 *s_root = fin_sm;
+            const int H = (int)T.height[a];
+            if (H > 1)
+                reduce_block(T, a, 0, c_lo, (uint32_t)(c_hi + 1 - c_lo), H - 1 < kRedBlockLog ? H - 1 : kRedBlockLog, s_root);
+            if (H - 1 > kRedBlockLog) {
+                // the last group of the array builds the array's remaining levels
+                const uint32_t n_g = (uint32_t)((cnt0[a] + kGroup - 1) / kGroup);     // the array's groups
+                if (threadIdx.x == 0) {
+                    unsigned int *c = P.lctr + (uint32_t)ti * (uint32_t)na + (uint32_t)a;
+                    const unsigned int old = atom_add_acq_rel_u32(c, 1u);
+                    s_ticket = old;
+                    if (old == n_g - 1) *c = 0u;
+                }
+                __syncthreads();
+                if (s_ticket != n_g - 1) continue;
+                reduce_up(T, a, kRedBlockLog, T.count(a, kRedBlockLog), s_root);
+            }
+            // the array root is final: it is level-0 node a of the top tree; the last array
+            // of the tree builds the top
+            if (threadIdx.x == 0) {
+                *T.at(na, 0, (uint64_t)a) = __ldcg(T.at(a, H - 1, 0));
+                unsigned int *c = P.lctr + 2 * (uint32_t)na + (uint32_t)ti;
+                const unsigned int old = atom_add_acq_rel_u32(c, 1u);
+                s_ticket = old;
+                if (old == (unsigned int)na - 1) *c = 0u;
+            }
+            __syncthreads();
+            if (s_ticket != (unsigned int)na - 1) continue;
+            reduce_up(T, na, 0, (uint64_t)na, s_root);
             continue;
         }
         // ------------------------------ verify item k ------------------------------
