@@ -1302,11 +1302,8 @@ static ckpt_status prepare_finish(const void *const *a, const void *const *b, co
     CK_CUDA(cudaGetDevice(&dev));
     std::memset(&fs.fp, 0, sizeof(fs.fp));
     const uint64_t n_tiles = (pp.n_pair + kTileTasks - 1) / kTileTasks;
-    // look-back states: [0, n_tiles) element ids (p.states), [n_tiles, 2 n_tiles) chunk positions
     CK_TRY(verify_setup(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps, idx,
-                        idx_cap, counts_dev + 1, s, 0, 0, &pp, kTileIdsFin, fs.fp.v, &fs.tab, &fs.max_chunks,
-                        n_tiles * (uint64_t)kTileIdsFin, 2 * n_tiles));
-    fs.fp.states_c = fs.fp.v.states + n_tiles;
+                        idx_cap, counts_dev + 1, s, 0, 0, &pp, kFinBlock, fs.fp.v, &fs.tab, &fs.max_chunks));
     unsigned long long *tickets = nullptr;
     {
         std::lock_guard<std::mutex> lk(g_scr_mu);
@@ -1344,7 +1341,7 @@ static ckpt_status launch_finish(ckpt_dtype dtype, cudaStream_t s, FinishStage &
         CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, kFinThreads, kFinSmem));
         occ[d].store(std::max(o, 1));
     }
-    const uint64_t work = (uint64_t)fs.fp.n_level + fs.fp.v.n_tiles;
+    const uint64_t work = (uint64_t)fs.fp.n_level + (fs.max_chunks + kFinBlock - 1) / kFinBlock;
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(work, (uint64_t)sms * occ[d].load()));
     {
         ProfScope prof(3, s);
@@ -1398,7 +1395,7 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     // gather pass
     const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
     const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
-    const bool finish = chunks_cap > 0 && !before_emit && !tile_gather_forced();
+    const bool finish = tiles_in_mark && !before_emit;
     if (!finish) pp.tdone = nullptr;          // tile flags: only for the finish kernel
     static FinishStage fs;                    // large (kernel parameters); one call at a time
     static std::mutex fs_mu;

@@ -13,15 +13,16 @@
 // complete: its CTAs take the SM slots K1's CTAs free during K1's tail (the last ~10% of K1,
 // where warps run out of tasks) and consume K1's tiles as they are published.
 //
-//  * tickets [0, n_tiles): verify item k = K1 tile k.  Wait for tdone[k]; mark the tile's
-//    flagged chunks (one warp per chunk: binary64 |a-b| > eps, R11; hit bits to the work
-//    buffer), scan their hit counts in the CTA, then a decoupled look-back over the preceding
-//    items gives both the tile's first chunk-list position and its first element-id position;
-//    write the chunk ids and the element ids (ascending, coalesced).
-//  * tickets [n_tiles, n_tiles + n_level): level groups of both trees, each after the K1
-//    tiles holding its leaves are published: 2048 leaves of one array per CTA reduced 11
-//    levels up (reduce.cuh: registers, shuffles, one barrier); the last group of an array
-//    builds the array's remaining levels, the last array of a tree the top tree (R15).
+//  * tickets [0, n_level): level groups of both trees, each after the K1 tiles holding its
+//    leaves are published: 2048 leaves of one array per CTA reduced 11 levels up (reduce.cuh);
+//    the last group of an array builds the array's remaining levels, the last array of a tree
+//    the top tree (R15).  These overlap K1's tail.
+//  * the following tickets: verify blocks of kFinBlock consecutive positions of the flagged
+//    chunk list, once every K1 tile is published (the list is K1's per-tile compaction,
+//    prefixed in shared memory).  A block marks its chunks (one warp per chunk: binary64
+//    |a-b| > eps, R11; hit bits to the work buffer), scans their hit counts, finds its output
+//    offset by a decoupled look-back over the preceding blocks and writes the element ids
+//    (ascending, coalesced) -- a single pass.
 //
 // Tickets are drawn in order by running CTAs and every wait is on work that K1 (resident from
 // its start) or an earlier ticket's CTA completes, so nothing waits on a CTA that cannot run.
@@ -38,20 +39,18 @@ namespace ckpt {
 
 constexpr int kFinThreads = kLevelThreads;         // 512 (the level groups' CTA shape)
 constexpr int kFinWarps = kFinThreads / 32;
-constexpr int kTileIdsFin = 4096;                  // chunk slots per K1 tile (kTileTasks * 32)
-// dynamic shared memory: per-chunk hit counts of a tile (16 KB) + per-warp emit scratch
-// (2 KB each), or the level groups' kLevelSmem
-constexpr size_t kFinSmemVerify = (size_t)kTileIdsFin * 4 + (size_t)kFinWarps * 2048;
-constexpr size_t kFinSmem = kFinSmemVerify > (size_t)kLevelSmem ? kFinSmemVerify : (size_t)kLevelSmem;
+constexpr int kFinBlock = kFinWarps;              // flagged chunks per verify block (a warp each)
+// dynamic shared memory: 2 x 512 nodes for the level blocks, or 2 KB of emit scratch per warp
+constexpr size_t kFinSmem = (size_t)kFinWarps * 2048 > (size_t)2 * kRedThreads * 16
+                                ? (size_t)kFinWarps * 2048 : (size_t)2 * kRedThreads * 16;
 
 struct FinishParams {
     LevelBatch lv;                // both trees' level groups (lv.cta_begin[lv.n] CTAs)
-    VerifyParams v;               // tagg / tids / n_tiles: K1's tiles; mask: per tile slot
+    VerifyParams v;               // tagg / tids / n_tiles: K1's tiles; mask: per list position
     unsigned long long *ticket;   // 0 on entry; the last draw resets it
     unsigned int n_level;         // level tickets
     const uint32_t *tdone;        // [n_tiles] K1's tile flags
     uint32_t tepoch;              // this pair compare's tag in tdone
-    uint64_t *states_c;           // look-back states of the chunk-list positions (p.states: element ids)
     unsigned int *lctr;           // [2 * na + 2] level arrivals per (tree, array), per tree; 0 between launches
 };
 
@@ -97,17 +96,25 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     constexpr int ESZ = DT == 0 ? 4 : 8;
     extern __shared__ __align__(16) uint4 fin_sm[];
-    __shared__ uint32_t s_w[kFinWarps];
+    __shared__ uint32_t s_tpre[kVerifyMaxTiles + 1];             // K1 tile prefix (list positions)
+    __shared__ uint32_t s_cnt[kFinBlock], s_len[kFinBlock];
+    __shared__ uint64_t s_gb[kFinBlock];
+    __shared__ const uint8_t *s_pa[kFinBlock], *s_pb[kFinBlock];
+    __shared__ uint32_t s_ex[kFinBlock], s_sum;
     __shared__ uint64_t s_t;
     __shared__ unsigned int s_ticket;
     const VerifyParams &p = P.v;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t n_tiles = p.n_tiles;
-    const uint64_t n_total = n_tiles + P.n_level;
-    for (uint64_t t = fin_draw(P.ticket, n_total, &s_t); t < n_total; t = fin_draw(P.ticket, n_total, &s_t)) {
-        if (t >= n_tiles) {
+    bool listed = false;                      // s_tpre holds the tile prefix
+    uint64_t n_list = 0, n_vb = 0;
+    for (;;) {
+        __syncthreads();                      // the previous item is done with shared memory
+        if (threadIdx.x == 0) s_t = atomicAdd(P.ticket, 1ull);
+        __syncthreads();
+        const uint64_t t = s_t;
+        if (t < P.n_level) {
             // ------------------------------ a level group ------------------------------
-            const unsigned int cta = (unsigned int)(t - n_tiles);
+            const unsigned int cta = (unsigned int)t;
             int ti = 0;
             while (ti + 1 < P.lv.n && cta >= P.lv.cta_begin[ti + 1]) ++ti;
             const LevelParams &lp = P.lv.t[ti];
@@ -120,8 +127,7 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
             // pair-tasks (32 chunks of one array each, array-major) holding the group's leaves
             uint64_t tb = 0;
             for (int k = 0; k < a; ++k) tb += (cnt0[k] + 31) / 32;
-            const uint64_t g = gid - gbegin[a];
-            const uint64_t c_lo = g * kGroup;
+            const uint64_t c_lo = (gid - gbegin[a]) * kGroup;
             const uint64_t c_hi = (c_lo + kGroup < cnt0[a] ? c_lo + kGroup : cnt0[a]) - 1;
             fin_wait_tiles(P, (tb + c_lo / 32) / kTileTasks, (tb + c_hi / 32) / kTileTasks);
             if (lp.inl >= 0 && gid == 0) {
@@ -136,13 +142,12 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
             T.height = reinterpret_cast<const uint32_t *>(mb + lp.o_h);
             T.top_off = lp.top_off;
             T.na = na;
-            uint4 *s_root = fin_sm;
             const int H = (int)T.height[a];
             if (H > 1)
-                reduce_block(T, a, 0, c_lo, (uint32_t)(c_hi + 1 - c_lo), H - 1 < kRedBlockLog ? H - 1 : kRedBlockLog, s_root);
+                reduce_block(T, a, 0, c_lo, (uint32_t)(c_hi + 1 - c_lo), H - 1 < kRedBlockLog ? H - 1 : kRedBlockLog, fin_sm);
             if (H - 1 > kRedBlockLog) {
                 // the last group of the array builds the array's remaining levels
-                const uint32_t n_g = (uint32_t)((cnt0[a] + kGroup - 1) / kGroup);     // the array's groups
+                const uint32_t n_g = (uint32_t)((cnt0[a] + kGroup - 1) / kGroup);
                 if (threadIdx.x == 0) {
                     unsigned int *c = P.lctr + (uint32_t)ti * (uint32_t)na + (uint32_t)a;
                     const unsigned int old = atom_add_acq_rel_u32(c, 1u);
@@ -151,7 +156,7 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
                 }
                 __syncthreads();
                 if (s_ticket != n_g - 1) continue;
-                reduce_up(T, a, kRedBlockLog, T.count(a, kRedBlockLog), s_root);
+                reduce_up(T, a, kRedBlockLog, T.count(a, kRedBlockLog), fin_sm);
             }
             // the array root is final: it is level-0 node a of the top tree; the last array
             // of the tree builds the top
@@ -164,79 +169,71 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
             }
             __syncthreads();
             if (s_ticket != (unsigned int)na - 1) continue;
-            reduce_up(T, na, 0, (uint64_t)na, s_root);
+            reduce_up(T, na, 0, (uint64_t)na, fin_sm);
             continue;
         }
-        // ------------------------------ verify item k ------------------------------
-        const uint64_t k = t;
-        fin_wait_tiles(P, k, k);
-        const uint32_t n = __ldcg(p.tagg + k);
-        uint32_t *s_cnt = reinterpret_cast<uint32_t *>(fin_sm);           // [kTileIdsFin]
-        const uint64_t *ids = p.tids + k * kTileIdsFin;
-        for (uint32_t j = warp; j < n; j += kFinWarps) {                  // mark: a warp per chunk
-            const uint64_t g = __ldcg(reinterpret_cast<const unsigned long long *>(ids) + j);
-            const uint8_t *pa, *pb;
-            uint64_t len, gb;
-            verify_locate_g(p, g, ESZ, pa, pb, len, gb);
-            const uint32_t c = mark_chunk<DT>(pa, pb, len, p.eps, p.mask + (k * kTileIdsFin + j) * p.groups * 32, lane);
-            if (lane == 0) s_cnt[j] = c;
-        }
-        __syncthreads();
-        // exclusive prefix of the hit counts over the tile's chunks (8 per thread)
-        constexpr int kPer = kTileIdsFin / kFinThreads;
-        uint32_t v[kPer], sum = 0;
-        const uint32_t j0 = threadIdx.x * kPer;
-#pragma unroll
-        for (int i = 0; i < kPer; ++i) {
-            v[i] = j0 + i < n ? s_cnt[j0 + i] : 0u;
-            sum += v[i];
-        }
-        uint32_t wtot;
-        uint32_t ex = warp_excl_scan_u32(sum, lane, wtot);
-        if (lane == 0) s_w[warp] = wtot;
-        __syncthreads();
-        uint32_t hits = 0;
-#pragma unroll
-        for (int w = 0; w < kFinWarps; ++w) {
-            const uint32_t x = s_w[w];
-            if (w < warp) ex += x;
-            hits += x;
-        }
-#pragma unroll
-        for (int i = 0; i < kPer; ++i) {
-            if (j0 + i < n) s_cnt[j0 + i] = ex;                // now: first hit of chunk j inside the tile
-            ex += v[i];
-        }
-        __syncthreads();
-        // the tile's place: chunk-list positions and element-id positions of all earlier tiles
-        const uint64_t excl_c = cta_lookback<kFinThreads>(P.states_c, k, n, p.epoch);
-        const uint64_t excl_h = cta_lookback<kFinThreads>(p.states, k, hits, p.epoch);
-        const uint64_t cap_c = p.chunks_cap;
-        if (threadIdx.x == 0) {
-            if (k == n_tiles - 1) {
-                *p.n_chunks_out = excl_c + n;
-                if (excl_c + n <= cap_c) *p.count = excl_h + hits;
+        // -------- verify: blocks of kFinBlock consecutive positions of the flagged list --------
+        if (!listed) {
+            // every tile published: the list is K1's per-tile compaction, prefixed here
+            fin_wait_tiles(P, 0, p.n_tiles - 1);
+            tile_prefix<kFinThreads>(p, s_tpre);
+            const uint64_t total = s_tpre[p.n_tiles];
+            n_list = total < p.chunks_cap ? total : p.chunks_cap;
+            n_vb = (n_list + kFinBlock - 1) / kFinBlock;
+            listed = true;
+            if (threadIdx.x == 0 && t == P.n_level) {
+                *p.n_chunks_out = total;
+                if (n_vb == 0) *p.count = 0;
             }
-            // the chunk-list capacity cuts this tile: the element ids are those of listed chunks
-            if (excl_c < cap_c && cap_c < excl_c + n) *p.count = excl_h + s_cnt[cap_c - excl_c];
         }
-        const uint32_t n_listed = excl_c >= cap_c ? 0u : (uint32_t)((cap_c - excl_c) < n ? (cap_c - excl_c) : n);
-        for (uint32_t j = threadIdx.x; j < n_listed; j += kFinThreads)
-            p.list_out[excl_c + j] = __ldcg(reinterpret_cast<const unsigned long long *>(ids) + j);
-        uint16_t *s_off = reinterpret_cast<uint16_t *>(reinterpret_cast<uint8_t *>(fin_sm) + kTileIdsFin * 4) + warp * 1024;
-        for (uint32_t j = warp; j < n_listed; j += kFinWarps) {           // ids: a warp per chunk
-            const uint32_t c0 = s_cnt[j];
-            const uint32_t c1 = j + 1 < n ? s_cnt[j + 1] : hits;
-            if (c1 == c0) continue;                                       // warp-uniform
-            const uint64_t g = __ldcg(reinterpret_cast<const unsigned long long *>(ids) + j);
-            const uint8_t *pa, *pb;
-            uint64_t len, gb;
-            verify_locate_g(p, g, ESZ, pa, pb, len, gb);
-            uint64_t pos = excl_h + c0;
-            const uint32_t groups = (uint32_t)((len + 1023) / 1024);
-            const uint32_t *mq = p.mask + (k * kTileIdsFin + j) * p.groups * 32 + lane;
+        if (t >= P.n_level + n_vb) {
+            // the last of the launch's final draws resets the ticket
+            if (threadIdx.x == 0 && t == P.n_level + n_vb + gridDim.x - 1) *P.ticket = 0ull;
+            break;
+        }
+        const uint64_t vb = t - P.n_level;
+        const uint64_t q0 = vb * kFinBlock;
+        const uint32_t nq = (uint32_t)((n_list - q0) < (uint64_t)kFinBlock ? (n_list - q0) : kFinBlock);
+        if (threadIdx.x < kFinBlock) {               // locate the block's chunks, one thread each
+            const uint32_t j = threadIdx.x;
+            const uint8_t *pa = nullptr, *pb = nullptr;
+            uint64_t len = 0, gb = 0;
+            if (j < nq) {
+                const uint64_t g = tile_chunk(p, s_tpre, q0 + j);
+                p.list_out[q0 + j] = g;
+                verify_locate_g(p, g, ESZ, pa, pb, len, gb);
+            }
+            s_pa[j] = pa;
+            s_pb[j] = pb;
+            s_len[j] = (uint32_t)len;
+            s_gb[j] = gb;
+        }
+        __syncthreads();
+        {                                             // mark: warp w takes position q0 + w
+            uint32_t c = 0;
+            if ((uint32_t)warp < nq)
+                c = mark_chunk<DT>(s_pa[warp], s_pb[warp], s_len[warp], p.eps,
+                                   p.mask + (q0 + warp) * p.groups * 32, lane);
+            if (lane == 0) s_cnt[warp] = c;
+        }
+        __syncthreads();
+        if (warp == 0) {                              // the block's exclusive prefix of hit counts
+            uint32_t tot;
+            const uint32_t ex = warp_excl_scan_u32(lane < kFinBlock ? s_cnt[lane] : 0u, lane, tot);
+            if (lane < kFinBlock) s_ex[lane] = ex;
+            if (lane == 0) s_sum = tot;
+        }
+        __syncthreads();
+        const uint64_t excl = cta_lookback<kFinThreads>(p.states, vb, s_sum, p.epoch);
+        if (threadIdx.x == 0 && vb == n_vb - 1) *p.count = excl + s_sum;
+        if ((uint32_t)warp < nq && s_cnt[warp]) {     // ids: warp w writes its chunk's
+            uint16_t *s_off = reinterpret_cast<uint16_t *>(fin_sm) + warp * 1024;
+            uint64_t pos = excl + s_ex[warp];
+            const uint32_t groups = (s_len[warp] + 1023) / 1024;
+            const uint32_t *mq = p.mask + (q0 + warp) * p.groups * 32 + lane;
             for (uint32_t gr = 0; gr < groups; ++gr)
-                pos += emit_words(__ldcs(mq + gr * 32), gb + (uint64_t)gr * 1024, pos, p.out, p.cap, lane, s_off);
+                pos += emit_words(__ldcs(mq + gr * 32), s_gb[warp] + (uint64_t)gr * 1024, pos, p.out, p.cap, lane,
+                                  s_off);
         }
     }
 }

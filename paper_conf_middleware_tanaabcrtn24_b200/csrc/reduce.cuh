@@ -1,18 +1,14 @@
-// reduce.cuh -- latency-first interior levels for the finish kernel (finish.cuh).
+// reduce.cuh -- interior levels for the finish kernel (finish.cuh).
 //
 // Alg. 1 lines 13-20, reading R13/R14: node j of level l+1 is
 // Murmur3F(node 2j || node 2j+1, 32 B, seed 0), or node 2j promoted when it has no right
 // sibling.  Any aligned block of 2^k nodes of a level is an exact subtree, so a CTA can reduce
 // a block of up to 2048 nodes to its root on its own.  The levels kernel (levels.cuh) does it in
 // passes of two levels through shared memory, which keeps lanes busy when there are many
-// groups; here the goal is the shortest dependent chain, since the finish kernel's level work
-// is small and sits at the end of the step:
-//   * registers: each of the 512 threads takes 4 consecutive nodes and hashes them two levels up
-//     (2 independent hashes, then 1);
-//   * warp shuffles: the 32 results of a warp go 5 levels up (lane-halving);
-//   * one barrier: the 16 warp results go the last 4 levels up in warp 0.
-// 11 dependent hash latencies and one __syncthreads per 2048-node block; every node produced is
-// stored at its place in the tree.
+// groups, and hands everything above the groups to one CTA; here a block is reduced the same
+// way (passes of two levels, whole warps busy) down to 32 nodes, warp 0 finishes with
+// shuffles, and the levels above the blocks are built by the last block of each array (then
+// of each tree), in parallel over arrays.  Every node produced is stored at its place.
 #pragma once
 #include <cstdint>
 
@@ -53,56 +49,63 @@ struct TreeRef {
 };
 
 // Levels l0+1 .. l0+kmax (kmax <= 11) of the block of m <= 2048 level-l0 nodes of array aa
-// starting at node s0 (s0 a multiple of 2^11); c_l = the block's node counts per level.
-// Called by all 512 threads; s_root: 16 nodes of shared memory.
+// starting at node s0 (s0 a multiple of 2^11).  Passes of two levels: the first ceil(c/4)
+// threads each take 4 consecutive nodes (2 independent hashes, then 1) -- whole warps busy --
+// until at most 32 nodes remain, which warp 0 takes the rest of the way with shuffles.
+// Called by all 512 threads; sm: 2 x 512 nodes of shared memory.
 __device__ __noinline__ void reduce_block(const TreeRef &T, int aa, int l0, uint64_t s0, uint32_t m,
-                                          int kmax, uint4 *s_root) {
+                                          int kmax, uint4 *sm) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    // the block's node count at relative level k
-    auto cnt = [&](int k) -> uint32_t { return (m + (1u << k) - 1) >> k; };
-    // ---- registers: levels 1 and 2 ----
-    uint4 x[4];
-    const uint32_t i0 = 4u * (uint32_t)tid;
-    const uint4 *src = T.at(aa, l0, s0);
+    uint4 *buf[2] = {sm, sm + kRedThreads};
+    int r = 0;                       // relative level of the current nodes
+    uint32_t c = m;                  // their count
+    while (r < kmax && (c > 32 || r == 0)) {
+        const int d = kmax - r >= 2 ? 2 : 1;
+        const uint32_t per = 1u << d;
+        const uint32_t need = (c + per - 1) >> d;
+        const uint4 *in = buf[(r >> 1) & 1];
+        uint4 *out = buf[((r >> 1) + 1) & 1];
+        if ((uint32_t)tid < need) {
+            const uint32_t i0 = per * (uint32_t)tid;
+            uint4 x[4];
 #pragma unroll
-    for (int q = 0; q < 4; ++q) x[q] = i0 + q < m ? __ldcg(src + i0 + q) : make_uint4(0u, 0u, 0u, 0u);
-    uint4 y0 = x[0], y1 = x[2];
-    const uint4 h0 = hash_children32(x[0], x[1]), h1 = hash_children32(x[2], x[3]);
-    if (i0 + 1 < m) y0 = h0;
-    if (i0 + 3 < m) y1 = h1;
-    uint4 z = y0;
-    if (kmax >= 1) {
-        uint4 *d = T.at(aa, l0 + 1, s0 >> 1);
-        if (2 * tid < cnt(1)) d[2 * tid] = y0;
-        if (2 * tid + 1 < cnt(1)) d[2 * tid + 1] = y1;
-    }
-    if (kmax >= 2) {
-        const uint4 hz = hash_children32(y0, y1);
-        if (2 * tid + 1 < cnt(1)) z = hz;
-        if ((uint32_t)tid < cnt(2)) T.at(aa, l0 + 2, s0 >> 2)[tid] = z;
-    }
-    // ---- warp shuffles: levels 3..7 (lane l holds level-2 node 32*warp + l) ----
-    for (int k = 3, step = 1; k <= 7 && k <= kmax; ++k, step <<= 1) {
-        const uint4 r = shfl_down4(z, step);
-        const uint32_t j = (32u * warp + lane) >> (k - 2);
-        if ((lane & (2 * step - 1)) == 0 && j < cnt(k)) {
-            if (2 * j + 1 < cnt(k - 1)) z = hash_children32(z, r);
-            T.at(aa, l0 + k, s0 >> k)[j] = z;
+            for (int q = 0; q < 4; ++q) {
+                x[q] = make_uint4(0u, 0u, 0u, 0u);
+                if (q < (int)per && i0 + q < c) x[q] = r == 0 ? __ldcg(T.at(aa, l0, s0) + i0 + q) : in[i0 + q];
+            }
+            const uint32_t c1 = (c + 1) >> 1;
+            uint4 y0 = x[0], y1 = x[2];
+            const uint4 h0 = hash_children32(x[0], x[1]);
+            if (i0 + 1 < c) y0 = h0;
+            uint4 *d1 = T.at(aa, l0 + r + 1, s0 >> (r + 1));
+            d1[i0 >> 1] = y0;
+            if (d == 2) {
+                const uint4 h1 = hash_children32(x[2], x[3]);
+                if (i0 + 3 < c) y1 = h1;
+                if ((i0 >> 1) + 1 < c1) d1[(i0 >> 1) + 1] = y1;
+                uint4 z = y0;
+                const uint4 hz = hash_children32(y0, y1);
+                if ((i0 >> 1) + 1 < c1) z = hz;
+                T.at(aa, l0 + r + 2, s0 >> (r + 2))[tid] = z;
+                out[tid] = z;
+            } else {
+                out[tid] = y0;
+            }
         }
-    }
-    // ---- one barrier: levels 8..11 in warp 0 (lane w holds warp w's level-7 node) ----
-    if (kmax >= 8) {
-        if (lane == 0) s_root[warp] = z;
+        r += d;
+        c = need;
         __syncthreads();
-        if (warp == 0) {
-            uint4 w = lane < 16 ? s_root[lane] : make_uint4(0u, 0u, 0u, 0u);
-            for (int k = 8, step = 1; k <= kmax; ++k, step <<= 1) {
-                const uint4 r = shfl_down4(w, step);
-                const uint32_t j = (uint32_t)lane >> (k - 7);
-                if ((lane & (2 * step - 1)) == 0 && j < cnt(k)) {
-                    if (2 * j + 1 < cnt(k - 1)) w = hash_children32(w, r);
-                    T.at(aa, l0 + k, s0 >> k)[j] = w;
-                }
+    }
+    if (r < kmax && warp == 0) {
+        // c <= 32 nodes of relative level r in buf: lane l holds node l
+        uint4 z = (uint32_t)lane < c ? buf[(r >> 1) & 1][lane] : make_uint4(0u, 0u, 0u, 0u);
+        for (int k = r + 1, step = 1; k <= kmax; ++k, step <<= 1) {
+            const uint4 rr = shfl_down4(z, step);
+            const uint32_t j = (uint32_t)lane >> (k - r);
+            const uint32_t cp = (m + (1u << (k - 1)) - 1) >> (k - 1);     // nodes at level k-1
+            if ((lane & (2 * step - 1)) == 0 && j < ((cp + 1) >> 1)) {
+                if (2 * j + 1 < cp) z = hash_children32(z, rr);
+                T.at(aa, l0 + k, s0 >> k)[j] = z;
             }
         }
     }
