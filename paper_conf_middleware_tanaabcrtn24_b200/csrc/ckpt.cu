@@ -1324,7 +1324,9 @@ static ckpt_status prepare_finish(const void *const *a, const void *const *b, co
         fs.fp.lctr = sc.lctr;
     }
     CK_TRY(fill_level_batch(trees, 2, s, tickets, fs.fp.lv));
-    fs.fp.n_level = fs.fp.lv.cta_begin[fs.fp.lv.n];
+    uint64_t nlev = 0;
+    for (uint32_t k = 0; k < n_arrays; ++k) nlev += (trees[0]->n_leaves[k] + kFinGroup - 1) / kFinGroup;
+    fs.fp.n_level = (unsigned int)(2 * nlev);
     fs.fp.ticket = tickets + 24;              // slots 1..4: level trees, 16: K1
     fs.fp.tdone = pp.tdone;
     fs.fp.tepoch = pp.tepoch;

@@ -37,9 +37,11 @@
 
 namespace ckpt {
 
-constexpr int kFinThreads = kLevelThreads;         // 512 (the level groups' CTA shape)
+constexpr int kFinThreads = kRedThreads;           // 128: fits beside K1's CTAs as they retire
 constexpr int kFinWarps = kFinThreads / 32;
-constexpr int kFinBlock = kFinWarps;              // flagged chunks per verify block (a warp each)
+constexpr uint64_t kFinGroup = 1u << kRedBlockLog;  // leaves per level item
+constexpr int kFinPerWarp = 4;                     // flagged chunks per warp and verify block
+constexpr int kFinBlock = kFinWarps * kFinPerWarp; // 16
 // dynamic shared memory: 2 x 512 nodes for the level blocks, or 2 KB of emit scratch per warp
 constexpr size_t kFinSmem = (size_t)kFinWarps * 2048 > (size_t)2 * kRedThreads * 16
                                 ? (size_t)kFinWarps * 2048 : (size_t)2 * kRedThreads * 16;
@@ -90,7 +92,7 @@ __device__ __forceinline__ void fin_wait_tiles(const FinishParams &P, uint64_t l
 }
 
 template <int DT>
-__global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_constant__ FinishParams P) {
+__global__ void __launch_bounds__(kFinThreads, 8) finish_kernel(const __grid_constant__ FinishParams P) {
     // no griddepcontrol.wait: this grid runs while K1 still does (see above); its successor
     // waits for it as usual
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -114,23 +116,28 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
         const uint64_t t = s_t;
         if (t < P.n_level) {
             // ------------------------------ a level group ------------------------------
-            const unsigned int cta = (unsigned int)t;
-            int ti = 0;
-            while (ti + 1 < P.lv.n && cta >= P.lv.cta_begin[ti + 1]) ++ti;
+            // both trees have the same shape: the first half of the level tickets is run A's
+            const unsigned int half = P.n_level / 2;
+            const int ti = t >= half ? 1 : 0;
+            uint64_t gid = ti ? t - half : t;
             const LevelParams &lp = P.lv.t[ti];
             const uint8_t *mb = lp.inl >= 0 ? reinterpret_cast<const uint8_t *>(P.lv.blob + lp.inl) : lp.meta;
-            const uint64_t *gbegin = reinterpret_cast<const uint64_t *>(mb + lp.o_g);
             const uint64_t *cnt0 = reinterpret_cast<const uint64_t *>(mb + lp.o_cnt);   // level 0
             const int na = lp.n_arrays;
-            const uint64_t gid = cta - P.lv.cta_begin[ti];
-            const int a = find_le(gbegin, na, gid);
-            // pair-tasks (32 chunks of one array each, array-major) holding the group's leaves
+            // the array of group gid (blocks of kFinGroup leaves, arrays in order), and the
+            // pair-tasks (32 chunks of one array each, array-major) before it
+            int a = 0;
             uint64_t tb = 0;
-            for (int k = 0; k < a; ++k) tb += (cnt0[k] + 31) / 32;
-            const uint64_t c_lo = (gid - gbegin[a]) * kGroup;
-            const uint64_t c_hi = (c_lo + kGroup < cnt0[a] ? c_lo + kGroup : cnt0[a]) - 1;
+            for (;; ++a) {
+                const uint64_t ng = (cnt0[a] + kFinGroup - 1) / kFinGroup;
+                if (gid < ng || a == na - 1) break;
+                gid -= ng;
+                tb += (cnt0[a] + 31) / 32;
+            }
+            const uint64_t c_lo = gid * kFinGroup;
+            const uint64_t c_hi = (c_lo + kFinGroup < cnt0[a] ? c_lo + kFinGroup : cnt0[a]) - 1;
             fin_wait_tiles(P, (tb + c_lo / 32) / kTileTasks, (tb + c_hi / 32) / kTileTasks);
-            if (lp.inl >= 0 && gid == 0) {
+            if (lp.inl >= 0 && a == 0 && gid == 0) {
                 // publish the inline tables to device memory for later BFS launches
                 uint64_t *dst = reinterpret_cast<uint64_t *>(lp.meta);
                 for (uint32_t w = threadIdx.x; w < lp.meta_words; w += kFinThreads) dst[w] = P.lv.blob[lp.inl + w];
@@ -147,7 +154,7 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
                 reduce_block(T, a, 0, c_lo, (uint32_t)(c_hi + 1 - c_lo), H - 1 < kRedBlockLog ? H - 1 : kRedBlockLog, fin_sm);
             if (H - 1 > kRedBlockLog) {
                 // the last group of the array builds the array's remaining levels
-                const uint32_t n_g = (uint32_t)((cnt0[a] + kGroup - 1) / kGroup);
+                const uint32_t n_g = (uint32_t)((cnt0[a] + kFinGroup - 1) / kFinGroup);
                 if (threadIdx.x == 0) {
                     unsigned int *c = P.lctr + (uint32_t)ti * (uint32_t)na + (uint32_t)a;
                     const unsigned int old = atom_add_acq_rel_u32(c, 1u);
@@ -209,12 +216,12 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
             s_gb[j] = gb;
         }
         __syncthreads();
-        {                                             // mark: warp w takes position q0 + w
+        for (int k = 0; k < kFinPerWarp; ++k) {      // mark: warp w takes positions w, w+4, ...
+            const uint32_t j = (uint32_t)(warp + kFinWarps * k);
             uint32_t c = 0;
-            if ((uint32_t)warp < nq)
-                c = mark_chunk<DT>(s_pa[warp], s_pb[warp], s_len[warp], p.eps,
-                                   p.mask + (q0 + warp) * p.groups * 32, lane);
-            if (lane == 0) s_cnt[warp] = c;
+            if (j < nq)
+                c = mark_chunk<DT>(s_pa[j], s_pb[j], s_len[j], p.eps, p.mask + (q0 + j) * p.groups * 32, lane);
+            if (lane == 0) s_cnt[j] = c;
         }
         __syncthreads();
         if (warp == 0) {                              // the block's exclusive prefix of hit counts
@@ -226,13 +233,15 @@ __global__ void __launch_bounds__(kFinThreads, 2) finish_kernel(const __grid_con
         __syncthreads();
         const uint64_t excl = cta_lookback<kFinThreads>(p.states, vb, s_sum, p.epoch);
         if (threadIdx.x == 0 && vb == n_vb - 1) *p.count = excl + s_sum;
-        if ((uint32_t)warp < nq && s_cnt[warp]) {     // ids: warp w writes its chunk's
+        for (int k = 0; k < kFinPerWarp; ++k) {      // ids: warp w writes its chunks'
+            const uint32_t j = (uint32_t)(warp + kFinWarps * k);
+            if (j >= nq || s_cnt[j] == 0) continue;   // warp-uniform
             uint16_t *s_off = reinterpret_cast<uint16_t *>(fin_sm) + warp * 1024;
-            uint64_t pos = excl + s_ex[warp];
-            const uint32_t groups = (s_len[warp] + 1023) / 1024;
-            const uint32_t *mq = p.mask + (q0 + warp) * p.groups * 32 + lane;
+            uint64_t pos = excl + s_ex[j];
+            const uint32_t groups = (s_len[j] + 1023) / 1024;
+            const uint32_t *mq = p.mask + (q0 + j) * p.groups * 32 + lane;
             for (uint32_t gr = 0; gr < groups; ++gr)
-                pos += emit_words(__ldcs(mq + gr * 32), s_gb[warp] + (uint64_t)gr * 1024, pos, p.out, p.cap, lane,
+                pos += emit_words(__ldcs(mq + gr * 32), s_gb[j] + (uint64_t)gr * 1024, pos, p.out, p.cap, lane,
                                   s_off);
         }
     }

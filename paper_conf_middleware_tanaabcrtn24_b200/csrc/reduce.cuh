@@ -3,7 +3,7 @@
 // Alg. 1 lines 13-20, reading R13/R14: node j of level l+1 is
 // Murmur3F(node 2j || node 2j+1, 32 B, seed 0), or node 2j promoted when it has no right
 // sibling.  Any aligned block of 2^k nodes of a level is an exact subtree, so a CTA can reduce
-// a block of up to 2048 nodes to its root on its own.  The levels kernel (levels.cuh) does it in
+// a block of up to 512 nodes to its root on its own.  The levels kernel (levels.cuh) does it in
 // passes of two levels through shared memory, which keeps lanes busy when there are many
 // groups, and hands everything above the groups to one CTA; here a block is reduced the same
 // way (passes of two levels, whole warps busy) down to 32 nodes, warp 0 finishes with
@@ -17,8 +17,8 @@
 
 namespace ckpt {
 
-constexpr int kRedBlockLog = 11;                 // nodes per block: 2^11 = 512 threads x 4
-constexpr int kRedThreads = 512;
+constexpr int kRedThreads = 128;                 // the finish kernel's CTA
+constexpr int kRedBlockLog = 9;                  // nodes per block: 2^9 = 128 threads x 4
 
 // A tree's addressing: array levels from the metadata tables, the top tree over the array
 // roots (array index na) after them, level-ordered.
@@ -48,15 +48,20 @@ struct TreeRef {
     }
 };
 
-// Levels l0+1 .. l0+kmax (kmax <= 11) of the block of m <= 2048 level-l0 nodes of array aa
-// starting at node s0 (s0 a multiple of 2^11).  Passes of two levels: the first ceil(c/4)
+// Levels l0+1 .. l0+kmax (kmax <= 9) of the block of m <= 512 level-l0 nodes of array aa
+// starting at node s0 (s0 a multiple of 2^9).  Passes of two levels: the first ceil(c/4)
 // threads each take 4 consecutive nodes (2 independent hashes, then 1) -- whole warps busy --
 // until at most 32 nodes remain, which warp 0 takes the rest of the way with shuffles.
-// Called by all 512 threads; sm: 2 x 512 nodes of shared memory.
+// Called by all kRedThreads threads; sm: 2 x kRedThreads nodes of shared memory.
 __device__ __noinline__ void reduce_block(const TreeRef &T, int aa, int l0, uint64_t s0, uint32_t m,
                                           int kmax, uint4 *sm) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     uint4 *buf[2] = {sm, sm + kRedThreads};
+    // the block's start node on each level l0 .. l0+kmax, once (the tables live in the kernel
+    // parameters or global memory; every node store below addresses through shared memory)
+    __shared__ uint4 *s_lv[kRedBlockLog + 1];
+    if (tid <= kmax) s_lv[tid] = T.at(aa, l0 + tid, s0 >> tid);
+    __syncthreads();
     int r = 0;                       // relative level of the current nodes
     uint32_t c = m;                  // their count
     while (r < kmax && (c > 32 || r == 0)) {
@@ -71,13 +76,13 @@ __device__ __noinline__ void reduce_block(const TreeRef &T, int aa, int l0, uint
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 x[q] = make_uint4(0u, 0u, 0u, 0u);
-                if (q < (int)per && i0 + q < c) x[q] = r == 0 ? __ldcg(T.at(aa, l0, s0) + i0 + q) : in[i0 + q];
+                if (q < (int)per && i0 + q < c) x[q] = r == 0 ? __ldcg(s_lv[0] + i0 + q) : in[i0 + q];
             }
             const uint32_t c1 = (c + 1) >> 1;
             uint4 y0 = x[0], y1 = x[2];
             const uint4 h0 = hash_children32(x[0], x[1]);
             if (i0 + 1 < c) y0 = h0;
-            uint4 *d1 = T.at(aa, l0 + r + 1, s0 >> (r + 1));
+            uint4 *d1 = s_lv[r + 1];
             d1[i0 >> 1] = y0;
             if (d == 2) {
                 const uint4 h1 = hash_children32(x[2], x[3]);
@@ -86,7 +91,7 @@ __device__ __noinline__ void reduce_block(const TreeRef &T, int aa, int l0, uint
                 uint4 z = y0;
                 const uint4 hz = hash_children32(y0, y1);
                 if ((i0 >> 1) + 1 < c1) z = hz;
-                T.at(aa, l0 + r + 2, s0 >> (r + 2))[tid] = z;
+                s_lv[r + 2][tid] = z;
                 out[tid] = z;
             } else {
                 out[tid] = y0;
@@ -105,7 +110,7 @@ __device__ __noinline__ void reduce_block(const TreeRef &T, int aa, int l0, uint
             const uint32_t cp = (m + (1u << (k - 1)) - 1) >> (k - 1);     // nodes at level k-1
             if ((lane & (2 * step - 1)) == 0 && j < ((cp + 1) >> 1)) {
                 if (2 * j + 1 < cp) z = hash_children32(z, rr);
-                T.at(aa, l0 + k, s0 >> k)[j] = z;
+                s_lv[k][j] = z;
             }
         }
     }

@@ -35,6 +35,7 @@ for sep in (False, True):
     lib.ckpt_debug_fin_trace(buf)
     tr = np.frombuffer(buf, dtype=np.uint64).reshape(-1, 2)
     n_tiles = (L // 32 + 127) // 128
+    n_level = 2 * sum(-(-(t.numel() * 4 // 4096) // 512) for t in A)
     used = tr[:, 0] > 0
     t0 = tr[used, 0].min()
     tt = (tr[:, 0].astype(np.int64) - int(t0)) / 1e3
@@ -54,8 +55,8 @@ for sep in (False, True):
             durs.append((last[c][0], tt[i] - last[c][1]))
         last[c] = (i, tt[i])
     d = np.array(durs)
-    ver = d[d[:, 0] < n_tiles]
-    lev = d[d[:, 0] >= n_tiles]
+    lev = d[d[:, 0] < n_level]
+    ver = d[d[:, 0] >= n_level]
     for name, x in (("verify", ver), ("level", lev)):
         if len(x):
             print(f"  {name:6s} items {len(x):4d}: duration us mean {x[:, 1].mean():6.1f} p50 {np.median(x[:, 1]):6.1f} max {x[:, 1].max():6.1f}")
