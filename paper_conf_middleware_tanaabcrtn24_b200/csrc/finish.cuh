@@ -74,20 +74,28 @@ __device__ __forceinline__ uint64_t fin_draw(unsigned long long *ticket, uint64_
     return *s_t;
 }
 
-// Thread 0 waits (acquire, growing sleep) until K1 published tiles [lo, hi]; then a barrier.
+// Wait until K1 published tiles [lo, hi]: the CTA's threads poll the flags in parallel with
+// relaxed loads (a sequential acquire per tile would cost one L2 round trip each), then one
+// acquire fence orders everything the flags published before this CTA's reads.
 __device__ __forceinline__ void fin_wait_tiles(const FinishParams &P, uint64_t lo, uint64_t hi) {
-    if (threadIdx.x == 0) {
-        unsigned int nap = 64;
-        for (uint64_t k = lo; k <= hi; ++k) {
-            for (;;) {
-                uint32_t v;
-                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.tdone + k) : "memory");
-                if (v == P.tepoch) break;
-                __nanosleep(nap);
-                nap = nap < 2048u ? 2u * nap : 2048u;
-            }
+    __shared__ int s_pending;
+    unsigned int nap = 64;
+    for (;;) {
+        int mine = 0;
+        for (uint64_t k = lo + threadIdx.x; k <= hi; k += blockDim.x) {
+            uint32_t v;
+            asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.tdone + k) : "memory");
+            mine |= v != P.tepoch;
         }
+        if (threadIdx.x == 0) s_pending = 0;
+        __syncthreads();
+        if (mine) s_pending = 1;
+        __syncthreads();
+        if (!s_pending) break;
+        __nanosleep(nap);
+        nap = nap < 2048u ? 2u * nap : 2048u;
     }
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
     __syncthreads();
 }
 
