@@ -26,7 +26,6 @@
 #include "hash.cuh"
 #include "leaf.cuh"
 #include "levels.cuh"
-#include "finish.cuh"
 
 using namespace ckpt;
 
@@ -424,48 +423,6 @@ static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms, 
 static ckpt_status get_scratch(int dev, cudaStream_t s, size_t n_states, uint64_t **states,
                                unsigned long long **ticket, uint32_t *epoch);
 
-// The launch record of up to kMaxLevelTrees trees' level groups (tree metadata inline in
-// the parameters when it fits, else staged to each tree's device blob).
-static ckpt_status fill_level_batch(ckpt_tree *const *trees, int n, cudaStream_t s,
-                                    unsigned long long *tickets, LevelBatch &b) {
-    std::memset(&b, 0, offsetof(LevelBatch, blob));
-    b.n = n;
-    unsigned ctas = 0;
-    uint32_t words = 0;
-    for (int i = 0; i < b.n; ++i) {
-        ckpt_tree *t = trees[i];
-        LevelParams &p = b.t[i];
-        p.nodes = t->nodes;
-        p.meta = t->meta;
-        p.meta_words = (uint32_t)t->meta_host.size();
-        if (words + p.meta_words <= (uint32_t)kLevelInlineWords) {
-            std::memcpy(b.blob + words, t->meta_host.data(), (size_t)p.meta_words * 8);
-            p.inl = (int)words;
-            words += p.meta_words;
-        } else {
-            p.inl = -1;
-            CK_TRY(g_ring.copy(t->meta, t->meta_host.data(), t->meta_host.size() * 8, s));
-        }
-        p.o_off = t->o_off;
-        p.o_cnt = t->o_cnt;
-        p.o_lb = t->o_lb;
-        p.o_lt = t->o_lt;
-        p.o_h = t->o_h;
-        p.o_g = t->o_g;
-        p.o_cb = t->o_cb;
-        p.top_off = t->top_off;
-        p.ticket = reinterpret_cast<unsigned int *>(tickets + 1 + i);   // slot 0: compactions
-        p.n_arrays = (int)t->n_arrays;
-        p.n_levels = (int)t->n_levels;
-        p.ls = 0;
-        p.n_groups = (unsigned)t->n_groups;
-        b.cta_begin[i] = ctas;
-        ctas += (unsigned)t->n_groups;
-    }
-    b.cta_begin[b.n] = ctas;
-    return CKPT_OK;
-}
-
 static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s) {
     static std::atomic<int> attr_done{0};
     if (!attr_done.load()) {
@@ -482,9 +439,42 @@ static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s)
     static std::mutex b_mu;
     std::lock_guard<std::mutex> lk(b_mu);
     for (int k0 = 0; k0 < n; k0 += kMaxLevelTrees) {
-        CK_TRY(fill_level_batch(trees + k0, std::min(kMaxLevelTrees, n - k0), s, tickets, b));
+        std::memset(&b, 0, offsetof(LevelBatch, blob));
+        b.n = std::min(kMaxLevelTrees, n - k0);
+        unsigned ctas = 0;
+        uint32_t words = 0;
+        for (int i = 0; i < b.n; ++i) {
+            ckpt_tree *t = trees[k0 + i];
+            LevelParams &p = b.t[i];
+            p.nodes = t->nodes;
+            p.meta = t->meta;
+            p.meta_words = (uint32_t)t->meta_host.size();
+            if (words + p.meta_words <= (uint32_t)kLevelInlineWords) {
+                std::memcpy(b.blob + words, t->meta_host.data(), (size_t)p.meta_words * 8);
+                p.inl = (int)words;
+                words += p.meta_words;
+            } else {
+                p.inl = -1;
+                CK_TRY(g_ring.copy(t->meta, t->meta_host.data(), t->meta_host.size() * 8, s));
+            }
+            p.o_off = t->o_off;
+            p.o_cnt = t->o_cnt;
+            p.o_lb = t->o_lb;
+            p.o_lt = t->o_lt;
+            p.o_h = t->o_h;
+            p.o_g = t->o_g;
+            p.top_off = t->top_off;
+            p.ticket = reinterpret_cast<unsigned int *>(tickets + 1 + i);   // slot 0: compactions
+            p.n_arrays = (int)t->n_arrays;
+            p.n_levels = (int)t->n_levels;
+            p.ls = 0;
+            p.n_groups = (unsigned)t->n_groups;
+            b.cta_begin[i] = ctas;
+            ctas += (unsigned)t->n_groups;
+        }
+        b.cta_begin[b.n] = ctas;
         ProfScope prof(1, s);
-        CK_CUDA(launch_k(levels_kernel, dim3(b.cta_begin[b.n]), dim3(kLevelThreads), kLevelSmem, s, b));
+        CK_CUDA(launch_k(levels_kernel, dim3(ctas), dim3(kLevelThreads), kLevelSmem, s, b));
         CK_LAUNCH();
     }
     return CKPT_OK;
@@ -582,9 +572,6 @@ struct Scratch {
     size_t flags_cap = 0;
     uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
     size_t tile_pairs = 0;              // pair-tasks the buffers hold
-    uint32_t tepoch = 0;                // tag of the last fused compare's tile flags
-    unsigned int *lctr = nullptr;       // finish kernel level arrivals (zeroed once, self-resetting)
-    size_t lctr_cap = 0;
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -621,33 +608,29 @@ static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, Pa
     std::lock_guard<std::mutex> lk(g_scr_mu);
     Scratch &sc = g_scr[std::make_pair(dev, s)];
     n_pair = std::max<uint64_t>(n_pair, 1);
-    // [tctr: n_tiles u32][tdone: n_tiles u32] (zeroed once) [tagg][tmask][tbase][tids]
-    auto layout_of = [](uint64_t np, size_t o[6]) {
+    auto layout_of = [](uint64_t np, size_t o[5]) {
         const uint64_t nt = (np + kTileTasks - 1) / kTileTasks;
         o[0] = 0;
         o[1] = align256(nt * 4);
         o[2] = o[1] + align256(nt * 4);
-        o[3] = o[2] + align256(nt * 4);
-        o[4] = o[3] + align256(np * 4);
-        o[5] = o[4] + align256(np * 8);
-        return o[5] + nt * kTileTasks * 32 * 8;
+        o[3] = o[2] + align256(np * 4);
+        o[4] = o[3] + align256(np * 8);
+        return o[4] + nt * kTileTasks * 32 * 8;
     };
-    size_t o[6];
+    size_t o[5];
     if (sc.tile_pairs < n_pair) {
         if (sc.tile) CK_CUDA(cudaFreeAsync(sc.tile, s));
         sc.tile_pairs = std::max<uint64_t>(n_pair, 2 * sc.tile_pairs);
         const size_t bytes = layout_of(sc.tile_pairs, o);
         CK_CUDA(cudaMallocAsync((void **)&sc.tile, bytes, s));
-        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[2], s));      // tile counters and flags
-        sc.tepoch = 0;
+        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters
     }
     layout_of(sc.tile_pairs, o);
     pp->tctr = (unsigned int *)(sc.tile + o[0]);
-    pp->tdone = (uint32_t *)(sc.tile + o[1]);
-    pp->tagg = (uint32_t *)(sc.tile + o[2]);
-    pp->tmask = (uint32_t *)(sc.tile + o[3]);
-    pp->tbase = (uint64_t *)(sc.tile + o[4]);
-    pp->tids = (uint64_t *)(sc.tile + o[5]);
+    pp->tagg = (uint32_t *)(sc.tile + o[1]);
+    pp->tmask = (uint32_t *)(sc.tile + o[2]);
+    pp->tbase = (uint64_t *)(sc.tile + o[3]);
+    pp->tids = (uint64_t *)(sc.tile + o[4]);
     return CKPT_OK;
 }
 
@@ -672,8 +655,7 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
                                     const uint32_t *arrays_per_tree, uint32_t n_trees,
                                     ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
                                     uint32_t hash_block, void *stream, ckpt_tree **out,
-                                    const PairParams *pair, bool defer_levels = false,
-                                    const std::function<ckpt_status(ckpt_tree **, PairParams *)> &pre_launch = nullptr) {
+                                    const PairParams *pair) {
     if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
     for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
     if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
@@ -742,13 +724,10 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
         st = get_scratch(dev, s, 0, &unused_states, &ticket, &unused_epoch);
         ticket += kLeafTicketSlot;
     }
-    // work the caller stages between the trees' creation and the leaf launch (host->device
-    // copies must precede K1: a copy node after it would end the overlap with K1's tail)
-    if (st == CKPT_OK && pre_launch) st = pre_launch(out, pair ? &pp : nullptr);
     if (st == CKPT_OK)
         st = launch_leaves(table, task, dtype, eps, chunk_bytes, hash_block, s, di.sms,
                            pair ? &pp : nullptr, ticket);
-    if (st == CKPT_OK && !defer_levels) {
+    if (st == CKPT_OK) {
         // K2 on the side stream, after the leaves; each tree records its own event
         cudaStream_t ss = nullptr;
         cudaEvent_t leaves_done = nullptr;
@@ -943,7 +922,7 @@ static void release_scratch(int dev, cudaStream_t s) {
     auto it = g_scr.find(std::make_pair(dev, s));
     if (it == g_scr.end()) return;
     Scratch &sc = it->second;
-    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile, sc.lctr};
+    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile};
     for (void *b : bufs)
         if (b) cudaFreeAsync(b, s);
     g_scr.erase(it);
@@ -1114,17 +1093,6 @@ extern "C" ckpt_status ckpt_tree_diff(const ckpt_tree *a, const ckpt_tree *b, ui
 // it may replace the output buffer and its capacity (exact-size outputs).
 using EmitHook = std::function<ckpt_status(uint64_t **idx, uint64_t *cap)>;
 
-// The verify parameters, table and scratch for `max_tiles` look-back tiles of `tile`
-// list positions (the finish kernel's tiles; the scan kernel's otherwise).
-static ckpt_status verify_setup(const void *const *a, const void *const *b, const uint64_t *n,
-                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
-                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
-                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
-                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
-                                uint64_t chunk_base0, uint64_t elem_base0, const PairParams *tiles,
-                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out,
-                                uint64_t mask_slots = 0, uint64_t n_states = 0);
-
 static ckpt_status verify_impl(const void *const *a, const void *const *b, const uint64_t *n,
                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
@@ -1132,63 +1100,8 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
                                const EmitHook &before_emit = nullptr, uint64_t chunk_base0 = 0,
                                uint64_t elem_base0 = 0, const PairParams *tiles = nullptr) {
-    if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
-    VerifyParams p;
-    uint8_t *tab = nullptr;
-    uint64_t max_chunks = 0;
-    CK_TRY(verify_setup(a, b, n, na, dtype, chunk_bytes, chunks, n_chunks_dev, n_chunks_host, chunks_cap,
-                        eps, idx, cap, n_diff_dev, s, chunk_base0, elem_base0, tiles, kVerifyScanTile, p,
-                        &tab, &max_chunks));
-    int dev;
-    DevInfo di;
-    CK_TRY(dev_info(&dev, &di));
-    static std::atomic<int> occ[5] = {{0}, {0}, {0}, {0}, {0}};
-    const int d = dtype == CKPT_F32 ? 0 : 1;
-    if (occ[d].load() == 0) {
-        int m = 0, e = 0, sc = 0;
-        if (d == 0) {
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<0>, kVerifyThreads, 0));
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<0>, kVerifyThreads, 0));
-        } else {
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<1>, kVerifyThreads, 0));
-            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<1>, kVerifyThreads, 0));
-        }
-        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sc, verify_scan_kernel, kVerifyThreads, 0));
-        occ[4].store(std::max(sc, 1));
-        occ[2 + d].store(std::max(e, 1));
-        occ[d].store(std::max(m, 1));
-    }
-    const uint64_t warp_ctas = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
-    const unsigned g_mark = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[d].load()));
-    const unsigned g_emit = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[2 + d].load()));
-    // co-resident grid (the look-back relies on it); tiles are strided statically
-    const uint64_t max_tiles = (max_chunks + kVerifyScanTile - 1) / kVerifyScanTile;
-    const unsigned g_scan = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * occ[4].load()));
-    {
-        ProfScope prof(3, s);
-        CK_CUDA(launch_k(d == 0 ? verify_mark_kernel<0> : verify_mark_kernel<1>, dim3(g_mark),
-                         dim3(kVerifyThreads), 0, s, p));
-        CK_LAUNCH();
-        CK_CUDA(launch_k(verify_scan_kernel, dim3(g_scan), dim3(kVerifyThreads), 0, s, p));
-        CK_LAUNCH();
-        if (before_emit) CK_TRY(before_emit(&p.out, &p.cap));
-        CK_CUDA(launch_k(d == 0 ? verify_emit_kernel<0> : verify_emit_kernel<1>, dim3(g_emit),
-                         dim3(kVerifyThreads), 0, s, p));
-    }
-    CK_LAUNCH();
-    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
-    return CKPT_OK;
-}
-
-static ckpt_status verify_setup(const void *const *a, const void *const *b, const uint64_t *n,
-                                uint32_t na, ckpt_dtype dtype, uint32_t chunk_bytes,
-                                const uint64_t *chunks, const uint64_t *n_chunks_dev,
-                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
-                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
-                                uint64_t chunk_base0, uint64_t elem_base0, const PairParams *tiles,
-                                uint64_t tile, VerifyParams &p, uint8_t **tab_out, uint64_t *max_chunks_out,
-                                uint64_t mask_slots, uint64_t n_states) {
     if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
+    if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
     const uint64_t esz = dtype == CKPT_F32 ? 4 : 8;
     std::vector<VerifyArray> va(na);
@@ -1213,6 +1126,7 @@ static ckpt_status verify_setup(const void *const *a, const void *const *b, cons
     DevInfo di;
     CK_TRY(dev_info(&dev, &di));
     const uint64_t max_chunks = std::min<uint64_t>(chunks_cap, c - chunk_base0);
+    VerifyParams p;
     std::memset(&p, 0, sizeof(p));
     uint8_t *tab = nullptr;
     if (na <= (uint32_t)kVerifyInline) {
@@ -1248,19 +1162,50 @@ static ckpt_status verify_setup(const void *const *a, const void *const *b, cons
         p.list_out = const_cast<uint64_t *>(chunks);
         p.n_chunks_out = const_cast<uint64_t *>(n_chunks_dev);
     }
-    const uint64_t max_tiles = n_states ? n_states : (max_chunks + tile - 1) / tile;
+    static std::atomic<int> occ[5] = {{0}, {0}, {0}, {0}, {0}};
+    const int d = dtype == CKPT_F32 ? 0 : 1;
+    if (occ[d].load() == 0) {
+        int m = 0, e = 0, sc = 0;
+        if (d == 0) {
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<0>, kVerifyThreads, 0));
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<0>, kVerifyThreads, 0));
+        } else {
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&m, verify_mark_kernel<1>, kVerifyThreads, 0));
+            CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&e, verify_emit_kernel<1>, kVerifyThreads, 0));
+        }
+        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&sc, verify_scan_kernel, kVerifyThreads, 0));
+        occ[4].store(std::max(sc, 1));
+        occ[2 + d].store(std::max(e, 1));
+        occ[d].store(std::max(m, 1));
+    }
+    const uint64_t warp_ctas = (max_chunks + kVerifyWarps - 1) / kVerifyWarps;
+    const unsigned g_mark = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[d].load()));
+    const unsigned g_emit = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(warp_ctas, (uint64_t)di.sms * occ[2 + d].load()));
+    // co-resident grid (the look-back relies on it); tiles are strided statically
+    const uint64_t max_tiles = (max_chunks + kVerifyScanTile - 1) / kVerifyScanTile;
+    const unsigned g_scan = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(max_tiles, (uint64_t)di.sms * occ[4].load()));
     unsigned long long *ticket_unused = nullptr;
     CK_TRY(get_scratch(dev, s, max_tiles, &p.states, &ticket_unused, &p.epoch));
     const size_t o_off = align256((size_t)max_chunks * 4);
     const size_t o_mask = o_off + align256((size_t)max_chunks * 8);
     uint8_t *work = nullptr;
-    const uint64_t slots = mask_slots ? mask_slots : max_chunks;
-    CK_TRY(get_work(dev, s, o_mask + (size_t)slots * p.groups * 128, &work));
+    CK_TRY(get_work(dev, s, o_mask + (size_t)max_chunks * p.groups * 128, &work));
     p.cnt = (uint32_t *)work;
     p.off = (uint64_t *)(work + o_off);
     p.mask = (uint32_t *)(work + o_mask);
-    *tab_out = tab;
-    *max_chunks_out = max_chunks;
+    {
+        ProfScope prof(3, s);
+        CK_CUDA(launch_k(d == 0 ? verify_mark_kernel<0> : verify_mark_kernel<1>, dim3(g_mark),
+                         dim3(kVerifyThreads), 0, s, p));
+        CK_LAUNCH();
+        CK_CUDA(launch_k(verify_scan_kernel, dim3(g_scan), dim3(kVerifyThreads), 0, s, p));
+        CK_LAUNCH();
+        if (before_emit) CK_TRY(before_emit(&p.out, &p.cap));
+        CK_CUDA(launch_k(d == 0 ? verify_emit_kernel<0> : verify_emit_kernel<1>, dim3(g_emit),
+                         dim3(kVerifyThreads), 0, s, p));
+    }
+    CK_LAUNCH();
+    if (tab) CK_CUDA(cudaFreeAsync(tab, s));
     return CKPT_OK;
 }
 
@@ -1284,76 +1229,6 @@ extern "C" ckpt_status ckpt_diff_verify_async(const ckpt_tree *ta, const ckpt_tr
 // fused pair compare: K1 in pair mode (digest compare and
 // element marking in-kernel), then the ordered chunk list and the element ids
 // ---------------------------------------------------------------------------
-// K5 (finish.cuh): both trees' level groups and the verify items over K1's tiles, launched
-// right after K1 and running alongside its tail.  prepare_finish runs before K1 is launched
-// (its table copies must not sit between the two kernels), launch_finish after.
-struct FinishStage {
-    FinishParams fp;
-    uint8_t *tab = nullptr;
-    uint64_t max_chunks = 0;
-};
-
-static ckpt_status prepare_finish(const void *const *a, const void *const *b, const uint64_t *n,
-                                  uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
-                                  uint64_t *chunks, uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
-                                  uint64_t *counts_dev, cudaStream_t s, ckpt_tree *const *trees,
-                                  PairParams &pp, FinishStage &fs) {
-    int dev = 0;
-    CK_CUDA(cudaGetDevice(&dev));
-    std::memset(&fs.fp, 0, sizeof(fs.fp));
-    const uint64_t n_tiles = (pp.n_pair + kTileTasks - 1) / kTileTasks;
-    CK_TRY(verify_setup(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps, idx,
-                        idx_cap, counts_dev + 1, s, 0, 0, &pp, kFinBlock, fs.fp.v, &fs.tab, &fs.max_chunks));
-    unsigned long long *tickets = nullptr;
-    {
-        std::lock_guard<std::mutex> lk(g_scr_mu);
-        Scratch &sc = g_scr[std::make_pair(dev, s)];
-        tickets = sc.ticket;                  // allocated by verify_setup's get_scratch
-        if (++sc.tepoch == 0) {               // epoch wrap: clear the tile flags once
-            CK_CUDA(cudaMemsetAsync(pp.tdone, 0, n_tiles * 4, s));
-            sc.tepoch = 1;
-        }
-        pp.tepoch = sc.tepoch;
-        const size_t need = 2 * (size_t)n_arrays + 2;
-        if (sc.lctr_cap < need) {
-            if (sc.lctr) CK_CUDA(cudaFreeAsync(sc.lctr, s));
-            sc.lctr_cap = std::max(need, 2 * sc.lctr_cap);
-            CK_CUDA(cudaMallocAsync((void **)&sc.lctr, sc.lctr_cap * 4, s));
-            CK_CUDA(cudaMemsetAsync(sc.lctr, 0, sc.lctr_cap * 4, s));
-        }
-        fs.fp.lctr = sc.lctr;
-    }
-    CK_TRY(fill_level_batch(trees, 2, s, tickets, fs.fp.lv));
-    uint64_t nlev = 0;
-    for (uint32_t k = 0; k < n_arrays; ++k) nlev += (trees[0]->n_leaves[k] + kFinGroup - 1) / kFinGroup;
-    fs.fp.n_level = (unsigned int)(2 * nlev);
-    fs.fp.ticket = tickets + 24;              // slots 1..4: level trees, 16: K1
-    fs.fp.tdone = pp.tdone;
-    fs.fp.tepoch = pp.tepoch;
-    return CKPT_OK;
-}
-
-static ckpt_status launch_finish(ckpt_dtype dtype, cudaStream_t s, FinishStage &fs, int sms) {
-    const int d = dtype == CKPT_F32 ? 0 : 1;
-    auto kern = d == 0 ? finish_kernel<0> : finish_kernel<1>;
-    static std::atomic<int> occ[2] = {{0}, {0}};
-    if (occ[d].load() == 0) {
-        int o = 0;
-        CK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFinSmem));
-        CK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, kFinThreads, kFinSmem));
-        occ[d].store(std::max(o, 1));
-    }
-    const uint64_t work = (uint64_t)fs.fp.n_level + (fs.max_chunks + kFinBlock - 1) / kFinBlock;
-    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(work, (uint64_t)sms * occ[d].load()));
-    {
-        ProfScope prof(3, s);
-        CK_CUDA(launch_k(kern, dim3(grid), dim3(kFinThreads), kFinSmem, s, fs.fp));
-    }
-    CK_LAUNCH();
-    if (fs.tab) CK_CUDA(cudaFreeAsync(fs.tab, s));
-    return CKPT_OK;
-}
-
 static ckpt_status compare_pair_impl(const void *const *a, const void *const *b, const uint64_t *n,
                                      uint32_t n_arrays, ckpt_dtype dtype, uint32_t chunk_bytes,
                                      double eps, uint32_t hash_block, uint64_t *chunks,
@@ -1392,39 +1267,14 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     }
     const uint32_t apt[2] = {n_arrays, n_arrays};
     ckpt_tree *trees[2] = {nullptr, nullptr};
-    // the ordered chunk list from K1's per-tile compaction: read directly by the finish kernel
-    // (or, with an exact-size output hook, K4a) up to kVerifyMaxTiles tiles, else placed by one
-    // gather pass
+    CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
+                            trees, &pp));
+    // the ordered chunk list from K1's per-tile compaction: read by K4a directly (up to
+    // kVerifyMaxTiles tiles), else placed by one gather pass
+    ckpt_status st = CKPT_OK;
     const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
     const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
-    const bool finish = tiles_in_mark && !before_emit;
-    if (!finish) pp.tdone = nullptr;          // tile flags: only for the finish kernel
-    static FinishStage fs;                    // large (kernel parameters); one call at a time
-    static std::mutex fs_mu;
-    std::unique_lock<std::mutex> fs_lk(fs_mu, std::defer_lock);
-    std::function<ckpt_status(ckpt_tree **, PairParams *)> pre = nullptr;
-    if (finish) {
-        fs_lk.lock();
-        pre = [&](ckpt_tree **tt, PairParams *kp) -> ckpt_status {
-            return prepare_finish(a, b, n, n_arrays, dtype, chunk_bytes, eps, chunks, chunks_cap, idx,
-                                  idx_cap, counts_dev, s, tt, *kp, fs);
-        };
-    }
-    CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
-                            trees, &pp, finish, pre));
-    ckpt_status st = CKPT_OK;
     pp.n_pair = n_pair;
-    if (finish) {
-        st = launch_finish(dtype, s, fs, di.sms);
-        if (st != CKPT_OK) {
-            ckpt_tree_free_on(trees[0], stream);
-            ckpt_tree_free_on(trees[1], stream);
-            return st;
-        }
-        *out_a = trees[0];
-        *out_b = trees[1];
-        return CKPT_OK;
-    }
     if (!tiles_in_mark) {
         TileGatherParams g;
         g.tagg = pp.tagg;

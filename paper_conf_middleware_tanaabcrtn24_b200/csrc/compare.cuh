@@ -430,12 +430,10 @@ __device__ __forceinline__ void verify_locate(const VerifyParams &p, uint64_t q,
 }
 
 // Tile mode: exclusive prefix of the tile counts into s_tpre[0..n_tiles]
-// (s_tpre[n_tiles] = total).  Called by all NT threads of the CTA.
-template <int NT = kVerifyThreads>
+// (s_tpre[n_tiles] = total).  Called by all threads of the CTA.
 __device__ __forceinline__ void tile_prefix(const VerifyParams &p, uint32_t *s_tpre) {
-    constexpr int NW = NT / 32;
-    __shared__ uint32_t s_w[NW];
-    constexpr int kPer = kVerifyMaxTiles / NT;
+    __shared__ uint32_t s_w[kVerifyWarps];
+    constexpr int kPer = kVerifyMaxTiles / kVerifyThreads;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t nt = p.n_tiles;
     const uint32_t t0 = threadIdx.x * kPer;
@@ -450,13 +448,13 @@ __device__ __forceinline__ void tile_prefix(const VerifyParams &p, uint32_t *s_t
     if (lane == 0) s_w[warp] = wt;
     __syncthreads();
 #pragma unroll
-    for (int w = 0; w < NW; ++w) ex += w < warp ? s_w[w] : 0u;
+    for (int w = 0; w < kVerifyWarps; ++w) ex += w < warp ? s_w[w] : 0u;
 #pragma unroll
     for (int k = 0; k < kPer; ++k) {
         if (t0 + k <= nt) s_tpre[t0 + k] = ex;
         ex += v[k];
     }
-    if (threadIdx.x == NT - 1 && nt == kVerifyMaxTiles) s_tpre[nt] = ex;
+    if (threadIdx.x == kVerifyThreads - 1 && nt == kVerifyMaxTiles) s_tpre[nt] = ex;
     __syncthreads();
 }
 

@@ -231,8 +231,6 @@ struct PairParams {
     unsigned int *tctr;           // [n_tiles] 0 between launches
     uint32_t *tagg;               // [n_tiles] flagged chunks per tile
     uint64_t *tids;               // [n_tiles * kTileTasks * 32] tile-compacted chunk ids
-    uint32_t *tdone;              // [n_tiles] = tepoch once the tile is compacted (release), or null
-    uint32_t tepoch;              // this launch's tag (never 0; the buffer is never cleared)
 };
 
 // The tile's ordered chunk ids, by the warp that completed its last pair-task
@@ -261,13 +259,7 @@ __device__ __noinline__ void tile_compact(const PairParams &pr, uint64_t tile, i
         for (uint32_t mm = m; mm; mm &= mm - 1) dst[pos++] = b + (uint64_t)(__ffs(mm) - 1);
         run += tot;
     }
-    if (lane == 0) {
-        pr.tagg[tile] = run;
-        // the tile is final: its ids and count, and (through the pair hand-offs this warp
-        // acquired) both runs' leaves of its chunks, for a consumer running alongside K1
-        if (pr.tdone)
-            asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(pr.tdone + tile), "r"(pr.tepoch) : "memory");
-    }
+    if (lane == 0) pr.tagg[tile] = run;
 }
 
 struct LeafParams {

@@ -47,7 +47,6 @@ struct LevelParams {
     uint32_t o_lt;                // u64 [level]: nodes in level (all arrays)
     uint32_t o_h;                 // u32 [a]: number of levels of array a
     uint32_t o_g;                 // u64 [a]: first group of array a
-    uint32_t o_cb;                // u64 [a]: global chunk id of array a's leaf 0
     uint64_t top_off;             // node index of the top tree's level 0
     unsigned int *ticket;         // zero on entry, reset to zero by the last CTA
     int n_arrays;
@@ -128,14 +127,13 @@ __device__ __forceinline__ void build_level(const LvView &p, int l, const uint4 
 }
 
 
-// The work of level CTA `cta` (0 .. cta_begin[n]-1) of a batch: phase 1 for its group,
-// phase 2 if it is the last of its tree.  Called by all kLevelThreads threads of a CTA;
-// `sm` = kLevelSmem bytes of shared memory, s_ticket a shared word.
-__device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int cta, uint4 *sm,
-                                        unsigned int &s_ticket) {
+__global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_constant__ LevelBatch pb) {
+    pdl_enter();
+    extern __shared__ __align__(16) uint4 sm[];
+    __shared__ unsigned int s_ticket;
     const int tid = threadIdx.x;
     int ti = 0;
-    while (ti + 1 < pb.n && cta >= pb.cta_begin[ti + 1]) ++ti;
+    while (ti + 1 < pb.n && blockIdx.x >= pb.cta_begin[ti + 1]) ++ti;
     const LevelParams &lp = pb.t[ti];
     const uint8_t *mb = lp.inl >= 0 ? reinterpret_cast<const uint8_t *>(pb.blob + lp.inl) : lp.meta;
     LvView p;
@@ -153,7 +151,7 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
     p.ls = lp.ls;
     p.n_groups = lp.n_groups;
     const int na = p.n_arrays;
-    if (lp.inl >= 0 && cta == pb.cta_begin[ti]) {
+    if (lp.inl >= 0 && blockIdx.x == pb.cta_begin[ti]) {
         // publish the inline tables to device memory for later BFS launches
         uint64_t *dst = reinterpret_cast<uint64_t *>(lp.meta);
         for (uint32_t w = tid; w < lp.meta_words; w += kLevelThreads) dst[w] = pb.blob[lp.inl + w];
@@ -167,7 +165,7 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
         // Every pass but the last few keeps whole warps busy, so the CTA's
         // 2047 hashes cost ~2047/32 warp-hashes instead of a lane-halving
         // shuffle tree, and 16 warps per CTA hide the hash latency.
-        const uint64_t gid = cta - pb.cta_begin[ti];
+        const uint64_t gid = blockIdx.x - pb.cta_begin[ti];
         const int a = find_le(p.gbegin, na, gid);
         const uint64_t g = gid - p.gbegin[a];
         const uint64_t n0 = p.cnt[(uint64_t)p.ls * na + a];
@@ -195,8 +193,8 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
                         uint4 *l2 = p.nodes + p.off[(uint64_t)(p.ls + r + 2) * na + a] + (start >> (r + 2));
                         uint4 x0, x1, x2, x3;
                         if (r == 0) {
-                            x0 = __ldcg(src + 4 * tid); x1 = __ldcg(src + 4 * tid + 1);
-                            x2 = __ldcg(src + 4 * tid + 2); x3 = __ldcg(src + 4 * tid + 3);
+                            x0 = __ldg(src + 4 * tid); x1 = __ldg(src + 4 * tid + 1);
+                            x2 = __ldg(src + 4 * tid + 2); x3 = __ldg(src + 4 * tid + 3);
                         } else {
                             x0 = in[4 * tid]; x1 = in[4 * tid + 1]; x2 = in[4 * tid + 2]; x3 = in[4 * tid + 3];
                         }
@@ -230,7 +228,7 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
                     x[j] = make_uint4(0u, 0u, 0u, 0u);
-                    if (j < mt) x[j] = r == 0 ? __ldcg(src + per * tid + j) : in[per * tid + j];
+                    if (j < mt) x[j] = r == 0 ? __ldg(src + per * tid + j) : in[per * tid + j];
                 }
                 const uint4 y0 = mt >= 2 ? hash_children32(x[0], x[1]) : x[0];
                 write(r + 1, (uint64_t)(per / 2) * tid, y0);
@@ -339,13 +337,6 @@ __device__ __forceinline__ void levels_cta(const LevelBatch &pb, unsigned int ct
         n = up;
     }
     if (tid == 0) *p.ticket = 0u;
-}
-
-__global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_constant__ LevelBatch pb) {
-    pdl_enter();
-    extern __shared__ __align__(16) uint4 sm[];
-    __shared__ unsigned int s_ticket;
-    levels_cta(pb, blockIdx.x, sm, s_ticket);
 }
 
 }  // namespace ckpt

@@ -601,9 +601,9 @@ def test_compare_pair_identical_and_truncated():
         ck.compare_pair_async(a, [b[0]], 4096, 1e-6, chunks, idx, counts)
 
 
-# K1 tile compaction (128 pair-tasks = 4096 chunks per tile) + in-kernel marking +
-# pair_emit_kernel: ragged arrays (pair-tasks of < 32 chunks), several tiles with
-# a ragged last one, every chunk flagged (every marking job queued at once), no
+# K1 tile compaction (128 pair-tasks = 4096 chunks per tile) read by verify_mark
+# (and, past 4096 tiles, placed by tile_gather_kernel): ragged arrays (pair-tasks
+# of < 32 chunks), several tiles with a ragged last one, every chunk flagged, no
 # chunk flagged, and a chunk-list cap that cuts through a tile -- all against the
 # plain leaf comparison and brute force.
 @pytest.mark.parametrize("mode", ["all", "none", "sparse", "cap"])
@@ -654,10 +654,24 @@ def test_compare_pair_tile_compaction(mode):
     assert np.array_equal(np_of(idx[:nd]), ref_idx)
 
 
+def test_compare_pair_tile_gather_path():
+    """The gather kernel (used past 4096 tiles) in a fresh process with CKPT_TILE_GATHER=1."""
+    import subprocess
+    import sys
+    code = (
+        "import sys; sys.path.insert(0, %r); import test_gpu_parity as t; "
+        "[t.test_compare_pair_tile_compaction(m) for m in ('all', 'none', 'sparse', 'cap')]; print('ok')"
+        % os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, CKPT_TILE_GATHER="1")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stdout[-2000:] + r.stderr[-2000:]
+
+
 @pytest.mark.parametrize("dt,chunk", [(torch.float32, 2 << 20), (torch.float64, 4 << 20)])
-def test_compare_pair_fallback_path_large_chunks(dt, chunk):
-    """Chunks above 1 MiB take the fallback of the fused call (flags-only leaf kernel, levels
-    kernel, flag compaction, verify kernels): same results as the oracle."""
+def test_compare_pair_large_chunks(dt, chunk):
+    """Multi-MiB chunks (several mask groups per chunk, few long chains) through the fused call:
+    every node, the chunk list and the element ids equal the oracle's."""
     sizes = [3 * chunk // 8 + 5, chunk // 16, 2 * chunk // 4 + 1]
     a = [_data(n, dt, 300 + i) for i, n in enumerate(sizes)]
     b = [t.clone() for t in a]
@@ -669,8 +683,8 @@ def test_compare_pair_fallback_path_large_chunks(dt, chunk):
 
 
 def test_compare_pair_repeated_and_alternating_shapes():
-    """The in-kernel counters, job queue and tile state return to zero after every launch: many
-    compares on one stream, alternating between shapes (per-shape table cache), all exact."""
+    """The self-resetting pair-task and tile counters and the epoch-tagged look-back states stay
+    consistent over many compares on one stream, alternating between shapes: all exact."""
     p1 = synth.c1_pair(n=(1 << 19) + 3, seed=61, device="cuda")
     p2 = synth.c5_pair(n_ranks=1, n_particles=(1 << 15), seed=62, device="cuda")
     ref = {}
