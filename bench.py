@@ -374,8 +374,8 @@ def run_ours(args):
         torch.cuda.synchronize()
         local_counts = counts.cpu().tolist()
         # timed region: no events between the kernels (an event after the leaf kernel would end
-        # the finish kernel's overlap with its tail); the leaf kernel's own duration is timed in
-        # a separate pass below
+        # the programmatic-launch overlap of the next kernel with its tail); the leaf kernel's
+        # own duration is timed in a separate pass below
         l0 = ck.launch_count()
         if collect:
             dist.barrier()
@@ -430,8 +430,7 @@ def run_ours(args):
         phases[k] = {"ms_per_step": round(pms / k_prof, 4), "launches": pn}
     if phases["diff"]["launches"] == 0:
         phases["diff"]["note"] = ("fused path: the leaf-level diff and its ordered compaction run inside "
-                                  "the leaf kernel (per tile); levels and verify are the finish kernel "
-                                  "(timed here without its overlap with the leaf kernel's tail)")
+                                  "the leaf kernel (per tile), the chunk list is written by verify_mark")
     ck.profile_reset()
     # side reference K5: "Direct" on the device -- verify with every chunk
     # flagged, i.e. 2S bytes compared element-wise with no hashing and no tree
