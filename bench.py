@@ -409,9 +409,9 @@ def run_ours(args):
         ck.profile_reset()
         if len(snaps) > 1:
             # all trees kept, without references to this snapshot's arrays
-            for t in keep:
-                if isinstance(t, ck.Tree):
-                    t.detach_inputs()
+            for tr in keep:
+                if isinstance(tr, ck.Tree):
+                    tr.detach_inputs()
             kept_trees.append(list(keep))
             per_snap.append({"snapshot": snap, "ms": round(float(t.item()), 4),
                              "flagged_chunks_per_gpu": local_counts[0],
