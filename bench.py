@@ -458,12 +458,16 @@ def run_ours(args):
     peak, peak_src = peaks()
     achieved = leaf_bytes / leaf_avg_s / 1e9
     traffic = None
+    traffic_src = None
     tp = os.path.join(ROOT, "profiles", "leaf_traffic.json")
     # the stored capture is of the default workload's pair launch (c2, 4 KiB, 16-byte blocks)
     same = CFG == "c2" and CHUNK == 4096 and args.hash_block == 16 and args.path != "saved"
     if same and os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+            tj = json.load(open(tp))
+            traffic = tj.get("dram_bytes_per_launch")
+            traffic_src = ("stored ncu --set full capture (profiles/leaf_traffic.json, commit "
+                           f"{tj.get('captured_at_commit', '?')}), not measured in this run")
         except Exception:
             traffic = None
 
@@ -530,9 +534,12 @@ def run_ours(args):
             "roofline": {"bound": "hbm", "kernel": "leaf_kernel (K1: quantize + chained Murmur3F)",
                          "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "traffic_source": traffic_src,
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_launch": leaf_bytes,
-                         "avg_launch_ms": round(leaf_avg_s * 1e3, 4)},
+                         "avg_launch_ms": round(leaf_avg_s * 1e3, 4),
+                         "timing": "CUDA events around every leaf launch of a second pass of the same "
+                                   "K steps (events in the timed pass would end the launch overlap)"},
             "phases_profiled_pass": phases, "host_enqueue_ms_per_step": round(host_ms, 4),
             "flagged_chunks_per_gpu": local_counts[0], "diff_elems_per_gpu": local_counts[1],
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
