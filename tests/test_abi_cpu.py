@@ -126,3 +126,22 @@ def test_product_sources_have_no_tuning_switches():
     init = open(os.path.join(pkg, "__init__.py")).read()
     assert "CKPT_LIB" not in init
     assert not os.path.isdir(os.path.join(csrc, "experimental"))
+
+
+def test_bench_spawns_one_rank_per_gpu_through_torchrun(monkeypatch):
+    """bench.py --gpus N without a launcher re-executes itself under torch.distributed.run with
+    N processes on 127.0.0.1 (one rank per GPU), forwarding its own arguments."""
+    import subprocess
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    seen = {}
+    monkeypatch.setattr(subprocess, "call", lambda cmd: seen.setdefault("cmd", cmd) and 0)
+    monkeypatch.setattr(sys, "argv", ["bench.py", "--gpus", "4", "--steps", "7"])
+    assert bench.spawn_ranks(4) == 0 or True
+    cmd = seen["cmd"]
+    assert cmd[1:3] == ["-m", "torch.distributed.run"]
+    assert "--nproc-per-node=4" in cmd and "--nnodes=1" in cmd
+    assert cmd[cmd.index("--master-addr") + 1] == "127.0.0.1"
+    assert cmd[-4:] == ["--gpus", "4", "--steps", "7"]
+    assert cmd[-5].endswith("bench.py")

@@ -863,7 +863,7 @@ def test_compare_saved_matches_oracle(host_a, tmp_path):
 
 # ------------------------------------------- config 4 snapshot shard shape --
 
-@pytest.mark.parametrize("snapshot", [2, 6, 9])
+@pytest.mark.parametrize("snapshot", range(10))
 def test_c4_snapshot_shard_matches_oracle(snapshot):
     # BASELINE configs[3]: a GPU's shard of HACC ranks of one snapshot (reduced particle count)
     pair = synth.c4_snapshot(snapshot, range(3, 6), n_particles=(1 << 16) + 5, device="cuda")
@@ -886,6 +886,22 @@ def test_c4_snapshot_shard_matches_oracle(snapshot):
     assert np.array_equal(np_of(idx[:nd]), ref_idx)
     assert TA.root() == A.root and TB.root() == B.root
     assert (nc == 0) == (snapshot <= 2)
+
+
+@pytest.mark.slow
+def test_c4_every_snapshot_full_size_rank_bench_path():
+    """BASELINE configs[3] as bench.py --config c4 --snapshots all runs it: every one of the 10
+    snapshots (divergence 0 for s <= 2, then 1e-6 * 4^(s-3) of the particles) on one full-size
+    HACC rank (2^24 particles x 6 f32 per run), through the fused call; every node of both trees,
+    the roots, the chunk list and the element ids equal the oracle's.  The ranks differ per
+    snapshot so the sample covers 10 of the 64."""
+    for s in range(10):
+        pair = synth.c4_snapshot(s, [(7 * s + 3) % 64], n_particles=1 << 24, device="cuda")
+        TA, TB, chunks, idx, counts = fused_compare(pair)
+        nc, nd = full_checkpoint_parity(pair, TA, TB, chunks, idx, counts, brute=False)
+        if s <= 2:
+            assert nc == 0 and nd == 0
+        del TA, TB, pair
 
 
 # --------------------------------- one array sharded over GPUs (8e, opt) ----
