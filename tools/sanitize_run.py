@@ -64,4 +64,20 @@ cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
 TA, TB = ck.compare_pair_async(p5.a, p5.b, C, p5.eps, ch, ix, cnt)
 TA.wait(); TB.wait()
 torch.cuda.synchronize()
+# a flagged short last chunk of 64 KiB chunks after a fully differing compare on the same stream
+# (the verify work buffer holds all-ones masks; emit must read only the groups the chunk has)
+n7 = 70_001
+a7 = synth.uniform(17, n7, "cuda") * 2.0 - 1.0
+L7 = -(-n7 * 4 // 65536)
+ch = torch.empty(L7, dtype=torch.int64, device="cuda")
+ix = torch.empty(n7, dtype=torch.int64, device="cuda")
+cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+TA, TB = ck.compare_pair_async([a7], [a7 + 1.0], 65536, 1e-6, ch, ix, cnt)
+TA.wait(); TB.wait()
+b7 = a7.clone()
+b7[-1] += 1.0
+TA, TB = ck.compare_pair_async([a7], [b7], 65536, 1e-6, ch, ix, cnt)
+TA.wait(); TB.wait()
+torch.cuda.synchronize()
+assert cnt.tolist() == [1, 1] and ix[0].item() == n7 - 1
 print("sanitize workload ok", ck.launch_count(), "launches")
