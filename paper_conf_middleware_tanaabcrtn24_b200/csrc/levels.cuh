@@ -30,6 +30,7 @@ constexpr int kLevelSmem = kLevelSmemNodes * 16;
 constexpr int kMaxLevelTrees = 4;
 
 constexpr int kLevelInlineWords = 512;   // 4 KiB of tree metadata in the kernel params
+constexpr int kLevelTabWords = 512;      // phase 2: level tables staged in shared memory
 
 // Per-tree launch record.  The metadata tables live in one blob (layout below)
 // that is either inline in the kernel parameters (small trees: no H2D copy;
@@ -173,8 +174,14 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
         const int m0 = (int)((n0 - start) < (uint64_t)kGroup ? (n0 - start) : (uint64_t)kGroup);
         const int h = (int)p.height[a];
         const uint4 *src = p.nodes + p.off[(uint64_t)p.ls * na + a] + start;
+        // the group's first node on each of its levels, formed once (threads 0..kLog in
+        // parallel): the level tables are not re-read on the dependent path of the passes
+        __shared__ uint4 *s_lvb[kLog + 1];
+        if (tid <= kLog && p.ls + tid < h)
+            s_lvb[tid] = p.nodes + p.off[(uint64_t)(p.ls + tid) * na + a] + (start >> tid);
+        __syncthreads();
         auto write = [&](int k, uint64_t j, uint4 v) {
-            if (p.ls + k < h) p.nodes[p.off[(uint64_t)(p.ls + k) * na + a] + (start >> k) + j] = v;
+            if (p.ls + k < h) s_lvb[k][j] = v;
         };
         uint4 *buf[2] = {sm, sm + kLevelThreads};       // ping-pong: 512 + 128 nodes
         int cnt = m0;
@@ -188,9 +195,9 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
                 const uint4 *in = buf[(r >> 1) & 1];
                 uint4 *out = buf[((r >> 1) + 1) & 1];
                 if (tid < need) {
-                    uint4 *l1 = p.nodes + p.off[(uint64_t)(p.ls + r + 1) * na + a] + (start >> (r + 1));
+                    uint4 *l1 = s_lvb[r + 1];
                     if (two) {
-                        uint4 *l2 = p.nodes + p.off[(uint64_t)(p.ls + r + 2) * na + a] + (start >> (r + 2));
+                        uint4 *l2 = s_lvb[r + 2];
                         uint4 x0, x1, x2, x3;
                         if (r == 0) {
                             x0 = __ldg(src + 4 * tid); x1 = __ldg(src + 4 * tid + 1);
@@ -263,6 +270,28 @@ __global__ void __launch_bounds__(kLevelThreads, 3) levels_kernel(const __grid_c
     }
     __syncthreads();
     if (s_ticket != p.n_groups - 1) return;
+    {
+        // the last CTA walks the level tables for every node it builds: stage them in shared
+        // memory when they fit (a few KB for a handful of arrays)
+        __shared__ uint64_t s_tab[kLevelTabWords];
+        const uint32_t nl = (uint32_t)p.n_levels;
+        const uint32_t nt = nl * (uint32_t)na;
+        if (2 * nt + 2 * (nl + 1) <= (uint32_t)kLevelTabWords) {
+            for (uint32_t i = tid; i < nt; i += kLevelThreads) {
+                s_tab[i] = p.off[i];
+                s_tab[nt + i] = p.cnt[i];
+            }
+            for (uint32_t i = tid; i <= nl; i += kLevelThreads) {
+                s_tab[2 * nt + i] = p.level_base[i];
+                s_tab[2 * nt + nl + 1 + i] = p.level_total[i];
+            }
+            __syncthreads();
+            p.off = s_tab;
+            p.cnt = s_tab + nt;
+            p.level_base = s_tab + 2 * nt;
+            p.level_total = s_tab + 2 * nt + nl + 1;
+        }
+    }
     int F = p.ls + kLog;                       // highest level phase 1 completed
     if (F > p.n_levels - 1) F = p.n_levels - 1;
     if (F + 1 <= p.n_levels - 1) {

@@ -40,6 +40,6 @@ p1 = (tr[used, 1] - tr[used, 0]) / 1e3
 end1 = (tr[used, 1] - t0) / 1e3
 last = tr[used, 2]
 print(f"{n} CTAs; start p0/p50/p100 {np.percentile(start, [0, 50, 100]).round(1)} us")
-print(f"phase-1 duration p0/p50/p90/p100 {np.percentile(p1, [0, 50, 90, 100]).round(1)} us; phase-1 ends by {end1.max():.1f} us")
+print(f"phase1 duration p0/p50/p90/p100 {np.percentile(p1, [0, 50, 90, 100]).round(1)} us; phase-1 ends by {end1.max():.1f} us")
 for i in np.nonzero(last > 0)[0]:
     print(f"  last CTA {i}: phase 2 {(last[i] - tr[used][i, 1]) / 1e3:.1f} us, ends at {(last[i] - t0) / 1e3:.1f} us")
