@@ -1,7 +1,8 @@
 #!/usr/bin/env python
 """Per-kernel timeline of bench steps (events around every library launch).
 
-usage: step_timeline.py [N_STEPS] [--unfused]   (default: the fused pair path bench.py times)"""
+usage: step_timeline.py [N_STEPS] [--unfused] [--c5]   (default: the fused pair path bench.py times,
+on c2; --c5: the configs[4] per-GPU shard)"""
 import os
 import sys
 
@@ -11,7 +12,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_middleware_tanaabcrtn24_b200 as ck  # noqa: E402
 import synth  # noqa: E402
 
-pair = synth.c2_pair(device="cuda")
+pair = synth.c5_pair(device="cuda") if "--c5" in sys.argv else synth.c2_pair(device="cuda")
 A, B = pair.a, pair.b
 L = sum(t.numel() * 4 // 4096 for t in A)
 chunks = torch.empty(L, dtype=torch.int64, device="cuda")
@@ -54,6 +55,6 @@ for kind in ("leaf", "levels", "diff", "verify"):
     if d:
         print(f"  {kind:7s} mean {sum(d) / len(d):8.1f} us  min {min(d):8.1f}  max {max(d):8.1f}")
 prev_end = 0.0
-for k, s0, s1 in tl[:8]:
+for k, s0, s1 in sorted(tl, key=lambda r: r[1])[:8]:
     print(f"{k:7s} start {s0 * 1e3:9.1f} us  end {s1 * 1e3:9.1f} us  dur {(s1 - s0) * 1e3:7.1f} us  gap {(s0 - prev_end) * 1e3:7.1f}")
     prev_end = max(prev_end, s1)
