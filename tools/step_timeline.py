@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Per-kernel timeline of bench steps (events around every library launch).
 
-usage: step_timeline.py [N_STEPS] [--unfused] [--c5]   (default: the fused pair path bench.py times,
+usage: step_timeline.py [N_STEPS] [--unfused] [--c5] [--lib=PATH]   (default: the fused pair path bench.py times,
 on c2; --c5: the configs[4] per-GPU shard)"""
 import os
 import sys
@@ -11,6 +11,12 @@ import torch
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_middleware_tanaabcrtn24_b200 as ck  # noqa: E402
 import synth  # noqa: E402
+
+for a in sys.argv[1:]:
+    if a.startswith("--lib="):        # an A/B variant library (tools/variant.py)
+        import ctypes
+        ck._lib = ck._declare(ctypes.CDLL(a[6:]))
+        print("library:", a[6:], flush=True)
 
 pair = synth.c5_pair(device="cuda") if "--c5" in sys.argv else synth.c2_pair(device="cuda")
 A, B = pair.a, pair.b
