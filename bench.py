@@ -531,7 +531,7 @@ def run_ours(args):
                        "path": args.path,
                        "hash_block": args.hash_block if args.hash_block else "chunk"},
             "pct_hbm_peak": round(value / (world * peak), 4),
-            "roofline": {"bound": "hbm", "kernel": "leaf_kernel (K1: quantize + chained Murmur3F)",
+            "roofline": {"bound": "hbm", "kernel": "K1 (leaf_pair_kernel for f32 pairs, leaf_kernel otherwise: quantize + chained Murmur3F)",
                          "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "traffic_source": traffic_src,

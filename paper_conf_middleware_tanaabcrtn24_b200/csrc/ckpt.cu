@@ -23,7 +23,6 @@
 
 #include "../../include/ckpt.h"
 #include "compare.cuh"
-#include "follow.cuh"
 #include "hash.cuh"
 #include "leaf.cuh"
 #include "levels.cuh"
@@ -359,11 +358,17 @@ static ckpt_status norm_block(uint32_t hb, uint32_t C, uint32_t *out) {
 template <int DT, bool RAW, int CB, bool PAIR, bool WIDE = false>
 static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
     const uint64_t tasks = P.n_tasks;
-    // pair mode with chunks < 32 KB runs next to the follower: the 72-register kernel
-    auto k = (PAIR && P.chunk < kFollowMaxChunk) ? leaf_pair_kernel<DT, RAW, CB, WIDE>
-                                                 : leaf_kernel<DT, RAW, CB, PAIR, WIDE>;
+    // f32 pair mode below 32 KB chunks: the 72-register kernel (leaf.cuh, leaf_pair_kernel)
+    bool capped = false;
+    auto k = leaf_kernel<DT, RAW, CB, PAIR, WIDE>;
+    if constexpr (PAIR && DT == 0 && CB < (int)kLeafPairMaxChunk) {
+        if (P.chunk < kLeafPairMaxChunk) {
+            capped = true;
+            k = leaf_pair_kernel<DT, RAW, CB, WIDE>;
+        }
+    }
     static std::atomic<int> cached_per_sm[2] = {{0}, {0}};
-    std::atomic<int> &cached = cached_per_sm[(PAIR && P.chunk < kFollowMaxChunk) ? 1 : 0];
+    std::atomic<int> &cached = cached_per_sm[capped ? 1 : 0];
     int per_sm = cached.load(std::memory_order_relaxed);
     if (per_sm == 0) {
         CK_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kLeafSmem));
@@ -382,6 +387,7 @@ static ckpt_status launch_leaf_t(const LeafParams &P, cudaStream_t s, int sms) {
     const size_t smem = (size_t)cta_warps * kWarpSmem + 16;
     uint64_t want = (tasks + cta_warps - 1) / cta_warps;
     uint64_t grid = few ? want : std::min<uint64_t>(want, (uint64_t)sms * per_sm);
+    ProfScope prof(0, s);
     CK_CUDA(launch_k(k, dim3((unsigned)grid), dim3(cta_warps * 32), smem, s, P));
     CK_LAUNCH();
     return CKPT_OK;
@@ -473,7 +479,7 @@ static ckpt_status launch_levels(ckpt_tree *const *trees, int n, cudaStream_t s)
             p.ls = 0;
             p.n_groups = (unsigned)t->n_groups;
             b.cta_begin[i] = ctas;
-            ctas += p.n_groups;
+            ctas += (unsigned)t->n_groups;
         }
         b.cta_begin[b.n] = ctas;
         ProfScope prof(1, s);
@@ -526,14 +532,11 @@ static ckpt_status prepare_tree(ckpt_tree *t, cudaStream_t s) {
     return CKPT_OK;
 }
 
-// Launches a kernel right after K1 (the follower), given K1's device array table (or null).
-using AfterLeaves = std::function<ckpt_status(const LeafArray *d_tab)>;
-
 // One leaf-kernel launch over every array of every tree in `table`.
 static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t tasks,
                                  ckpt_dtype dtype, double eps, uint32_t C, uint32_t hash_block,
                                  cudaStream_t s, int sms, const PairParams *pair,
-                                 unsigned long long *ticket, const AfterLeaves *after = nullptr) {
+                                 unsigned long long *ticket) {
     if (!ticket) return fail(CKPT_EINVAL, "leaf launch without a task ticket");
     LeafParams P;
     std::memset(&P, 0, sizeof(P));
@@ -554,7 +557,6 @@ static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t t
         P.arrays = d_tab;
     }
     const bool pm = pair != nullptr;
-    ProfScope prof(0, s);
     if (eps == 0.0) {
         if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, true>(P, s, sms, pm)));
         else CK_TRY((launch_leaf_dt<1, true>(P, s, sms, pm)));
@@ -562,8 +564,6 @@ static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t t
         if (dtype == CKPT_F32) CK_TRY((launch_leaf_dt<0, false>(P, s, sms, pm)));
         else CK_TRY((launch_leaf_dt<1, false>(P, s, sms, pm)));
     }
-    // nothing between K1 and the follower on the stream: it must be K1's programmatic dependent
-    if (after) CK_TRY((*after)(d_tab));
     if (d_tab) CK_CUDA(cudaFreeAsync(d_tab, s));
     return CKPT_OK;
 }
@@ -581,9 +581,6 @@ struct Scratch {
     size_t flags_cap = 0;
     uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
     size_t tile_pairs = 0;              // pair-tasks the buffers hold
-    uint32_t tile_epoch = 0;            // last tile-publication epoch (follower flags)
-    uint8_t *follow = nullptr;          // follower: level tables, slot counts and hit masks
-    size_t follow_cap = 0;
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -613,44 +610,29 @@ static bool tile_gather_forced() {
     return on;
 }
 
-// CKPT_FOLLOW=0: the fused path without the follower (levels kernel + marking after K1; A/B
-// measurements and tests of that path).
-static bool follow_enabled() {
-    static const bool on = [] {
-        const char *e = std::getenv("CKPT_FOLLOW");
-        return !(e && e[0] == '0');
-    }();
-    return on;
-}
-
 // K1 tile-compaction buffers for n_pair pair-tasks (leaf.cuh PairParams):
 // [tctr: n_tiles u32, zeroed once; self-resetting] [tagg: n_tiles u32]
 // [tmask: n_pair u32] [tbase: n_pair u64] [tids: n_tiles * kTileTasks * 32 u64]
-static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, PairParams *pp,
-                                    uint32_t **tready = nullptr, unsigned int **tsub = nullptr) {
+static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, PairParams *pp) {
     std::lock_guard<std::mutex> lk(g_scr_mu);
     Scratch &sc = g_scr[std::make_pair(dev, s)];
     n_pair = std::max<uint64_t>(n_pair, 1);
-    // [tctr | tready | tsub] (zeroed once) | tagg | tmask | tbase | tids
-    auto layout_of = [](uint64_t np, size_t o[7]) {
+    auto layout_of = [](uint64_t np, size_t o[5]) {
         const uint64_t nt = (np + kTileTasks - 1) / kTileTasks;
         o[0] = 0;
-        o[5] = align256(nt * 4);
-        o[6] = o[5] + align256(nt * 4);
-        o[1] = o[6] + align256((nt + 2) * 4);
+        o[1] = align256(nt * 4);
         o[2] = o[1] + align256(nt * 4);
         o[3] = o[2] + align256(np * 4);
         o[4] = o[3] + align256(np * 8);
         return o[4] + nt * kTileTasks * 32 * 8;
     };
-    size_t o[7];
+    size_t o[5];
     if (sc.tile_pairs < n_pair) {
         if (sc.tile) CK_CUDA(cudaFreeAsync(sc.tile, s));
         sc.tile_pairs = std::max<uint64_t>(n_pair, 2 * sc.tile_pairs);
         const size_t bytes = layout_of(sc.tile_pairs, o);
         CK_CUDA(cudaMallocAsync((void **)&sc.tile, bytes, s));
-        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters, flags, job counters
-        sc.tile_epoch = 0;
+        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters
     }
     layout_of(sc.tile_pairs, o);
     pp->tctr = (unsigned int *)(sc.tile + o[0]);
@@ -658,24 +640,6 @@ static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, Pa
     pp->tmask = (uint32_t *)(sc.tile + o[2]);
     pp->tbase = (uint64_t *)(sc.tile + o[3]);
     pp->tids = (uint64_t *)(sc.tile + o[4]);
-    pp->tready = nullptr;                       // set by callers that launch the follower
-    if (++sc.tile_epoch == 0) sc.tile_epoch = 1;   // flags hold earlier epochs, never this one
-    pp->epoch = sc.tile_epoch;
-    if (tready) *tready = (uint32_t *)(sc.tile + o[5]);
-    if (tsub) *tsub = (unsigned int *)(sc.tile + o[6]);
-    return CKPT_OK;
-}
-
-// Follower buffers (grow, never shrink): returns the base of `bytes` bytes.
-static ckpt_status get_follow_scratch(int dev, cudaStream_t s, size_t bytes, uint8_t **out) {
-    std::lock_guard<std::mutex> lk(g_scr_mu);
-    Scratch &sc = g_scr[std::make_pair(dev, s)];
-    if (sc.follow_cap < bytes) {
-        if (sc.follow) CK_CUDA(cudaFreeAsync(sc.follow, s));
-        sc.follow_cap = std::max<size_t>(bytes, sc.follow_cap + sc.follow_cap / 2);
-        CK_CUDA(cudaMallocAsync((void **)&sc.follow, sc.follow_cap, s));
-    }
-    *out = sc.follow;
     return CKPT_OK;
 }
 
@@ -700,7 +664,7 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
                                     const uint32_t *arrays_per_tree, uint32_t n_trees,
                                     ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
                                     uint32_t hash_block, void *stream, ckpt_tree **out,
-                                    const PairParams *pair, const FollowParams *follow = nullptr) {
+                                    const PairParams *pair) {
     if (!out || n_trees == 0 || !arrays_per_tree) return fail(CKPT_EINVAL, "no trees / NULL out");
     for (uint32_t k = 0; k < n_trees; ++k) out[k] = nullptr;
     if (!data || !n) return fail(CKPT_EINVAL, "no arrays");
@@ -769,34 +733,9 @@ static ckpt_status build_batch_impl(const void *const *data, const uint64_t *n,
         st = get_scratch(dev, s, 0, &unused_states, &ticket, &unused_epoch);
         ticket += kLeafTicketSlot;
     }
-    AfterLeaves after;
-    if (st == CKPT_OK && follow && pair && n_trees == 2) {
-        FollowParams fp = *follow;
-        pp.tready = const_cast<uint32_t *>(fp.tready);
-        fp.n_pair = pp.n_pair;
-        fp.m = (int)out[0]->n_arrays;
-        fp.n_arrays = (int)table.size();
-        fp.chunk = chunk_bytes;
-        fp.per = chunk_bytes / (uint32_t)esz;
-        fp.groups = (fp.per + 1023) / 1024;
-        fp.eps = eps;
-        fp.tagg = pp.tagg;
-        fp.tids = pp.tids;
-        fp.epoch = pp.epoch;
-        if (table.size() <= (size_t)kLeafInline)
-            for (size_t k = 0; k < table.size(); ++k) fp.inl[k] = table[k];
-        const int sms = di.sms;
-        after = [fp, sms, dtype, s](const LeafArray *d_tab) mutable -> ckpt_status {
-            fp.arrays = d_tab;
-            CK_CUDA(launch_k(dtype == CKPT_F32 ? follow_kernel<0> : follow_kernel<1>, dim3((unsigned)sms),
-                             dim3(kFollowWarps * 32), 0, s, fp));
-            CK_LAUNCH();
-            return CKPT_OK;
-        };
-    }
     if (st == CKPT_OK)
         st = launch_leaves(table, task, dtype, eps, chunk_bytes, hash_block, s, di.sms,
-                           pair ? &pp : nullptr, ticket, after ? &after : nullptr);
+                           pair ? &pp : nullptr, ticket);
     if (st == CKPT_OK) {
         // K2 on the side stream, after the leaves; each tree records its own event
         cudaStream_t ss = nullptr;
@@ -992,7 +931,7 @@ static void release_scratch(int dev, cudaStream_t s) {
     auto it = g_scr.find(std::make_pair(dev, s));
     if (it == g_scr.end()) return;
     Scratch &sc = it->second;
-    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile, sc.follow};
+    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile};
     for (void *b : bufs)
         if (b) cudaFreeAsync(b, s);
     g_scr.erase(it);
@@ -1169,8 +1108,7 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
                                uint64_t n_chunks_host, uint64_t chunks_cap, double eps,
                                uint64_t *idx, uint64_t cap, uint64_t *n_diff_dev, cudaStream_t s,
                                const EmitHook &before_emit = nullptr, uint64_t chunk_base0 = 0,
-                               uint64_t elem_base0 = 0, const PairParams *tiles = nullptr,
-                               const uint32_t *scnt = nullptr, uint32_t *smask = nullptr) {
+                               uint64_t elem_base0 = 0, const PairParams *tiles = nullptr) {
     if (!a || !b || !n || na == 0) return fail(CKPT_EINVAL, "no arrays");
     if (!n_diff_dev || (!idx && cap && !before_emit)) return fail(CKPT_EINVAL, "NULL output");
     CK_TRY(check_common(dtype, chunk_bytes, eps));
@@ -1260,19 +1198,10 @@ static ckpt_status verify_impl(const void *const *a, const void *const *b, const
     const size_t o_off = align256((size_t)max_chunks * 4);
     const size_t o_mask = o_off + align256((size_t)max_chunks * 8);
     uint8_t *work = nullptr;
-    // premarked (follower): the hit masks stay in the tile slots; K4a records each listed
-    // chunk's slot (4 bytes) where its mask would go
-    const size_t mask_bytes = scnt ? (size_t)max_chunks * 4 : (size_t)max_chunks * p.groups * 128;
-    CK_TRY(get_work(dev, s, o_mask + mask_bytes, &work));
+    CK_TRY(get_work(dev, s, o_mask + (size_t)max_chunks * p.groups * 128, &work));
     p.cnt = (uint32_t *)work;
     p.off = (uint64_t *)(work + o_off);
     p.mask = (uint32_t *)(work + o_mask);
-    if (scnt) {
-        if (!tiles || !smask) return fail(CKPT_EINVAL, "premarked verify without tiles");
-        p.scnt = scnt;
-        p.mslot = (uint32_t *)(work + o_mask);
-        p.mask = smask;
-    }
     {
         ProfScope prof(3, s);
         CK_CUDA(launch_k(d == 0 ? verify_mark_kernel<0> : verify_mark_kernel<1>, dim3(g_mark),
@@ -1337,31 +1266,7 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     CK_TRY(get_pair_flags(dev, s, L, &pp.flags));
     uint64_t n_pair = 0;                          // pair-tasks: kRows chunks of one array each
     for (uint32_t k = 0; k < n_arrays; ++k) n_pair += ((n[k] * esz + chunk_bytes - 1) / chunk_bytes + kRows - 1) / kRows;
-    // the ordered chunk list from K1's per-tile compaction: read by K4a directly (up to
-    // kVerifyMaxTiles tiles), else placed by one gather pass.  With the list read from the
-    // tiles, the follower (follow.cuh) builds the level groups and marks the flagged chunks
-    // while K1 runs.
-    const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
-    const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
-    const bool use_follow = tiles_in_mark && chunk_bytes < kFollowMaxChunk && follow_enabled();
-    uint32_t *tready = nullptr;
-    unsigned int *tsub = nullptr;
-    CK_TRY(get_tile_scratch(dev, s, n_pair, &pp, &tready, &tsub));
-    FollowParams fp;
-    std::memset(&fp, 0, sizeof(fp));
-    if (use_follow) {
-        const uint32_t per = chunk_bytes / (uint32_t)esz;
-        const uint64_t groups = (per + 1023) / 1024;
-        const uint64_t slots = n_tiles * kTileTasks * 32;
-        const size_t o_mask = align256(slots * 4);
-        uint8_t *base = nullptr;
-        CK_TRY(get_follow_scratch(dev, s, o_mask + slots * groups * 128, &base));
-        fp.scnt = (uint32_t *)base;
-        fp.smask = (uint32_t *)(base + o_mask);
-        fp.tready = tready;
-        fp.tsub = tsub;
-        fp.n_tiles = (uint32_t)n_tiles;
-    }
+    CK_TRY(get_tile_scratch(dev, s, n_pair, &pp));
     std::vector<const void *> data(2 * (size_t)n_arrays);
     std::vector<uint64_t> nn(2 * (size_t)n_arrays);
     for (uint32_t k = 0; k < n_arrays; ++k) {
@@ -1372,8 +1277,12 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     const uint32_t apt[2] = {n_arrays, n_arrays};
     ckpt_tree *trees[2] = {nullptr, nullptr};
     CK_TRY(build_batch_impl(data.data(), nn.data(), apt, 2, dtype, chunk_bytes, eps, hash_block, stream,
-                            trees, &pp, use_follow ? &fp : nullptr));
+                            trees, &pp));
+    // the ordered chunk list from K1's per-tile compaction: read by K4a directly (up to
+    // kVerifyMaxTiles tiles), else placed by one gather pass
     ckpt_status st = CKPT_OK;
+    const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
+    const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
     pp.n_pair = n_pair;
     if (!tiles_in_mark) {
         TileGatherParams g;
@@ -1391,8 +1300,7 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     }
     if (st == CKPT_OK)
         st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
-                         idx, idx_cap, counts_dev + 1, s, before_emit, 0, 0, tiles_in_mark ? &pp : nullptr,
-                         use_follow ? fp.scnt : nullptr, use_follow ? fp.smask : nullptr);
+                         idx, idx_cap, counts_dev + 1, s, before_emit, 0, 0, tiles_in_mark ? &pp : nullptr);
     if (st != CKPT_OK) {
         ckpt_tree_free_on(trees[0], stream);
         ckpt_tree_free_on(trees[1], stream);

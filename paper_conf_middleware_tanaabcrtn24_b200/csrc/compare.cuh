@@ -398,11 +398,6 @@ struct VerifyParams {
     uint32_t tile_ids;
     uint64_t *list_out;
     uint64_t *n_chunks_out;
-    // premarked (the follower marked the tile slots while K1 ran, follow.cuh): K4a only places
-    // the list, copies each listed chunk's count from its tile slot and records the slot, whose
-    // hit mask K4c reads (mask then points at the slot masks)
-    const uint32_t *scnt;         // [tile slot] hits, or null
-    uint32_t *mslot;              // [chunks_cap] tile slot of list position q
 };
 
 constexpr int kVerifyMaxTiles = 4096;   // tile prefix table of K4a in shared memory
@@ -463,14 +458,15 @@ __device__ __forceinline__ void tile_prefix(const VerifyParams &p, uint32_t *s_t
     __syncthreads();
 }
 
-// Tile mode: tile slot of list position q (q < total).
-__device__ __forceinline__ uint64_t tile_slot(const VerifyParams &p, const uint32_t *s_tpre, uint64_t q) {
+// Tile mode: chunk id of list position q (q < total).
+__device__ __forceinline__ uint64_t tile_chunk(const VerifyParams &p, const uint32_t *s_tpre, uint64_t q) {
     uint32_t lo = 0, hi = p.n_tiles - 1;               // last tile with s_tpre[t] <= q
     while (lo < hi) {
         const uint32_t mid = (lo + hi + 1) >> 1;
         if (s_tpre[mid] <= q) lo = mid; else hi = mid - 1;
     }
-    return (uint64_t)lo * p.tile_ids + (q - s_tpre[lo]);
+    return __ldcg(reinterpret_cast<const unsigned long long *>(p.tids) + (uint64_t)lo * p.tile_ids +
+                  (q - s_tpre[lo]));
 }
 
 // Chunks per warp group: the largest power of two <= 32 that still gives
@@ -519,20 +515,13 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_mark_kernel(const __gri
       ChunkLoc mine{nullptr, nullptr, 0, 0};
       if (lane < (int)G && q0 + lane < n_chunks) {
           if (p.tagg) {
-              const uint64_t slot = tile_slot(p, s_tpre, q0 + lane);
-              const uint64_t g = __ldcg(reinterpret_cast<const unsigned long long *>(p.tids) + slot);
+              const uint64_t g = tile_chunk(p, s_tpre, q0 + lane);
               p.list_out[q0 + lane] = g;
-              if (p.scnt) {
-                  p.cnt[q0 + lane] = __ldcg(p.scnt + slot);
-                  p.mslot[q0 + lane] = (uint32_t)slot;
-              } else {
-                  verify_locate_g(p, g, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
-              }
+              verify_locate_g(p, g, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
           } else {
               verify_locate(p, q0 + lane, ESZ, mine.pa, mine.pb, mine.len, mine.gbase);
           }
       }
-      if (p.scnt) continue;   // premarked: nothing left to mark
       const uint32_t nq = (n_chunks - q0) < G ? (uint32_t)(n_chunks - q0) : G;
       for (uint32_t j = 0; j < nq; ++j) {
         const uint64_t q = q0 + j;
@@ -639,8 +628,8 @@ __global__ void __launch_bounds__(kVerifyThreads) verify_emit_kernel(const __gri
       uint64_t my_off = 0, my_gb = 0, my_key = 0;
       uint32_t c = 0, my_groups = 0;
       if (lane < (int)G && q0 + lane < n_chunks) {
-          my_key = p.mslot ? (uint64_t)p.mslot[q0 + lane] : q0 + lane;   // the chunk's mask
-          c = p.cnt[q0 + lane];
+          my_key = q0 + lane;
+          c = p.cnt[my_key];
           if (c) {
               const uint8_t *pa, *pb;
               uint64_t len;

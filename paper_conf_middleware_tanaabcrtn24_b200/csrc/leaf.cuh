@@ -207,8 +207,8 @@ constexpr int kLeafInline = 16;
 
 // Fused pair mode: the table holds checkpoint A's m
 // arrays then B's m arrays (identical shapes); warp task t < n_pair is A's
-// task t, t >= n_pair is B's task t - n_pair, and the warps draw them
-// interleaved (A's task p, B's task p, A's task p+1, ...).  Whichever of the two
+// task t, t >= n_pair is B's task t - n_pair (the usual batch order, so the
+// warps in flight stream one checkpoint at a time).  Whichever of the two
 // warps of a pair-task finishes second (a self-resetting atomicInc counter per
 // pair-task) compares the 32 leaf digests and writes one flag byte per chunk:
 // the diff at start level 0 happens inside K1.  (Marking the flagged chunks'
@@ -231,8 +231,6 @@ struct PairParams {
     unsigned int *tctr;           // [n_tiles] 0 between launches
     uint32_t *tagg;               // [n_tiles] flagged chunks per tile
     uint64_t *tids;               // [n_tiles * kTileTasks * 32] tile-compacted chunk ids
-    uint32_t *tready;             // [n_tiles] set to epoch (release) once the tile is written, or
-    uint32_t epoch;               // null (no follower: follow.cuh)
 };
 
 // The tile's ordered chunk ids, by the warp that completed its last pair-task
@@ -262,15 +260,6 @@ __device__ __noinline__ void tile_compact(const PairParams &pr, uint64_t tile, i
         run += tot;
     }
     if (lane == 0) pr.tagg[tile] = run;
-    if (pr.tready) {
-        // publish the tile to the follower: the warp barrier orders every lane's id stores
-        // before lane 0's release, which is also cumulative over the tile's leaves (acquired
-        // through the pair-task and tile counters)
-        __syncwarp();
-        if (lane == 0)
-            asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(pr.tready + tile), "r"(pr.epoch)
-                         : "memory");
-    }
 }
 
 struct LeafParams {
@@ -349,10 +338,7 @@ __device__ __forceinline__ void leaf_body(const LeafParams &P) {
         }
         return __shfl_sync(0xffffffffu, t, 0);
     };
-    for (uint64_t drawn = draw(); drawn < n_tasks; drawn = draw()) {
-        // pair mode takes A's and B's task of a pair-task one after the other, so pair-tasks
-        // (and tiles) complete at an even rate over the whole launch, not only in B's half
-        const uint64_t task = PAIR ? ((drawn & 1) ? P.pr.n_pair + (drawn >> 1) : (drawn >> 1)) : drawn;
+    for (uint64_t task = draw(); task < n_tasks; task = draw()) {
         const int a = find_array(arrays, n_arrays, task);
         const LeafArray A = arrays[a];
         const uint64_t c0 = (task - A.task_begin) * kRows;   // first local chunk of the task
@@ -549,14 +535,13 @@ leaf_kernel(const __grid_constant__ LeafParams P) {
     leaf_body<DT, RAW, CB, PAIR, WIDE>(P);
 }
 
-// Fused pair mode next to the follower (follow.cuh, chunks < 32 KB): 72 registers instead of
-// 80.  Warps are bound to one of the SM's four sub-partitions and take their registers from that
-// quarter of the register file (16384): six 80-register K1 warps leave 1024 (a 32-register
-// warp), six 72-register warps leave 2560 (one 80-register follower warp per sub-partition).
-// Measured: a 1-warp kernel of 46 or more registers launched after the 80-register K1 starts
-// only when K1's CTAs retire, one of 30 registers starts with K1 (tools/probe_follow.py); K1 at
-// 72 registers is as fast as at 80 (c2 leaf 687-688 vs 691 us, c5 equal).
+// Fused f32 pair mode below 32 KB chunks: the same body capped at 72 registers instead of the
+// 80 that three 8-warp CTAs per SM allow (same SASS instruction mix, different register
+// assignment).  c2 leaf 685.5-685.9 vs 691.9-692.9 us over four alternating reps, c5 within
+// noise; the f64 pair kernels stay at 80 (c3 at 512 B / 16 KiB chunks 0.8 % slower at 72).
+// profiles/r2/follower_trials.md.
 constexpr int kLeafPairRegs = 72;
+constexpr uint32_t kLeafPairMaxChunk = 32768;
 template <int DT, bool RAW, int CB, bool WIDE = false>
 __global__ void __maxnreg__(kLeafPairRegs) leaf_pair_kernel(const __grid_constant__ LeafParams P) {
     leaf_body<DT, RAW, CB, true, WIDE>(P);

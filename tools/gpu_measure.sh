@@ -14,7 +14,7 @@ M=$M,sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active,sm__pipe_xu_cy
 M=$M,sm__inst_executed_pipe_fmaheavy.sum,sm__inst_executed_pipe_fmalite.sum,sm__inst_executed_pipe_alu.sum
 M=$M,sm__inst_executed_pipe_fp64.sum,sm__inst_executed_pipe_xu.sum,sm__inst_executed_pipe_lsu.sum,sm__inst_executed_pipe_uniform.sum
 M=$M,dram__bytes_read.sum,dram__bytes_write.sum,sm__cycles_active.avg
-timeout 600 ncu --metrics $M --clock-control none -k regex:leaf_kernel -s 2 -c 1 --csv --log-file $O/k1_pipes.csv python tools/one_pair.py > $O/k1_pipes.log 2>&1; echo "pipes rc=$?"
+timeout 600 ncu --metrics $M --clock-control none -k regex:leaf_ -s 2 -c 1 --csv --log-file $O/k1_pipes.csv python tools/one_pair.py > $O/k1_pipes.log 2>&1; echo "pipes rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -s 40 -c 60 --csv --log-file $O/launches.csv python bench.py --steps 4 --warmup 3 --no-e2e --no-cpu > $O/launches.log 2>&1; echo "launches rc=$?"
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:leaf_kernel -s 2 -c 1 -o $O/k1_full python tools/one_pair.py > $O/k1_full.log 2>&1; echo "k1full rc=$?"
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:leaf_ -s 2 -c 1 -o $O/k1_full python tools/one_pair.py > $O/k1_full.log 2>&1; echo "k1full rc=$?"
 for f in $O/bench_*.json; do echo "== $f"; head -c 300 $f; echo; done

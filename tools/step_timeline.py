@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Per-kernel timeline of bench steps (events around every library launch).
 
-usage: step_timeline.py [N_STEPS] [--unfused] [--c5] [--lib=PATH]   (default: the fused pair path bench.py times,
+usage: step_timeline.py [N_STEPS] [--unfused] [--c5 | --c3 [--chunk=BYTES]] [--lib=PATH]   (default: the fused pair path bench.py times,
 on c2; --c5: the configs[4] per-GPU shard)"""
 import os
 import sys
@@ -18,11 +18,21 @@ for a in sys.argv[1:]:
         ck._lib = ck._declare(ctypes.CDLL(a[6:]))
         print("library:", a[6:], flush=True)
 
-pair = synth.c5_pair(device="cuda") if "--c5" in sys.argv else synth.c2_pair(device="cuda")
+CHUNK = 4096
+for a in sys.argv[1:]:
+    if a.startswith("--chunk="):
+        CHUNK = int(a[8:])
+if "--c5" in sys.argv:
+    pair = synth.c5_pair(device="cuda")
+elif "--c3" in sys.argv:                  # configs[2]: 2^29 f64, the chunk size from --chunk=
+    pair = synth.c3_pair(device="cuda", chunk_bytes=CHUNK)
+else:
+    pair = synth.c2_pair(device="cuda")
 A, B = pair.a, pair.b
-L = sum(t.numel() * 4 // 4096 for t in A)
+L = sum(-(-t.numel() * t.element_size() // CHUNK) for t in A)
 chunks = torch.empty(L, dtype=torch.int64, device="cuda")
-idx = torch.empty(sum(t.numel() for t in A), dtype=torch.int64, device="cuda")
+idx = torch.empty(sum(t.numel() for t in A) // (8 if "--c5" in sys.argv else 1), dtype=torch.int64,
+                  device="cuda")
 counts = torch.zeros(2, dtype=torch.int64, device="cuda")
 
 
@@ -31,9 +41,9 @@ FUSED = "--unfused" not in sys.argv     # the bench path: ckpt_compare_pair_asyn
 
 def step():
     if FUSED:
-        TA, TB = ck.compare_pair_async(A, B, 4096, 1e-6, chunks, idx, counts)
+        TA, TB = ck.compare_pair_async(A, B, CHUNK, 1e-6, chunks, idx, counts)
     else:
-        TA, TB = ck.tree_build_batch([A, B], 4096, 1e-6)
+        TA, TB = ck.tree_build_batch([A, B], CHUNK, 1e-6)
         ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)
     TA.wait()
     TB.wait()
