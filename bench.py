@@ -352,49 +352,6 @@ def run_ours(args):
         TA.wait()          # the step ends when both trees are complete (K2 runs on a side stream)
         TB.wait()
 
-    # --pipeline on (fused path): P steps = one ckpt_compare_pairs_async call over P pairs, so
-    # pair p's post-leaf kernels (list placement + verify on the verify stream, levels on the
-    # side stream) run in the tail of pair p+1's leaf kernel instead of between the two.  Every
-    # pair is compared in full (own trees, own counts; chunk/idx buffers shared, the last pair's
-    # values remain); for N > 1 the C1/C2 exchange of all P pairs is one all-gather.
-    pipelined = args.path == "fused" and args.pipeline == "on"
-    w_steps = max(3, args.warmup, args.steps if pipelined else 0)
-    max_p = max(3, args.warmup, args.steps)
-    cnt_all = torch.zeros((max_p, 2), dtype=torch.int64, device="cuda") if pipelined else None
-    send_p = recv_p = None
-    if pipelined and collect:
-        send_p = torch.empty((max_p, 2 * n_arrays + 1, 16), dtype=torch.uint8, device="cuda")
-        recv_p = torch.empty((world, max_p, 2 * n_arrays + 1, 16), dtype=torch.uint8, device="cuda")
-
-    def step_seq(P):
-        trees = ck.compare_pairs_async([A] * P, [B] * P, CHUNK, EPS, chunks, idx,
-                                       [cnt_all[p] for p in range(P)], hash_block=args.hash_block)
-        if collect:
-            for p, (TA, TB) in enumerate(trees):
-                TA.array_roots(out=send_p[p, :n_arrays])
-                TB.array_roots(out=send_p[p, n_arrays:2 * n_arrays])
-            send_p[:P, 2 * n_arrays].view(torch.int64).view(P, 2).copy_(cnt_all[:P])
-            rv = recv_p[:, :P].contiguous() if P < max_p else recv_p
-            dist.all_gather_into_tensor(rv.view(-1), send_p[:P].contiguous().view(-1))
-            # per pair: both top trees over all ranks' array roots
-            roots = rv[:, :, :2 * n_arrays].reshape(world, P, 2, n_arrays, 16).permute(1, 2, 0, 3, 4)
-            tops = ck.tree_from_digests_batch(roots.reshape(P * 2 * world * n_arrays, 16),
-                                              [world * n_arrays] * (2 * P))
-            tot = rv[:, :, 2 * n_arrays].contiguous().view(torch.int64).view(world, P, 2).sum(0)
-            keep[:] = [*trees[-1], *tops[-2:], tot]
-        else:
-            keep[:] = list(trees[-1])
-        for TA, TB in trees:
-            TA.wait()
-            TB.wait()
-
-    def run_steps(P):
-        if pipelined:
-            step_seq(P)
-        else:
-            for _ in range(P):
-                step()
-
     # configs[3] as written (--snapshots all): the 10 intermediate snapshots, one at a time
     # (each generated into HBM before its timed region), every snapshot's trees kept; the
     # sequence's time is the sum of the snapshots' device times.  Otherwise one snapshot / pair.
@@ -412,14 +369,10 @@ def run_ours(args):
             A = B = pair = None
             pair = make_pair(CFG, N_PARTICLES, SEED + 1000 * rank, "cuda")
             A, B = pair.a, pair.b
-        # pipelined: the warm-up sequence is as long as the timed one, so the memory pool already
-        # holds the trees of K in-flight pairs when the timed region starts
-        run_steps(w_steps)
+        for _ in range(max(3, args.warmup)):
+            step()
         torch.cuda.synchronize()
-        local_counts = (cnt_all[0] if pipelined else counts).cpu().tolist()
-        if pipelined:   # every pair of the sequence is the same pair: the same counts
-            assert bool((cnt_all[:w_steps] == cnt_all[0]).all()), "pipelined pairs disagree"
-
+        local_counts = counts.cpu().tolist()
         # timed region: no events between the kernels (an event after the leaf kernel would end
         # the programmatic-launch overlap of the next kernel with its tail); the leaf kernel's
         # own duration is timed in a separate pass below
@@ -431,7 +384,8 @@ def run_ours(args):
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record()
         h0 = time.perf_counter()
-        run_steps(args.steps)
+        for _ in range(args.steps):
+            step()
         host_ms += (time.perf_counter() - h0) * 1e3 / args.steps   # enqueue time per step (host)
         e1.record()
         torch.cuda.synchronize()
@@ -445,7 +399,8 @@ def run_ours(args):
         # the roofline kernel: events around every leaf launch of another K steps
         ck.profile_reset()
         ck.profile_enable(["leaf"])
-        run_steps(args.steps)
+        for _ in range(args.steps):
+            step()
         torch.cuda.synchronize()
         ck.profile_enable(False)
         lm, ln = ck.profile_read("leaf")
@@ -461,37 +416,12 @@ def run_ours(args):
             per_snap.append({"snapshot": snap, "ms": round(float(t.item()), 4),
                              "flagged_chunks_per_gpu": local_counts[0],
                              "diff_elems_per_gpu": local_counts[1]})
-    per_call = None
-    if pipelined:
-        # the same K steps as K separate ckpt_compare_pair_async calls (post-leaf kernels between
-        # the leaf kernels): reported beside the pipelined value
-        for _ in range(3):
-            step()
-        if collect:
-            dist.barrier()
-        torch.cuda.synchronize()
-        p0 = torch.cuda.Event(enable_timing=True)
-        p1 = torch.cuda.Event(enable_timing=True)
-        p0.record()
-        for _ in range(args.steps):
-            step()
-        p1.record()
-        torch.cuda.synchronize()
-        t = torch.tensor([p0.elapsed_time(p1) / args.steps], dtype=torch.float64, device="cuda")
-        if collect:
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        pc_ms = float(t.item())
-        per_call = {"ms_per_step": round(pc_ms, 4),
-                    "value": round(bytes_pair * world / (pc_ms / 1e3) / 1e9, 2), "unit": "GB/s",
-                    "api": "one ckpt_compare_pair_async per step (post-leaf kernels between the "
-                           "leaf kernels), last snapshot only" if len(snaps) > 1 else
-                           "one ckpt_compare_pair_async per step (post-leaf kernels between the "
-                           "leaf kernels)"}
     clocks = sampler.stop()
     # per-phase device times from a separate profiled pass (events around every family)
     k_prof = max(3, min(args.steps, 20))
     ck.profile_enable(True)
-    run_steps(k_prof)
+    for _ in range(k_prof):
+        step()
     torch.cuda.synchronize()
     ck.profile_enable(False)
     phases = {"steps": k_prof}
@@ -586,7 +516,7 @@ def run_ours(args):
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
-            "steps": args.steps, "warmup": w_steps, "ms_per_step": round(ms_max, 4),
+            "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": round(ms_max, 4),
             "higher_is_better": True, "scaling": "strong" if CFG == "c4" else "weak",
             "vs_baseline": None,
             "dtype": f"{'f64' if A[0].dtype == torch.float64 else 'f32'} in, f64 quantize/compare, u64 hash",
@@ -599,9 +529,6 @@ def run_ours(args):
                        "l2": f"inputs larger than L2 ({bytes_pair / 1e9:.1f} GB per GPU per step >> 126 MB)",
                        "parallelism": f"dp{world} (checkpoint arrays sharded by rank)",
                        "path": args.path,
-                       "pipeline": ("K steps = one ckpt_compare_pairs_async call over K pairs: pair "
-                                    "p's post-leaf kernels overlap pair p+1's leaf kernel")
-                       if pipelined else "off (one call per step)",
                        "hash_block": args.hash_block if args.hash_block else "chunk"},
             "pct_hbm_peak": round(value / (world * peak), 4),
             "roofline": {"bound": "hbm", "kernel": "K1 (leaf_pair_kernel for f32 pairs, leaf_kernel otherwise: quantize + chained Murmur3F)",
@@ -616,7 +543,7 @@ def run_ours(args):
             "phases_profiled_pass": phases, "host_enqueue_ms_per_step": round(host_ms, 4),
             "flagged_chunks_per_gpu": local_counts[0], "diff_elems_per_gpu": local_counts[1],
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
-            "direct_k5": direct_k5, "dist": nccl_info, "per_call": per_call,
+            "direct_k5": direct_k5, "dist": nccl_info,
         }
         if per_snap:
             line["snapshot_sequence"] = {
@@ -658,10 +585,6 @@ def main():
     ap.add_argument("--path", default="fused", choices=["fused", "unfused", "saved"],
                     help="fused: ckpt_compare_pair_async; unfused: build_batch + diff_verify_async; "
                          "saved: ckpt_compare_saved (A = stored tree + pinned host data)")
-    ap.add_argument("--pipeline", default="on", choices=["on", "off"],
-                    help="fused path: on = the K timed steps are one ckpt_compare_pairs_async call "
-                         "(pair p's post-leaf kernels overlap pair p+1's leaf kernel); off = one "
-                         "ckpt_compare_pair_async call per step")
     ap.add_argument("--snapshot", type=int, default=9, help="c4: snapshot index 0..9")
     ap.add_argument("--snapshots", default="one", choices=["one", "all"],
                     help="c4: 'all' = BASELINE configs[3] as written, the 10-snapshot sequence")

@@ -259,39 +259,6 @@ ckpt_status ckpt_compare_pair_ex(const void *const *a, const void *const *b, con
                                  uint64_t *counts_dev, void *stream, ckpt_tree **out_a,
                                  ckpt_tree **out_b);
 
-/* Pipelined sequence of fused pair compares: n_pairs checkpoint pairs (e.g.
- * the intermediate snapshots of two runs' histories, P:212-217, P:738-741,
- * compared snapshot by snapshot), each exactly as ckpt_compare_pair_ex.
- * Pair p's leaf kernel runs on `stream`; its list placement and verify
- * kernels run on a library-owned verify stream (one per caller stream) and
- * its interior levels on the side stream, so pair p+1's leaf kernel starts
- * when pair p's ends and pair p's latency-bound post-leaf kernels run in the
- * SM slots that free up in the tail of pair p+1's leaf kernel.  The K1 tile
- * buffers rotate over 3 slots; before pair p's leaf kernel, `stream` waits
- * for the verify of pair p-3 (the slot's last reader).
- *   a, b        (host) n_pairs * n_arrays device pointers, pair p's arrays at
- *               [p*n_arrays, (p+1)*n_arrays), 16-byte aligned
- *   n           (host) n_pairs * n_arrays element counts (A and B share them)
- *   chunks, idx, counts_dev   (host) n_pairs device pointers each, with
- *               chunks_cap / idx_cap (host) n_pairs capacities: pair p's
- *               outputs as in ckpt_compare_pair_async.  Outputs of different
- *               pairs may alias (the verify stream runs the pairs in order;
- *               the last pair's values remain).
- *   out_trees   (host) 2*n_pairs: pair p's trees at [2p] (A) and [2p+1] (B),
- *               owned by the caller (ckpt_tree_free)
- * On return every kernel is enqueued and `stream` is ordered after every
- * pair's verify (the outputs are valid in stream order); interior levels
- * are joined per tree as for ckpt_tree_build_batch.  Errors: EINVAL,
- * ENOMEM, ECUDA (every tree of the call is freed, out_trees set to NULL).
- * Asynchronous. */
-ckpt_status ckpt_compare_pairs_async(const void *const *a, const void *const *b, const uint64_t *n,
-                                     uint32_t n_arrays, uint32_t n_pairs, ckpt_dtype dtype,
-                                     uint32_t chunk_bytes, double eps, uint32_t hash_block,
-                                     uint64_t *const *chunks, const uint64_t *chunks_cap,
-                                     uint64_t *const *idx, const uint64_t *idx_cap,
-                                     uint64_t *const *counts_dev, void *stream,
-                                     ckpt_tree **out_trees);
-
 /* ------------------------------------------------------------------------
  * One-call pair comparison (steps 1-4 on two checkpoints of n_arrays
  * arrays each), the library API of P:254-257.  Device inputs.  Writes the

@@ -76,8 +76,6 @@ def _declare(L):
                                            vp, pp]
     L.ckpt_compare_pair_ex.argtypes = [pp, pp, pu64, u32, i32, u32, dbl, u32, vp, u64, vp, u64, vp,
                                        vp, pp, pp]
-    L.ckpt_compare_pairs_async.argtypes = [pp, pp, pu64, u32, u32, i32, u32, dbl, u32, pp, pu64, pp,
-                                           pu64, pp, vp, pp]
     L.ckpt_tree_serialized_size.argtypes = [vp, pu64]
     L.ckpt_tree_serialize.argtypes = [vp, vp, u64, pu64, vp]
     L.ckpt_tree_deserialize.argtypes = [vp, u64, vp, pp]
@@ -121,8 +119,7 @@ def _declare(L):
     L.ckpt_last_error.restype = ctypes.c_char_p
     L.ckpt_version.restype = u32
     for name in ("ckpt_tree_build", "ckpt_tree_build_arrays", "ckpt_tree_build_batch",
-                 "ckpt_tree_build_batch_ex", "ckpt_compare_pair_ex", "ckpt_compare_pairs_async",
-                 "ckpt_tree_params",
+                 "ckpt_tree_build_batch_ex", "ckpt_compare_pair_ex", "ckpt_tree_params",
                  "ckpt_tree_serialized_size", "ckpt_tree_serialize", "ckpt_tree_deserialize",
                  "ckpt_compare_saved", "ckpt_compare_stream",
                  "ckpt_tree_from_digests", "ckpt_tree_from_digests_batch",
@@ -680,51 +677,3 @@ def compare_pair_async(arrays_a, arrays_b, chunk_bytes: int, eps: float, chunks:
            "ckpt_compare_pair_ex")
     return (Tree(ta.value, la, code, chunk_bytes, float(eps), sp),
             Tree(tb.value, lb, code, chunk_bytes, float(eps), sp))
-
-
-def compare_pairs_async(pairs_a, pairs_b, chunk_bytes: int, eps: float, chunks, idx, counts,
-                        stream=None, hash_block: int = 16) -> List[Tuple[Tree, Tree]]:
-    """Pipelined sequence of fused pair compares (ckpt_compare_pairs_async): pair p =
-    (pairs_a[p], pairs_b[p]), each a list of arrays of one checkpoint (every pair may have its
-    own lengths, all pairs share the array count, dtype, chunk size and eps).
-
-    ``chunks``, ``idx``, ``counts``: one tensor per pair, or one tensor shared by every pair
-    (the verify stream runs the pairs in order; the last pair's values remain).  Returns each
-    pair's two trees.  Results per pair equal compare_pair_async on that pair."""
-    P = len(pairs_a)
-    if P == 0 or len(pairs_b) != P:
-        raise ValueError("need the same positive number of A and B checkpoints")
-    la = [_as_list(x) for x in pairs_a]
-    lb = [_as_list(x) for x in pairs_b]
-    m = len(la[0])
-    for x, y in zip(la, lb):
-        if len(x) != m or len(y) != m or any(u.numel() != v.numel() for u, v in zip(x, y)):
-            raise ValueError("every pair needs the same array count, A and B the same lengths")
-    flat_a = [t for x in la for t in x]
-    flat_b = [t for y in lb for t in y]
-    code = _check_arrays(flat_a + flat_b)
-
-    def per_pair(x, what, min_numel=0):
-        xs = [x] * P if isinstance(x, torch.Tensor) else list(x)
-        if len(xs) != P:
-            raise ValueError(f"{what}: one tensor per pair or one shared tensor")
-        for t in xs:
-            _check_out(t, what, min_numel)
-        return xs
-
-    cl, il, nl = per_pair(chunks, "chunks"), per_pair(idx, "idx"), per_pair(counts, "counts", 2)
-    pa, _k1 = _ptr_array(flat_a)
-    pb, _k2 = _ptr_array(flat_b)
-    pn, _k3 = _u64_array([t.numel() for t in flat_a])
-    pc, _k4 = _ptr_array(cl)
-    pcc, _k5 = _u64_array([t.numel() for t in cl])
-    pi, _k6 = _ptr_array(il)
-    pic, _k7 = _u64_array([t.numel() for t in il])
-    pk, _k8 = _ptr_array(nl)
-    trees = (ctypes.c_void_p * (2 * P))()
-    sp = _stream_ptr(stream)
-    _check(lib().ckpt_compare_pairs_async(pa, pb, pn, m, P, code, chunk_bytes, float(eps), hash_block,
-                                          pc, pcc, pi, pic, pk, sp, trees),
-           "ckpt_compare_pairs_async")
-    return [(Tree(trees[2 * p], la[p], code, chunk_bytes, float(eps), sp),
-             Tree(trees[2 * p + 1], lb[p], code, chunk_bytes, float(eps), sp)) for p in range(P)]

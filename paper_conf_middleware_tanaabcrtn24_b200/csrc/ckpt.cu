@@ -568,8 +568,6 @@ static ckpt_status launch_leaves(const std::vector<LeafArray> &table, uint64_t t
     return CKPT_OK;
 }
 
-constexpr int kPipeSlots = 3;   // tile-compaction buffer sets per stream (pipelined pair compares)
-
 struct Scratch {
     uint64_t *states = nullptr;
     size_t cap = 0;
@@ -581,11 +579,8 @@ struct Scratch {
     size_t pair_cap = 0;
     uint8_t *pair_flags = nullptr;      // fused pair mode: one flag byte per chunk
     size_t flags_cap = 0;
-    // fused pair mode: K1 tile compaction buffers, one set per pipeline slot
-    // (ckpt_compare_pairs_async: pair p uses slot p % kPipeSlots while the verify
-    // of an earlier pair may still read another slot)
-    uint8_t *tile[kPipeSlots] = {};
-    size_t tile_pairs[kPipeSlots] = {};  // pair-tasks each set holds
+    uint8_t *tile = nullptr;            // fused pair mode: K1 tile compaction buffers
+    size_t tile_pairs = 0;              // pair-tasks the buffers hold
 };
 static std::mutex g_scr_mu;
 static std::map<std::pair<int, cudaStream_t>, Scratch> g_scr;
@@ -618,12 +613,9 @@ static bool tile_gather_forced() {
 // K1 tile-compaction buffers for n_pair pair-tasks (leaf.cuh PairParams):
 // [tctr: n_tiles u32, zeroed once; self-resetting] [tagg: n_tiles u32]
 // [tmask: n_pair u32] [tbase: n_pair u64] [tids: n_tiles * kTileTasks * 32 u64]
-static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, PairParams *pp,
-                                    int slot) {
+static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, PairParams *pp) {
     std::lock_guard<std::mutex> lk(g_scr_mu);
     Scratch &sc = g_scr[std::make_pair(dev, s)];
-    uint8_t *&tile = sc.tile[slot];
-    size_t &tile_pairs = sc.tile_pairs[slot];
     n_pair = std::max<uint64_t>(n_pair, 1);
     auto layout_of = [](uint64_t np, size_t o[5]) {
         const uint64_t nt = (np + kTileTasks - 1) / kTileTasks;
@@ -635,19 +627,19 @@ static ckpt_status get_tile_scratch(int dev, cudaStream_t s, uint64_t n_pair, Pa
         return o[4] + nt * kTileTasks * 32 * 8;
     };
     size_t o[5];
-    if (tile_pairs < n_pair) {
-        if (tile) CK_CUDA(cudaFreeAsync(tile, s));
-        tile_pairs = std::max<uint64_t>(n_pair, 2 * tile_pairs);
-        const size_t bytes = layout_of(tile_pairs, o);
-        CK_CUDA(cudaMallocAsync((void **)&tile, bytes, s));
-        CK_CUDA(cudaMemsetAsync(tile, 0, o[1], s));      // tile counters
+    if (sc.tile_pairs < n_pair) {
+        if (sc.tile) CK_CUDA(cudaFreeAsync(sc.tile, s));
+        sc.tile_pairs = std::max<uint64_t>(n_pair, 2 * sc.tile_pairs);
+        const size_t bytes = layout_of(sc.tile_pairs, o);
+        CK_CUDA(cudaMallocAsync((void **)&sc.tile, bytes, s));
+        CK_CUDA(cudaMemsetAsync(sc.tile, 0, o[1], s));      // tile counters
     }
-    layout_of(tile_pairs, o);
-    pp->tctr = (unsigned int *)(tile + o[0]);
-    pp->tagg = (uint32_t *)(tile + o[1]);
-    pp->tmask = (uint32_t *)(tile + o[2]);
-    pp->tbase = (uint64_t *)(tile + o[3]);
-    pp->tids = (uint64_t *)(tile + o[4]);
+    layout_of(sc.tile_pairs, o);
+    pp->tctr = (unsigned int *)(sc.tile + o[0]);
+    pp->tagg = (uint32_t *)(sc.tile + o[1]);
+    pp->tmask = (uint32_t *)(sc.tile + o[2]);
+    pp->tbase = (uint64_t *)(sc.tile + o[3]);
+    pp->tids = (uint64_t *)(sc.tile + o[4]);
     return CKPT_OK;
 }
 
@@ -939,11 +931,9 @@ static void release_scratch(int dev, cudaStream_t s) {
     auto it = g_scr.find(std::make_pair(dev, s));
     if (it == g_scr.end()) return;
     Scratch &sc = it->second;
-    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags};
+    void *bufs[] = {sc.states, sc.ticket, sc.work, sc.pair_ctr, sc.pair_flags, sc.tile};
     for (void *b : bufs)
         if (b) cudaFreeAsync(b, s);
-    for (uint8_t *t : sc.tile)
-        if (t) cudaFreeAsync(t, s);
     g_scr.erase(it);
 }
 
@@ -1253,8 +1243,7 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
                                      double eps, uint32_t hash_block, uint64_t *chunks,
                                      uint64_t chunks_cap, uint64_t *idx, uint64_t idx_cap,
                                      uint64_t *counts_dev, void *stream, ckpt_tree **out_a,
-                                     ckpt_tree **out_b, const EmitHook &before_emit,
-                                     int slot = 0, cudaStream_t vs = nullptr) {
+                                     ckpt_tree **out_b, const EmitHook &before_emit) {
     if (out_a) *out_a = nullptr;
     if (out_b) *out_b = nullptr;
     if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
@@ -1277,7 +1266,7 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     CK_TRY(get_pair_flags(dev, s, L, &pp.flags));
     uint64_t n_pair = 0;                          // pair-tasks: kRows chunks of one array each
     for (uint32_t k = 0; k < n_arrays; ++k) n_pair += ((n[k] * esz + chunk_bytes - 1) / chunk_bytes + kRows - 1) / kRows;
-    CK_TRY(get_tile_scratch(dev, s, n_pair, &pp, slot));
+    CK_TRY(get_tile_scratch(dev, s, n_pair, &pp));
     std::vector<const void *> data(2 * (size_t)n_arrays);
     std::vector<uint64_t> nn(2 * (size_t)n_arrays);
     for (uint32_t k = 0; k < n_arrays; ++k) {
@@ -1292,20 +1281,10 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
     // the ordered chunk list from K1's per-tile compaction: read by K4a directly (up to
     // kVerifyMaxTiles tiles), else placed by one gather pass
     ckpt_status st = CKPT_OK;
-    // the list placement and the verify run on `vs` when given (pipelined pairs: the next
-    // pair's leaf kernel on `s` does not wait for them), else on `s`
-    cudaStream_t v = vs ? vs : s;
-    if (v != s) {
-        cudaEvent_t leaves_done = nullptr;
-        if (cudaEventCreateWithFlags(&leaves_done, cudaEventDisableTiming) != cudaSuccess ||
-            cudaEventRecord(leaves_done, s) != cudaSuccess || cudaStreamWaitEvent(v, leaves_done, 0) != cudaSuccess)
-            st = fail(CKPT_ECUDA, "verify-stream fork");
-        if (leaves_done) cudaEventDestroy(leaves_done);
-    }
     const uint64_t n_tiles = (n_pair + kTileTasks - 1) / kTileTasks;
     const bool tiles_in_mark = n_tiles <= (uint64_t)kVerifyMaxTiles && chunks_cap > 0 && !tile_gather_forced();
     pp.n_pair = n_pair;
-    if (st == CKPT_OK && !tiles_in_mark) {
+    if (!tiles_in_mark) {
         TileGatherParams g;
         g.tagg = pp.tagg;
         g.tids = pp.tids;
@@ -1315,13 +1294,13 @@ static ckpt_status compare_pair_impl(const void *const *a, const void *const *b,
         g.cap = chunks_cap;
         g.count = counts_dev;
         const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(g.n_tiles, (uint64_t)di.sms * 8));
-        ProfScope prof(2, v);
-        if (launch_k(tile_gather_kernel, dim3(grid), dim3(kGatherThreads), 0, v, g) != cudaSuccess)
+        ProfScope prof(2, s);
+        if (launch_k(tile_gather_kernel, dim3(grid), dim3(kGatherThreads), 0, s, g) != cudaSuccess)
             st = fail(CKPT_ECUDA, "tile gather launch");
     }
     if (st == CKPT_OK)
         st = verify_impl(a, b, n, n_arrays, dtype, chunk_bytes, chunks, counts_dev, 0, chunks_cap, eps,
-                         idx, idx_cap, counts_dev + 1, v, before_emit, 0, 0, tiles_in_mark ? &pp : nullptr);
+                         idx, idx_cap, counts_dev + 1, s, before_emit, 0, 0, tiles_in_mark ? &pp : nullptr);
     if (st != CKPT_OK) {
         ckpt_tree_free_on(trees[0], stream);
         ckpt_tree_free_on(trees[1], stream);
@@ -1350,82 +1329,6 @@ extern "C" ckpt_status ckpt_compare_pair_async(const void *const *a, const void 
                                                ckpt_tree **out_a, ckpt_tree **out_b) {
     return ckpt_compare_pair_ex(a, b, n, n_arrays, dtype, chunk_bytes, eps, 16, chunks, chunks_cap,
                                 idx, idx_cap, counts_dev, stream, out_a, out_b);
-}
-
-// ---------------------------------------------------------------------------
-// pipelined sequence of pair compares (checkpoint histories)
-// ---------------------------------------------------------------------------
-// One verify stream per (device, caller stream): pair p's list placement and verify
-// run there, so pair p+1's leaf kernel on the caller's stream starts as soon as pair
-// p's leaf kernel ends, and the latency-bound post-leaf kernels of pair p run beside
-// pair p+1's leaf kernel.  The greatest priority: the block scheduler hands the verify
-// CTAs the SM slots first (the lowest was 2-3 % slower per pair in steady state,
-// profiles/r2/pipeline_ab.md).
-static std::map<std::pair<int, cudaStream_t>, cudaStream_t> g_vstream;
-
-static ckpt_status verify_stream(int dev, cudaStream_t s, cudaStream_t *out) {
-    std::lock_guard<std::mutex> lk(g_dev_mu);
-    cudaStream_t &v = g_vstream[std::make_pair(dev, s)];
-    if (!v) {
-        int lo = 0, hi = 0;
-        CK_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        CK_CUDA(cudaStreamCreateWithPriority(&v, cudaStreamNonBlocking, hi));
-    }
-    *out = v;
-    return CKPT_OK;
-}
-
-extern "C" ckpt_status ckpt_compare_pairs_async(const void *const *a, const void *const *b,
-                                                const uint64_t *n, uint32_t n_arrays, uint32_t n_pairs,
-                                                ckpt_dtype dtype, uint32_t chunk_bytes, double eps,
-                                                uint32_t hash_block, uint64_t *const *chunks,
-                                                const uint64_t *chunks_cap, uint64_t *const *idx,
-                                                const uint64_t *idx_cap, uint64_t *const *counts_dev,
-                                                void *stream, ckpt_tree **out_trees) {
-    if (!out_trees) return fail(CKPT_EINVAL, "NULL tree outputs");
-    if (n_pairs == 0) return fail(CKPT_EINVAL, "no pairs");
-    for (uint64_t k = 0; k < 2ull * n_pairs; ++k) out_trees[k] = nullptr;
-    if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
-    if (!chunks || !chunks_cap || !idx || !idx_cap || !counts_dev) return fail(CKPT_EINVAL, "NULL output table");
-    int dev;
-    DevInfo di;
-    CK_TRY(dev_info(&dev, &di));
-    cudaStream_t s = (cudaStream_t)stream;
-    cudaStream_t v = nullptr;
-    CK_TRY(verify_stream(dev, s, &v));
-    std::vector<cudaEvent_t> vdone(n_pairs, nullptr);
-    ckpt_status st = CKPT_OK;
-    uint32_t done = 0;
-    for (uint32_t p = 0; p < n_pairs && st == CKPT_OK; ++p) {
-        const int slot = (int)(p % kPipeSlots);
-        // the slot's tile buffers were last read by the verify of pair p - kPipeSlots
-        if (p >= (uint32_t)kPipeSlots && cudaStreamWaitEvent(s, vdone[p - kPipeSlots], 0) != cudaSuccess) {
-            st = fail(CKPT_ECUDA, "slot wait");
-            break;
-        }
-        const size_t o = (size_t)p * n_arrays;
-        st = compare_pair_impl(a + o, b + o, n + o, n_arrays, dtype, chunk_bytes, eps, hash_block,
-                               chunks[p], chunks_cap[p], idx[p], idx_cap[p], counts_dev[p], stream,
-                               &out_trees[2 * p], &out_trees[2 * p + 1], nullptr, slot, v);
-        if (st != CKPT_OK) break;
-        done = p + 1;
-        if (cudaEventCreateWithFlags(&vdone[p], cudaEventDisableTiming) != cudaSuccess ||
-            cudaEventRecord(vdone[p], v) != cudaSuccess)
-            st = fail(CKPT_ECUDA, "verify-done event");
-    }
-    // join: the caller's stream continues after every pair's verify (the verify stream is
-    // serial, so its last event covers all); interior levels are joined per tree (wait_levels)
-    if (done > 0 && vdone[done - 1] && cudaStreamWaitEvent(s, vdone[done - 1], 0) != cudaSuccess && st == CKPT_OK)
-        st = fail(CKPT_ECUDA, "verify-stream join");
-    for (cudaEvent_t e : vdone)
-        if (e) cudaEventDestroy(e);
-    if (st != CKPT_OK) {
-        for (uint64_t k = 0; k < 2ull * n_pairs; ++k) {
-            ckpt_tree_free_on(out_trees[k], stream);
-            out_trees[k] = nullptr;
-        }
-    }
-    return st;
 }
 
 extern "C" ckpt_status ckpt_verify_arrays_async(const void *const *a, const void *const *b,

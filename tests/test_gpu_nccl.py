@@ -76,15 +76,13 @@ def test_nccl_compare_runs_and_sharded_array_match_oracle(world, tmp_path):
         assert z["sh_counts"].tolist() == [sc.size, si.size]
 
 
-@pytest.mark.parametrize("pipeline", ["on", "off"])
 @pytest.mark.parametrize("world", [1, 2])
-def test_bench_runs_n_nccl_ranks(world, pipeline):
-    """bench.py --gpus N under a launcher: N NCCL ranks, the C1/C2 all-gather (per step, or per
-    pipelined sequence of steps), one JSON line."""
+def test_bench_runs_n_nccl_ranks(world):
+    """bench.py --gpus N under a launcher: N NCCL ranks, the per-step all-gather, one JSON line."""
     if torch.cuda.device_count() < world:
         pytest.skip(f"needs {world} GPUs")
     args = [os.path.join(ROOT, "bench.py"), "--gpus", str(world), "--steps", "3", "--warmup", "3",
-            "--no-e2e", "--no-cpu", "--elems", str(1 << 20), "--collectives", "--pipeline", pipeline]
+            "--no-e2e", "--no-cpu", "--elems", str(1 << 20), "--collectives"]
     r = _torchrun(world, args)
     assert r.returncode == 0, r.stderr[-4000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
