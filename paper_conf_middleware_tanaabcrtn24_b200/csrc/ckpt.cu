@@ -404,11 +404,19 @@ static ckpt_status launch_leaf_dt(const LeafParams &P, cudaStream_t s, int sms, 
         if (C == 4096) return launch_leaf_t<DT, RAW, 4096, false, true>(P, s, sms);
         return launch_leaf_t<DT, RAW, 0, false, true>(P, s, sms);
     }
-    if (pair) {   // fused pair mode: the bench chunk size specialised, others generic
+    if (pair) {   // fused pair mode: the configs[2] sweep's chunk sizes specialised, others generic
         if constexpr (!RAW) {
-            if (C == 4096) return launch_leaf_t<DT, RAW, 4096, true>(P, s, sms);
-            if (C == 32768) return launch_leaf_t<DT, RAW, 32768, true>(P, s, sms);
-            if (C == 65536) return launch_leaf_t<DT, RAW, 65536, true>(P, s, sms);
+            switch (C) {
+                case 512: return launch_leaf_t<DT, RAW, 512, true>(P, s, sms);
+                case 1024: return launch_leaf_t<DT, RAW, 1024, true>(P, s, sms);
+                case 2048: return launch_leaf_t<DT, RAW, 2048, true>(P, s, sms);
+                case 4096: return launch_leaf_t<DT, RAW, 4096, true>(P, s, sms);
+                case 8192: return launch_leaf_t<DT, RAW, 8192, true>(P, s, sms);
+                case 16384: return launch_leaf_t<DT, RAW, 16384, true>(P, s, sms);
+                case 32768: return launch_leaf_t<DT, RAW, 32768, true>(P, s, sms);
+                case 65536: return launch_leaf_t<DT, RAW, 65536, true>(P, s, sms);
+                default: break;
+            }
         }
         return launch_leaf_t<DT, RAW, 0, true>(P, s, sms);
     }

@@ -668,6 +668,27 @@ def test_compare_pair_tile_gather_path():
     assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stdout[-2000:] + r.stderr[-2000:]
 
 
+@pytest.mark.parametrize("chunk", [1024, 2048, 8192, 16384, 32768, 65536])
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+def test_compare_pair_specialised_chunk_sizes(dt, chunk):
+    """The fused pair kernels compiled for the configs[2] sweep's chunk sizes (every size of
+    512 B..64 KiB has its own instantiation): ragged arrays (partial last chunk and partial last
+    16-byte block), changes above and below eps, a flagged last chunk -- every node, the chunk
+    list and the element ids equal the oracle's."""
+    per = chunk // (4 if dt == torch.float32 else 8)
+    sizes = [37 * per + 3, 5 * per, 1, 2 * per + per // 2 + 1]
+    a = [_data(n, dt, 400 + i) for i, n in enumerate(sizes)]
+    b = [t.clone() for t in a]
+    b[0][per // 3::7 * per + 11] += 3e-6        # above eps = 1e-6
+    b[0][5::3 * per + 1] += 2e-7                # below eps: straddles only
+    b[1][-1] -= 1e-3
+    b[3][-1] += 1.0                             # the flagged ragged last chunk
+    pair = synth.Pair("specialised", a, b, chunk, 1e-6)
+    TA, TB, chunks, idx, counts = fused_compare(pair)
+    nc, nd = full_checkpoint_parity(pair, TA, TB, chunks, idx, counts, brute=True)
+    assert nc > 2 and nd > 2
+
+
 @pytest.mark.parametrize("dt,chunk", [(torch.float32, 2 << 20), (torch.float64, 4 << 20)])
 def test_compare_pair_large_chunks(dt, chunk):
     """Multi-MiB chunks (several mask groups per chunk, few long chains) through the fused call:

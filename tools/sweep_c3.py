@@ -31,10 +31,21 @@ def main():
     ap.add_argument("--n", type=int, default=1 << 29)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--hash-block", type=int, default=16)
+    ap.add_argument("--chunks", default="", help="comma-separated subset of the chunk sizes")
+    ap.add_argument("--eps", default="", help="comma-separated subset of the bounds")
+    ap.add_argument("--lib", default="", help="an A/B variant libckpt.so (tools/variant.py)")
     args = ap.parse_args()
     import torch
     import paper_conf_middleware_tanaabcrtn24_b200 as ck
     import synth
+    global CHUNKS, EPSS
+    if args.chunks:
+        CHUNKS = [int(x) for x in args.chunks.split(",")]
+    if args.eps:
+        EPSS = [float(x) for x in args.eps.split(",")]
+    if args.lib:
+        import ctypes
+        ck._lib = ck._declare(ctypes.CDLL(args.lib))
 
     peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] \
         if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
