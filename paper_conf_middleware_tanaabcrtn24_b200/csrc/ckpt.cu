@@ -1390,6 +1390,7 @@ extern "C" ckpt_status ckpt_compare(const void *const *a, const void *const *b, 
                                     uint64_t *n_diff, uint8_t *root_a16, uint8_t *root_b16,
                                     void *stream) {
     if (!n_chunks || !n_diff) return fail(CKPT_EINVAL, "NULL count output");
+    if (!a || !b || !n || n_arrays == 0) return fail(CKPT_EINVAL, "no arrays");
     cudaStream_t s = (cudaStream_t)stream;
     ckpt_tree *ta = nullptr, *tb = nullptr;
     uint64_t *dc = nullptr;

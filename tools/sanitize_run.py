@@ -80,4 +80,25 @@ TA, TB = ck.compare_pair_async([a7], [b7], 65536, 1e-6, ch, ix, cnt)
 TA.wait(); TB.wait()
 torch.cuda.synchronize()
 assert cnt.tolist() == [1, 1] and ix[0].item() == n7 - 1
+# the fused pair kernels specialised per chunk size (f64, 1 KiB and 16 KiB, ragged arrays)
+for C8 in (1024, 16384):
+    a8 = [synth.normal(30 + k, n, "cuda", dtype=torch.float64) for k, n in enumerate((3 * C8 // 8 + 3, 777))]
+    b8 = [t.clone() for t in a8]
+    b8[0][::97] += 1e-3
+    b8[1][-1] += 1.0
+    L8 = sum(-(-t.numel() * 8 // C8) for t in a8)
+    ch = torch.empty(L8, dtype=torch.int64, device="cuda")
+    ix = torch.empty(sum(t.numel() for t in a8), dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(a8, b8, C8, 1e-6, ch, ix, cnt)
+    TA.wait(); TB.wait()
+    torch.cuda.synchronize()
+    an8 = [t.cpu().numpy() for t in a8]
+    bn8 = [t.cpu().numpy() for t in b8]
+    A8 = oracle.build_checkpoint(an8, C8, 1e-6)
+    B8 = oracle.build_checkpoint(bn8, C8, 1e-6)
+    rc8 = oracle.diff_checkpoint(A8, B8)
+    ri8 = oracle.verify_checkpoint(an8, bn8, C8, rc8, 1e-6, A8)
+    nc, nd = cnt.tolist()
+    assert np.array_equal(ch[:nc].cpu().numpy(), rc8) and np.array_equal(ix[:nd].cpu().numpy(), ri8)
 print("sanitize workload ok", ck.launch_count(), "launches")
