@@ -59,6 +59,7 @@ SNAPSHOT = 9
 C4_RANKS = 64
 CFG = "c2"
 HASH_BLOCK = 16
+JSON_OUT = sys.stdout
 N_PARTICLES = CONFIGS[CFG]["n"]
 WORKLOAD = CONFIGS[CFG]["workload"]
 
@@ -246,7 +247,7 @@ def run_reference(args):
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    print(json.dumps(line), file=JSON_OUT, flush=True)
     return 0
 
 
@@ -288,7 +289,8 @@ def run_ours(args):
             v = torch.cuda.nccl.version()
             nccl_info = {"backend": "nccl", "version": ".".join(str(x) for x in v)
                          if isinstance(v, tuple) else str(v), "world": dist.get_world_size(),
-                         "exchange": "one all_gather_into_tensor per step (C1 roots + C2 counts)"}
+                         "exchange": "one all_gather_into_tensor per step (C1 roots + C2 counts), on its "
+                                     "own stream beside the next step's leaf kernel"}
         else:
             dist.init_process_group(backend)
             nccl_info = {"backend": backend, "world": dist.get_world_size()}
@@ -324,33 +326,64 @@ def run_ours(args):
         del ta0
         host_a = [x.cpu().pin_memory() for x in A]
 
+    # N > 1: the C1/C2 exchange of step i runs on its own stream X while step i+1's leaf kernel
+    # runs on the compute stream (its kernels take the SM slots that free up in that kernel's
+    # tail; the NCCL transfer needs no SM of the compute stream).  Step i writes its counts to
+    # cnt2[i % 2]; before step i+2 overwrites them, the compute stream waits for exchange i.
+    xs = torch.cuda.Stream() if collect else None
+    cnt2 = [torch.zeros(2, dtype=torch.int64, device="cuda") for _ in range(2)] if collect else None
+    x_done = [None, None]
+    step_no = [0]
+    exch = []        # the last two exchanges' outputs (kept until their stream work is done)
+
+    def exchange(TA, TB, cnt):
+        # C1 + C2 in ONE collective: every rank contributes [A roots | B roots | counts]
+        # (2*n_arrays*16 + 16 bytes); the counts are summed locally and both top trees are
+        # built by one levels launch
+        TA.array_roots(out=send[:n_arrays], stream=xs)
+        TB.array_roots(out=send[n_arrays:2 * n_arrays], stream=xs)
+        send[2 * n_arrays].view(torch.int64).copy_(cnt)
+        dist.all_gather_into_tensor(recv.view(-1), send.view(-1))
+        roots = recv[:, :2 * n_arrays].reshape(world, 2, n_arrays, 16).transpose(0, 1)
+        tops = ck.tree_from_digests_batch(roots.reshape(2 * world * n_arrays, 16),
+                                          [world * n_arrays, world * n_arrays], stream=xs)
+        tot = recv[:, 2 * n_arrays].view(torch.int64).sum(0)
+        return [TA, TB, *tops, tot]
+
     def step():
+        i = step_no[0]
+        step_no[0] += 1
+        cnt = cnt2[i % 2] if collect else counts
+        cur = torch.cuda.current_stream()
+        if collect and x_done[i % 2] is not None:
+            cur.wait_event(x_done[i % 2])          # exchange i-2 has read cnt2[i % 2]
         if args.path == "saved":
-            TA, TB = ck.compare_saved(saved_a, host_a, B, chunks, idx, counts)
+            TA, TB = ck.compare_saved(saved_a, host_a, B, chunks, idx, cnt)
         elif args.path == "fused":
             # one leaf launch hashes both runs, compares the digests and marks the flagged chunks
-            TA, TB = ck.compare_pair_async(A, B, CHUNK, EPS, chunks, idx, counts,
+            TA, TB = ck.compare_pair_async(A, B, CHUNK, EPS, chunks, idx, cnt,
                                            hash_block=args.hash_block)
         else:
             TA, TB = ck.tree_build_batch([A, B], CHUNK, EPS, hash_block=args.hash_block)
-            ck.diff_verify_async(TA, TB, A, B, chunks, idx, counts)   # BFS diff, then verify
+            ck.diff_verify_async(TA, TB, A, B, chunks, idx, cnt)   # BFS diff, then verify
         if collect:
-            # C1 + C2 in ONE collective: every rank contributes [A roots | B roots | counts]
-            # (2*n_arrays*16 + 16 bytes); the counts are summed locally and both top trees
-            # are built by one levels launch
-            TA.array_roots(out=send[:n_arrays])
-            TB.array_roots(out=send[n_arrays:2 * n_arrays])
-            send[2 * n_arrays].view(torch.int64).copy_(counts)
-            dist.all_gather_into_tensor(recv.view(-1), send.view(-1))
-            roots = recv[:, :2 * n_arrays].reshape(world, 2, n_arrays, 16).transpose(0, 1)
-            tops = ck.tree_from_digests_batch(roots.reshape(2 * world * n_arrays, 16),
-                                              [world * n_arrays, world * n_arrays])
-            tot = recv[:, 2 * n_arrays].contiguous().view(torch.int64).view(world, 2).sum(0)
-            keep[:] = [TA, TB, *tops, tot]
+            xs.wait_stream(cur)                    # after this step's verify
+            with torch.cuda.stream(xs):
+                exch.append(exchange(TA, TB, cnt))
+                ev = torch.cuda.Event()
+                ev.record(xs)
+            x_done[i % 2] = ev
+            del exch[:-2]
+            keep[:] = [TA, TB]
         else:
             keep[:] = [TA, TB]
         TA.wait()          # the step ends when both trees are complete (K2 runs on a side stream)
         TB.wait()
+
+    def join():
+        # the timed region ends when every step's exchange has completed
+        if collect:
+            torch.cuda.current_stream().wait_stream(xs)
 
     # configs[3] as written (--snapshots all): the 10 intermediate snapshots, one at a time
     # (each generated into HBM before its timed region), every snapshot's trees kept; the
@@ -372,7 +405,13 @@ def run_ours(args):
         for _ in range(max(3, args.warmup)):
             step()
         torch.cuda.synchronize()
-        local_counts = counts.cpu().tolist()
+        join()
+        torch.cuda.synchronize()
+        local_counts = (cnt2[(step_no[0] - 1) % 2] if collect else counts).cpu().tolist()
+        if collect:   # the exchange's global counts equal an all-reduce of the local ones
+            chk = torch.tensor(local_counts, dtype=torch.int64, device="cuda")
+            dist.all_reduce(chk)
+            assert exch[-1][-1].tolist() == chk.tolist(), (exch[-1][-1].tolist(), chk.tolist())
         # timed region: no events between the kernels (an event after the leaf kernel would end
         # the programmatic-launch overlap of the next kernel with its tail); the leaf kernel's
         # own duration is timed in a separate pass below
@@ -386,6 +425,7 @@ def run_ours(args):
         h0 = time.perf_counter()
         for _ in range(args.steps):
             step()
+        join()
         host_ms += (time.perf_counter() - h0) * 1e3 / args.steps   # enqueue time per step (host)
         e1.record()
         torch.cuda.synchronize()
@@ -401,6 +441,7 @@ def run_ours(args):
         ck.profile_enable(["leaf"])
         for _ in range(args.steps):
             step()
+        join()
         torch.cuda.synchronize()
         ck.profile_enable(False)
         lm, ln = ck.profile_read("leaf")
@@ -422,6 +463,7 @@ def run_ours(args):
     ck.profile_enable(True)
     for _ in range(k_prof):
         step()
+    join()
     torch.cuda.synchronize()
     ck.profile_enable(False)
     phases = {"steps": k_prof}
@@ -580,7 +622,7 @@ def run_ours(args):
                 "what": "one step = the 10-snapshot sequence; per-snapshot device ms summed, every "
                         "snapshot's trees kept", "per_snapshot": per_snap,
                 "trees_kept": 2 * len(kept_trees)}
-        print(json.dumps(line), flush=True)
+        print(json.dumps(line), file=JSON_OUT, flush=True)
     if collect:
         dist.destroy_process_group()
     return 0
@@ -640,6 +682,12 @@ def main():
         WORKLOAD = f"REDUCED ({args.elems} elements per array, not a bench line): " + WORKLOAD
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         return spawn_ranks(args.gpus)
+    # stdout carries only the JSON line: whatever native code prints (e.g. NCCL's version banner)
+    # goes to stderr
+    global JSON_OUT
+    JSON_OUT = os.fdopen(os.dup(1), "w")
+    sys.stdout.flush()
+    os.dup2(2, 1)
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

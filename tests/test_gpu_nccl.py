@@ -85,13 +85,30 @@ def test_bench_runs_n_nccl_ranks(world):
             "--no-e2e", "--no-cpu", "--elems", str(1 << 20), "--collectives"]
     r = _torchrun(world, args)
     assert r.returncode == 0, r.stderr[-4000:]
-    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
-    assert len(lines) == 1, r.stdout
+    lines = [ln for ln in r.stdout.splitlines() if ln.strip()]
+    assert len(lines) == 1 and lines[0].startswith("{"), r.stdout    # stdout = the JSON line only
     line = json.loads(lines[0])
     assert line["n_gpus"] == world
     assert line["dist"]["backend"] == "nccl" and line["dist"]["world"] == world
     assert line["value"] > 0 and line["gpu_launches"] > 0
     assert "NCCL INFO" in r.stderr
+
+
+def test_bench_two_gloo_ranks_on_one_gpu():
+    """The N > 1 bench step's logic with two ranks sharing the GPU over gloo (a functional test:
+    timings are meaningless): the exchange of step i runs on its own stream beside step i+1, and
+    bench.py asserts that the exchanged global counts equal an all-reduce of the local ones."""
+    args = [os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "4", "--warmup", "3",
+            "--no-e2e", "--no-cpu", "--elems", str(1 << 20)]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), *args]
+    env = dict(os.environ, CKPT_DIST_BACKEND="gloo")
+    r = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-4000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.strip()]
+    assert len(lines) == 1, r.stdout
+    line = json.loads(lines[0])
+    assert line["n_gpus"] == 2 and line["dist"]["backend"] == "gloo" and line["value"] > 0
 
 
 def test_bench_spawns_ranks_itself_when_not_launched():
