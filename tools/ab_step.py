@@ -19,6 +19,8 @@ ap.add_argument("--lib", default="")
 ap.add_argument("--config", default="c2")
 ap.add_argument("--steps", type=int, default=20)
 ap.add_argument("--reps", type=int, default=3)
+ap.add_argument("--join", default="step", choices=["step", "end"],
+                help="step: every step waits for both trees' levels (bench.py); end: only the last")
 args = ap.parse_args()
 if args.lib:
     ck._lib = ck._declare(ctypes.CDLL(args.lib))
@@ -32,10 +34,11 @@ idx = torch.empty(sum(t.numel() for t in A), dtype=torch.int64, device="cuda")
 cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
 
 
-def step():
+def step(last=True):
     TA, TB = ck.compare_pair_async(A, B, C, eps, chunks, idx, cnt)
-    TA.wait()
-    TB.wait()
+    if last or args.join == "step":
+        TA.wait()
+        TB.wait()
     return TA, TB
 
 
@@ -46,10 +49,14 @@ best = 1e9
 for _ in range(args.reps):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
-    for _ in range(args.steps):
-        keep = step()
+    kept = []
+    for k in range(args.steps):
+        kept.append(step(k == args.steps - 1))
+    for TA, TB in kept:
+        TA.wait()
+        TB.wait()
     e1.record()
     torch.cuda.synchronize()
     best = min(best, e0.elapsed_time(e1) / args.steps)
 print(f"{args.config} {os.path.basename(os.path.dirname(args.lib)) if args.lib else 'product'}: "
-      f"{best:.4f} ms/step, counts {cnt.tolist()}", flush=True)
+      f"join={args.join} {best:.4f} ms/step, counts {cnt.tolist()}", flush=True)
