@@ -111,6 +111,38 @@ def test_bench_two_gloo_ranks_on_one_gpu():
     assert line["n_gpus"] == 2 and line["dist"]["backend"] == "gloo" and line["value"] > 0
 
 
+def test_bench_json_contract():
+    """python bench.py at N = 1 (reduced size): stdout is exactly one JSON line carrying every key
+    of the bench contract -- metric/value/unit, roofline (bound, achieved, peak, frac, traffic),
+    cpu_baseline (the oracle at all cores and one thread), e2e with its copied bytes, clocks and
+    the launch count -- with self-consistent numbers."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--steps", "3", "--warmup", "3",
+                        "--elems", str(1 << 20)], cwd=ROOT, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-4000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.strip()]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+              "scaling", "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e",
+              "clocks", "gpu_launches"):
+        assert k in d, k
+    assert d["n_gpus"] == 1 and d["steps"] == 3 and d["warmup"] >= 3 and d["higher_is_better"] is True
+    cfg = d["config"]
+    # value = pair bytes per step / step time
+    assert abs(d["value"] - cfg["bytes_per_step_per_gpu"] / (d["ms_per_step"] / 1e3) / 1e9) < 0.01 * d["value"]
+    rf = d["roofline"]
+    assert rf["bound"] == "hbm" and rf["unit"] == "GB/s" and rf["peak"] > 0
+    assert abs(rf["frac"] - rf["achieved"] / rf["peak"]) < 1e-3
+    cpu = d["cpu_baseline"]
+    assert cpu["kind"] == "oracle" and cpu["cores"] >= 1 and cpu["value"] > 0
+    assert cpu["single_thread"]["cores"] == 1
+    e2e = d["e2e"]
+    assert e2e["value"] > 0 and e2e["h2d_bytes_per_step"] == cfg["bytes_per_step_per_gpu"]
+    assert e2e["d2h_bytes_per_step"] > 0
+    assert {"sm_mhz", "sm_max_mhz", "reasons"} <= set(d["clocks"])
+    assert d["gpu_launches"] >= 3 * d["steps"]
+
+
 def test_bench_spawns_ranks_itself_when_not_launched():
     """python bench.py --gpus N (no launcher) re-executes itself as N ranks."""
     n = torch.cuda.device_count()
