@@ -112,3 +112,54 @@ def test_fuzz_unfused_calls_match_oracle(seed):
     assert nc == rc.size and np.array_equal(chunks[:nc].cpu().numpy(), rc), (dt, chunk, eps, hb)
     assert nd == ri.size and np.array_equal(idx[:nd].cpu().numpy(), ri), (dt, chunk, eps, hb)
     _check_trees(TA, TB, A, B)
+
+
+@pytest.mark.parametrize("seed", range(300, 340))
+def test_fuzz_stream_host_and_saved_paths_match_oracle(seed):
+    """The same random pairs through the host-data paths: streamed through the device ring with
+    a random (chunk-aligned) segment size, staged, and compared against a stored tree of run A."""
+    dt, chunk, eps, hb, a_list, b_list = _case(seed)
+    A, B, rc, ri = _oracle(a_list, b_list, chunk, eps, hb)
+    rng = np.random.default_rng(seed)
+    ha = [torch.from_numpy(x).pin_memory() for x in a_list]
+    hb_ = [torch.from_numpy(x).pin_memory() for x in b_list]
+    seg = int(chunk * rng.integers(1, 9))
+    c_s, i_s, nc, nd, root_a, root_b = ck.compare_stream(ha, hb_, chunk, eps, segment_bytes=seg,
+                                                          hash_block=hb)
+    assert nc == rc.size and np.array_equal(c_s[:nc].numpy(), rc), (dt, chunk, eps, hb, seg)
+    assert nd == ri.size and np.array_equal(i_s[:nd].numpy(), ri), (dt, chunk, eps, hb, seg)
+    assert root_a == A.root and root_b == B.root
+    if hb == 16:                       # compare_host and compare_saved use the default blocks
+        i_h, nc_h, nd_h, ra, rb = ck.compare_host(ha, hb_, chunk, eps)
+        assert (nc_h, nd_h) == (rc.size, ri.size) and np.array_equal(i_h[:nd_h].numpy(), ri)
+        assert ra == A.root and rb == B.root
+        ta0 = ck.tree_build([torch.from_numpy(x).cuda() for x in a_list], chunk, eps)
+        blob = ta0.serialize()
+        tb = [torch.from_numpy(x).cuda() for x in b_list]
+        chunks = torch.empty(max(sum(A.n_leaves), 1), dtype=torch.int64, device="cuda")
+        idx = torch.empty(max(sum(x.size for x in a_list), 1), dtype=torch.int64, device="cuda")
+        counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+        TA, TB = ck.compare_saved(blob, ha, tb, chunks, idx, counts)
+        torch.cuda.synchronize()
+        n1, n2 = counts.tolist()
+        assert n1 == rc.size and np.array_equal(chunks[:n1].cpu().numpy(), rc)
+        assert n2 == ri.size and np.array_equal(idx[:n2].cpu().numpy(), ri)
+        assert TA.root() == A.root and TB.root() == B.root
+
+
+@pytest.mark.parametrize("seed", range(400, 430))
+def test_fuzz_mid_level_bfs_matches_oracle(seed):
+    """The BFS diff from a random start level (threshold T) equals the oracle's chunk list."""
+    dt, chunk, eps, hb, a_list, b_list = _case(seed)
+    A, B, rc, _ = _oracle(a_list, b_list, chunk, eps, hb)
+    rng = np.random.default_rng(seed)
+    ta = [torch.from_numpy(x).cuda() for x in a_list]
+    tb = [torch.from_numpy(x).cuda() for x in b_list]
+    TA, TB = ck.tree_build_batch([ta, tb], chunk, eps, hash_block=hb)
+    chunks = torch.empty(max(sum(A.n_leaves), 1), dtype=torch.int64, device="cuda")
+    count = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for T in (1, int(rng.integers(2, 64)), int(rng.integers(64, 1 << 16))):
+        ck.tree_diff_async(TA, TB, chunks, count, T=T)
+        torch.cuda.synchronize()
+        n = int(count.item())
+        assert n == rc.size and np.array_equal(chunks[:n].cpu().numpy(), rc), (T, dt, chunk)
