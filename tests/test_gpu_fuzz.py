@@ -18,7 +18,7 @@ ck = pytest.importorskip("paper_conf_middleware_tanaabcrtn24_b200")
 SPECIALISED = [512, 1024, 2048, 4096, 8192, 16384, 32768, 65536]
 
 
-def _case(seed):
+def _case(seed, arrays=(1, 5)):
     rng = np.random.default_rng(1000 + seed)
     dt = np.float32 if rng.random() < 0.6 else np.float64
     esz = np.dtype(dt).itemsize
@@ -31,7 +31,7 @@ def _case(seed):
     hb = 16 if rng.random() < 0.7 else int(rng.choice([0, 32, 48, 64, 256]))
     if hb and hb > chunk:
         hb = 0
-    m = int(rng.integers(1, 5))
+    m = int(rng.integers(*arrays))
     per = chunk // esz
     a_list, b_list = [], []
     for k in range(m):
@@ -163,3 +163,23 @@ def test_fuzz_mid_level_bfs_matches_oracle(seed):
         torch.cuda.synchronize()
         n = int(count.item())
         assert n == rc.size and np.array_equal(chunks[:n].cpu().numpy(), rc), (T, dt, chunk)
+
+
+@pytest.mark.parametrize("seed", range(500, 516))
+def test_fuzz_many_arrays_device_tables(seed):
+    """17-80 arrays per checkpoint: the leaf, levels and verify kernels read their array tables
+    from device memory instead of the kernel parameters."""
+    dt, chunk, eps, hb, a_list, b_list = _case(seed, arrays=(17, 81))
+    A, B, rc, ri = _oracle(a_list, b_list, chunk, eps, hb)
+    ta = [torch.from_numpy(x).cuda() for x in a_list]
+    tb = [torch.from_numpy(x).cuda() for x in b_list]
+    chunks = torch.empty(max(sum(A.n_leaves), 1), dtype=torch.int64, device="cuda")
+    idx = torch.empty(max(sum(x.size for x in a_list), 1), dtype=torch.int64, device="cuda")
+    counts = torch.zeros(2, dtype=torch.int64, device="cuda")
+    TA, TB = ck.compare_pair_async(ta, tb, chunk, eps, chunks, idx, counts, hash_block=hb)
+    TA.wait(); TB.wait()
+    torch.cuda.synchronize()
+    nc, nd = counts.tolist()
+    assert nc == rc.size and np.array_equal(chunks[:nc].cpu().numpy(), rc), (len(a_list), chunk)
+    assert nd == ri.size and np.array_equal(idx[:nd].cpu().numpy(), ri), (len(a_list), chunk)
+    _check_trees(TA, TB, A, B)
